@@ -1,0 +1,352 @@
+#!/usr/bin/env python
+"""Benchmark: FP64 Cholesky GFLOP/s (n^3/3) of the STF tiled factorisation.
+
+Contract (driver): `python bench.py --gpus N --steps K --warmup W` prints ONE
+JSON line on rank 0.  Under torchrun (N > 1) every rank joins the barriers; the
+library is single-process multi-GPU by design (north_star's
+`stf_potrf(..., ngpus)`), so rank 0 drives all N GPUs and the other ranks
+contribute 0 device time to the max-over-ranks.
+
+One step = one synchronous stf_potrf of the whole matrix (every §8(a) row: DAG,
+placement, replica pushes, POTRF/TRSM/SYRK/GEMM kernels, completion) on
+device-resident 2D-block-cyclic tiles (TILED_2DBC).  The
+matrix is regenerated on the device before every step (untimed); it is 4.4 GB
+of tiles at the default n = 32768, far larger than the 126 MB L2.
+`value` = n^3/3 * steps / sum(device time), device time measured with CUDA
+events on the library's launch stream around the graph launch.
+
+`--impl reference` times the CPU oracle (the slow plain Cholesky, as it stands)
+on a bounded sample of the same workload: the leading n' x n' principal block of
+the same matrix (its factor is the leading block of L), n' sized so the whole
+run ends within a few minutes.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "FP64 Cholesky GFLOP/s (n³/3) at 1/2/4/8 B200; fraction of FP64 tensor peak"
+UNIT = "GFLOP/s"
+# FP64 DMMA peak measured on this pool's B200 (tools/calib_fp64.cu -> profiles/calib_fp64_r01.json):
+# 64 FMA/clk/SM x 148 SMs x 1965 MHz, clocks held at max under FP64 load.
+FP64_PEAK_TFLOPS = 37.09
+FP64_PEAK_SRC = "measured DMMA peak, profiles/calib_fp64_r01.json (MEASURED_PEAKS.json has no FP64 entry)"
+
+GRIDS = {1: (1, 1), 2: (1, 2), 4: (2, 2), 8: (2, 4)}
+
+
+def grid_for(n):
+    if n in GRIDS:
+        return GRIDS[n]
+    p = max(d for d in range(1, int(math.isqrt(n)) + 1) if n % d == 0)
+    return p, n // p
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "--query-gpu=" + self.FIELDS, "--format=csv,noheader,nounits",
+                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = []
+        for ln in open(self.f.name):
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append((int(parts[0]), float(parts[1]), float(parts[2]), float(parts[3]), parts[5:9]))
+            except ValueError:
+                continue
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        pmax = max(r[3] for r in rows)
+        load = [r for r in rows if r[3] >= 0.5 * pmax] or rows
+        sm = sorted(r[1] for r in load)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in load for k in range(4) if r[4][k].lower().startswith("active")})
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": max(r[2] for r in rows), "reasons": reasons,
+                "samples_under_load": len(load), "power_w_max": pmax}
+
+
+# ------------------------------------------------------------------ oracle (cpu_baseline / reference arm)
+def oracle_sample(n, seed, target_s, cap_n=None):
+    """Time the oracle on the leading n' x n' block of the order-n metric matrix,
+    n' chosen from a small calibration run so one sample takes ~target_s."""
+    import oracle
+    import synth
+
+    cal = 1536
+    A = synth.spd_block(seed, n, 0, 0, cal, cal)
+    oracle.potrf(A)  # builds/loads liboracle.so
+    t0 = time.perf_counter()
+    oracle.potrf(A)
+    tc = time.perf_counter() - t0
+    m = int(cal * (target_s / max(tc, 1e-3)) ** (1.0 / 3.0))
+    m = max(cal, min(m, cap_n or n, 16384))
+    m -= m % 64
+    A = synth.spd_block(seed, n, 0, 0, m, m)
+    t0 = time.perf_counter()
+    _, info = oracle.potrf(A)
+    dt = time.perf_counter() - t0
+    assert info == 0
+    return m, dt, oracle.max_threads()
+
+
+def reference_arm(args, rank, world):
+    if rank != 0:
+        return 0
+    n, nb = args.n, args.nb
+    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    m, _, cores = oracle_sample(n, 1, per_step)
+    import oracle
+    import synth
+
+    A = synth.spd_block(1, n, 0, 0, m, m)
+    for _ in range(args.warmup):
+        oracle.potrf(A)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        _, info = oracle.potrf(A)
+        ts.append(time.perf_counter() - t0)
+        assert info == 0
+    tot = sum(ts)
+    value = m ** 3 / 3 * len(ts) / tot / 1e9
+    sample = ("leading %dx%d principal block of the seed-1 n=%d metric matrix per step "
+              "(its factor is the leading block of L); plain unblocked Cholesky-Crout, OpenMP" % (m, m, n))
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1000 * tot / len(ts), 3),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": "n=%d nb=%d FP64 SPD (seeded, diagonally dominant), configs[2]" % (n, nb),
+                   "n": n, "nb": nb, "grid": "%dx%d" % grid_for(args.gpus), "sample_n": m, "l2": "n/a (CPU)"},
+        "cpu_baseline": {"value": round(value, 4), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(value, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def run_ours(args, rank, world):
+    import torch
+    import torch.distributed as dist
+
+    dist_on = world > 1
+    if dist_on:
+        dist.init_process_group("nccl" if torch.cuda.is_available() else "gloo")
+        torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+    N = args.gpus
+    n, nb = args.n, args.nb
+    P, Q = grid_for(N)
+    result = None
+    total_ms = 0.0
+    if rank == 0:
+        import paper_conf_sc_augonnetasg24_b200 as stf
+
+        devices = list(range(N)) if args.virtual == 0 else [0] * N
+        stf.init(N, devices)
+        M = stf.TiledMatrix(n, nb, P, Q, devices=devices)
+        first_ms = None
+        for w in range(args.warmup):
+            M.fill_spd(1)
+            t0 = time.perf_counter()
+            assert M.potrf() == 0
+            if w == 0:
+                first_ms = 1000 * (time.perf_counter() - t0)
+        for d in set(devices):
+            torch.cuda.synchronize(d)
+    if dist_on:
+        dist.barrier()
+    clocks = ClockSampler()
+    steps_ms = []
+    stats = None
+    if rank == 0:
+        clocks.start()
+        for _ in range(args.steps):
+            M.fill_spd(1)  # untimed regeneration (input is overwritten by L)
+            for d in set(devices):
+                torch.cuda.synchronize(d)
+            info = M.potrf()
+            assert info == 0, info
+            stats = stf.last_stats()
+            steps_ms.append(stats["device_ms"])
+        for d in set(devices):
+            torch.cuda.synchronize(d)
+        clk = clocks.stop()
+        total_ms = sum(steps_ms)
+    if dist_on:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+        dist.barrier()
+    if rank != 0:
+        if dist_on:
+            dist.destroy_process_group()
+        return 0
+
+    flops = n ** 3 / 3.0
+    value = flops * args.steps / (total_ms * 1e-3) / 1e9
+    ms_per_step = total_ms / args.steps
+
+    # ---- e2e: same metric through the C ABI with HOST buffers (pinned), copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        e2e = e2e_run(stf, n, nb, N, args)
+
+    # ---- roofline: the factorisation is one graph launch on the library's launch stream
+    achieved_tf = value / 1e3
+    roof = {"bound": "tensor", "achieved": round(achieved_tf, 3), "peak": FP64_PEAK_TFLOPS * N, "unit": "TFLOP/s",
+            "frac": round(achieved_tf / (FP64_PEAK_TFLOPS * N), 4), "traffic": None,
+            "kernel": "whole-DAG CUDA graph launch (n^3/3 flop per launch, %d kernels inside)" % stats["kernel_launches"],
+            "peak_src": FP64_PEAK_SRC}
+    # dominant kernel (GEMM tile update) timed alone on its own stream at this nb and at full occupancy
+    from paper_conf_sc_augonnetasg24_b200 import _abi
+    import ctypes
+
+    kern = {}
+    for name, kind, M_, N_, K_ in (("gemm_tile", 0, nb, nb, nb), ("gemm_full", 0, 8 * nb, 8 * nb, nb),
+                                   ("syrk_tile", 1, nb, nb, nb), ("trsm_tile", 2, nb, nb, 0),
+                                   ("potrf_tile", 3, nb, nb, nb)):
+        ms = ctypes.c_double()
+        torch.cuda.set_device(0)
+        rc = _abi.stf_bench_kernel(kind, M_, N_, K_, 10, ctypes.byref(ms))
+        if rc == 0:
+            fl = {0: 2.0 * M_ * N_ * K_, 1: 1.0 * M_ * M_ * K_, 2: 1.0 * M_ * N_ * N_, 3: M_ ** 3 / 3.0}[kind]
+            kern[name] = {"ms": round(ms.value, 4), "tflops": round(fl / (ms.value * 1e-3) / 1e12, 3),
+                          "frac": round(fl / (ms.value * 1e-3) / 1e12 / FP64_PEAK_TFLOPS, 4),
+                          "shape": [M_, N_, K_ if kind in (0, 1) else None]}
+    roof["kernels_alone"] = kern
+    traffic = load_traffic()
+    if traffic is not None:
+        roof["traffic"] = traffic
+
+    cpu = None
+    if N == 1 and not args.no_cpu:
+        m, dt, cores = oracle_sample(n, 1, args.cpu_seconds)
+        cpu = {"value": round(m ** 3 / 3 / dt / 1e9, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": "leading %dx%d principal block of the same seed-1 n=%d matrix (its factor is the "
+                         "leading block of L), %.1f s" % (m, m, n, dt)}
+
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": N, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": "n=%d nb=%d FP64 SPD (seeded, diagonally dominant), configs[2]" % (n, nb),
+                   "n": n, "nb": nb, "grid": "%dx%d" % (P, Q), "descriptor": "TILED_2DBC (device-resident tiles)",
+                   "l2": "inputs larger than L2 (%.1f GB of tiles) and regenerated before every step" %
+                         (n // nb * (n // nb + 1) / 2 * nb * nb * 8 / 1e9),
+                   "graph": stf.get_option("graph"), "streams": stf.get_option("streams"),
+                   "virtual_slots": bool(args.virtual)},
+        "gpu_launches": int(stats["kernel_launches"]) * args.steps,
+        "clocks": clk,
+        "roofline": roof,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "plan": {k: stats[k] for k in ("tasks", "transfers", "edges", "critical_path", "graph_nodes", "kernel_launches")},
+        "first_call_ms": round(first_ms, 1) if first_ms else None,
+        "step_ms": [round(x, 3) for x in steps_ms],
+    }
+    print(json.dumps(line), flush=True)
+    stf.finalize()
+    if dist_on:
+        dist.destroy_process_group()
+    return 0
+
+
+def e2e_run(stf, n, nb, N, args):
+    """stf_potrf on a pinned HOST column-major matrix: lower tiles H2D, factor,
+    lower tiles D2H, all tasks of one timed call.  Regeneration is untimed."""
+    import torch
+
+    T = n // nb
+    A_host = torch.empty((n, n), dtype=torch.float64, pin_memory=True)  # row-major storage = col-major A^T = A
+    dev = torch.empty((n, n), dtype=torch.float64, device="cuda:0")
+    from paper_conf_sc_augonnetasg24_b200 import _abi
+
+    def regen():
+        rc = _abi.stf_fill_spd_block(dev.data_ptr(), n, n, 0, 0, n, n, 1)
+        assert rc == 0
+        A_host.copy_(dev)
+        torch.cuda.synchronize()
+
+    times = []
+    for it in range(args.e2e_steps + 1):
+        regen()
+        t0 = time.perf_counter()
+        info = stf.potrf_colmajor(A_host.data_ptr(), n, n, nb, "L", None, N)
+        wall = time.perf_counter() - t0
+        assert info == 0
+        if it > 0:
+            times.append((stf.last_stats()["device_ms"], wall * 1e3))
+    del dev
+    tile_bytes = T * (T + 1) // 2 * nb * nb * 8
+    dev_ms = sum(t[0] for t in times) / len(times)
+    wall_ms = sum(t[1] for t in times) / len(times)
+    return {"value": round(n ** 3 / 3 / (dev_ms * 1e-3) / 1e9, 3), "unit": UNIT,
+            "h2d_bytes_per_step": tile_bytes, "d2h_bytes_per_step": tile_bytes,
+            "ms_per_step": round(dev_ms, 3), "host_wall_ms_per_step": round(wall_ms, 3),
+            "api": "stf_potrf(STF_DESC_HOST_COLMAJOR, pinned), lower tiles copied in and written back as tasks",
+            "steps": len(times)}
+
+
+def load_traffic():
+    """dram bytes per GEMM launch from the committed ncu --set full summary, if present."""
+    p = os.path.join(ROOT, "profiles", "gemm_traffic.json")
+    try:
+        return json.load(open(p)).get("traffic_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=32768)
+    ap.add_argument("--nb", type=int, default=1024)
+    ap.add_argument("--virtual", type=int, default=0, help="map all slots onto cuda:0")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    args = ap.parse_args()
+    assert args.warmup >= 1
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.impl == "reference":
+        return reference_arm(args, rank, world)
+    return run_ours(args, rank, world)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

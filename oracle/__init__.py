@@ -20,6 +20,8 @@ Functions and the passages they follow:
   modifies one of its data, and, when it modifies a datum, on every earlier
   reader of it.  Pinned by the worked example of Algorithm 1 / Fig. 1
   (PAPER.md:31-40, :50; tests/golden/alg1_dag.txt).
+* :func:`tile_gemm`, :func:`tile_syrk`, :func:`tile_trsm` -- the tile tasks
+  of PAPER.md:393 written as their definitions (numpy matmul as a step).
 * :func:`tiled_potrf` -- executes :func:`cholesky_tasks` in a topological
   order of :func:`stf_edges` with numpy tile operations (definition of each
   tile task), proving the task list + rule compute the same L as
@@ -146,11 +148,34 @@ def transitive_closure(n: int, edges) -> np.ndarray:
 # --------------------------------------------------------------------------
 # Tiled execution of the task list (numpy tile ops, one definition per task)
 # --------------------------------------------------------------------------
+def tile_gemm(C: np.ndarray, A: np.ndarray, B: np.ndarray) -> np.ndarray:
+    """GEMM tile task: C - A B^T (numpy matmul as a library step)."""
+    return C - A @ B.T
+
+
+def tile_syrk(C: np.ndarray, A: np.ndarray) -> np.ndarray:
+    """SYRK tile task: lower triangle of C - A A^T; strictly upper of C kept."""
+    return np.tril(C - A @ A.T) + np.triu(C, 1)
+
+
+def tile_trsm(B: np.ndarray, L: np.ndarray) -> np.ndarray:
+    """TRSM tile task: X with X L^T = B, L lower (only its lower
+    triangle is read); column-by-column forward substitution in plain numpy:
+    x_c = (b_c - sum_{p<c} x_p L_cp) / L_cc."""
+    L = np.tril(L)
+    X = np.array(B, dtype=np.float64)
+    for c in range(L.shape[0]):
+        if c:
+            X[:, c] -= X[:, :c] @ L[c, :c]
+        X[:, c] /= L[c, c]
+    return X
+
+
 def tiled_potrf(A: np.ndarray, nb: int) -> Tuple[np.ndarray, int]:
     """Run cholesky_tasks(T) in program order (a valid topological order of the
     STF DAG) on nb x nb tiles with the textbook tile operations of PAPER.md:393:
         POTRF: A_kk <- chol(A_kk) via :func:`potrf` on the tile
-        TRSM:  A_ik <- A_ik L_kk^-T     (numpy.linalg.solve of L_kk X^T = A_ik^T)
+        TRSM:  A_ik <- A_ik L_kk^-T     (forward substitution, tile_trsm)
         SYRK:  A_ii <- A_ii - L_ik L_ik^T
         GEMM:  A_ij <- A_ij - L_ik L_jk^T
     Used only to pin that the task list computes the same factor as potrf().
@@ -170,10 +195,9 @@ def tiled_potrf(A: np.ndarray, nb: int) -> Tuple[np.ndarray, int]:
                 return np.tril(A), k * nb + info
             tile(k, k)[:, :] = Lkk
         elif kind == "TRSM":
-            Lkk = np.tril(tile(k, k))
-            tile(i, k)[:, :] = np.linalg.solve(Lkk, tile(i, k).T).T
+            tile(i, k)[:, :] = tile_trsm(tile(i, k), tile(k, k))
         elif kind == "SYRK":
-            tile(i, i)[:, :] -= tile(i, k) @ tile(i, k).T
+            tile(i, i)[:, :] = tile_syrk(tile(i, i), tile(i, k))
         else:
-            tile(i, j)[:, :] -= tile(i, k) @ tile(j, k).T
+            tile(i, j)[:, :] = tile_gemm(tile(i, j), tile(i, k), tile(j, k))
     return np.tril(A), 0

@@ -1,0 +1,248 @@
+// K1 / K2: FP64 tile update C -= A * B^T on the sm_100a FP64 tensor pipe (DMMA),
+// operands staged by TMA into 128B-swizzled shared memory through an mbarrier
+// pipeline (north_star "SYRK/GEMM trailing updates as FP64
+// tensor-core (DMMA) contractions fed by TMA into shared memory").
+//
+// Tile task definitions ("calling cuBLAS ... kernels within tasks",
+// right-looking tiled Cholesky of ref. [17] PAPER.md:495):
+//   GEMM(i,j,k):  A_ij <- A_ij - L_ik * L_jk^T
+//   SYRK(i,k):    A_ii <- A_ii - L_ik * L_ik^T   (lower triangle only)
+//
+// B200 facts shaping the design (profiles/calib_fp64_r01.json):
+//   * tcgen05 has no f64 kind; FP64 tensor math is warp-level mma.sync -> DMMA.8x8x4,
+//     peak 64 FMA/clk/SM = 37.1 TFLOP/s measured (148 SMs, 1965 MHz held under load).
+//   * DMMA accumulates in registers, so the design is the classic register-tiled
+//     warp GEMM fed by a TMA/mbarrier producer warp.
+//
+// CTA tile 128 x 128 x 16, 4 stages (128 KB smem), 8 warps (warp tile 64 x 32 ->
+// 64 FP64 accumulators / thread); thread 0 doubles as the TMA producer.
+// Shared-memory layout of one operand stage: 8 boxes of [16 k-rows][16 m] doubles,
+// each k-row 128 B with the 128B swizzle (16-byte chunk c stored at c ^ (row & 7)).
+// Fragment k-permutation: within a k8 group the DMMA with kh in {0,1} takes
+// k = 2*t + kh from lane t = lane&3, so the 4 rows a half-warp touches have
+// row&7 in {kh, kh+2, kh+4, kh+6}: conflict-free 64-bit LDS under the swizzle.
+// The k order is fixed, so results are deterministic run to run.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+
+#include <cstdio>
+#include <mutex>
+
+#include "ptx.cuh"
+#include "tile_ops.hpp"
+
+namespace stfk {
+
+namespace g {
+constexpr int BM = 128, BN = 128, BK = 16, STAGES = 4;
+constexpr int WM = 64, WN = 32;
+constexpr int NCW = (BM / WM) * (BN / WN);  // consumer warps = 8
+constexpr int NTHREADS = NCW * 32;
+constexpr int BOX = 16;                      // doubles per 128-byte swizzle row
+constexpr int BOX_BYTES = BOX * BK * 8;      // 2 KB
+constexpr int A_BYTES = BM * BK * 8;         // 16 KB
+constexpr int B_BYTES = BN * BK * 8;         // 16 KB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 2 * STAGES * 8;
+}  // namespace g
+
+// Byte offset of element (row r in [0,128), k in [0,16)) inside one operand stage.
+__device__ __forceinline__ uint32_t swz_off(int r, int k) {
+  const int box = r >> 4, mi = r & 15;
+  return box * g::BOX_BYTES + k * 128 + ((((mi >> 1) ^ (k & 7)) << 4) | ((mi & 1) << 3));
+}
+
+__device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorMap* tmA, const CUtensorMap* tmB,
+                                           int m0, int n0, int kt, uint64_t* full) {
+  mbar_arrive_expect_tx(&full[s], g::STAGE_BYTES);
+  uint8_t* sa = smem + s * g::STAGE_BYTES;
+  uint8_t* sb = sa + g::A_BYTES;
+#pragma unroll
+  for (int b = 0; b < g::BM / g::BOX; ++b) tma_load_2d(sa + b * g::BOX_BYTES, tmA, m0 + b * g::BOX, kt * g::BK, &full[s]);
+#pragma unroll
+  for (int b = 0; b < g::BN / g::BOX; ++b) tma_load_2d(sb + b * g::BOX_BYTES, tmB, n0 + b * g::BOX, kt * g::BK, &full[s]);
+}
+
+// 8 warps, all consumers; thread 0 also issues the TMA loads (one stage behind,
+// so the refill of the stage consumed at kt-1 rarely waits).  8 warps keep the
+// register cap at 255/thread (a 9th producer warp would cap it at 168: the
+// register file is split per SM sub-partition and 9 warps round up to 12).
+__global__ void __launch_bounds__(g::NTHREADS, 1)
+    gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                        double* __restrict__ C, int64_t ldc, int M, int N, int K, int lower) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + g::STAGES * g::STAGE_BYTES);
+  uint64_t* empty = full + g::STAGES;
+
+  int tm, tn;
+  if (lower) {
+    // linear block -> (tm >= tn)
+    int b = blockIdx.x;
+    int t = (int)((sqrtf(8.0f * b + 1.0f) - 1.0f) * 0.5f);
+    while ((t + 1) * (t + 2) / 2 <= b) ++t;
+    while (t * (t + 1) / 2 > b) --t;
+    tm = t;
+    tn = b - t * (t + 1) / 2;
+  } else {
+    tm = blockIdx.x;
+    tn = blockIdx.y;
+  }
+  const int m0 = tm * g::BM, n0 = tn * g::BN;
+  const int KT = (K + g::BK - 1) / g::BK;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+    for (int s = 0; s < g::STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], g::NCW);
+    }
+    fence_barrier_init();
+    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage(smem, kt, &tmA, &tmB, m0, n0, kt, full);
+  }
+  __syncthreads();
+
+  const int wm0 = (warp % (g::BM / g::WM)) * g::WM;
+  const int wn0 = (warp / (g::BM / g::WM)) * g::WN;
+  const int gq = lane >> 2, tq = lane & 3;
+
+  // In lower mode, warps of a diagonal CTA whose warp tile is strictly upper idle.
+  const bool warp_dead = lower && (m0 == n0) && (wm0 + g::WM <= wn0);
+
+  double acc[g::WM / 8][g::WN / 8][2];
+#pragma unroll
+  for (int i = 0; i < g::WM / 8; ++i)
+#pragma unroll
+    for (int j = 0; j < g::WN / 8; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+
+  // Per-lane fragment offsets: swz_off(w0 + 8f + gq, 2tq + kh) depends on f only
+  // through the box (f >> 1, an immediate) and the chunk bit 2 (f & 1).
+  uint32_t offA[2][2], offB[2][2];
+#pragma unroll
+  for (int p = 0; p < 2; ++p)
+#pragma unroll
+    for (int kh = 0; kh < 2; ++kh) {
+      offA[p][kh] = swz_off(wm0 + 8 * p + gq, 2 * tq + kh);
+      offB[p][kh] = g::A_BYTES + swz_off(wn0 + 8 * p + gq, 2 * tq + kh);
+    }
+
+  for (int kt = 0; kt < KT; ++kt) {
+    const int s = kt % g::STAGES;
+    mbar_wait(&full[s], (kt / g::STAGES) & 1);
+    const uint8_t* st = smem + s * g::STAGE_BYTES;
+    if (!warp_dead) {
+#pragma unroll
+      for (int grp = 0; grp < g::BK / 8; ++grp) {
+        double a[g::WM / 8][2], b[g::WN / 8][2];
+#pragma unroll
+        for (int f = 0; f < g::WM / 8; ++f)
+#pragma unroll
+          for (int kh = 0; kh < 2; ++kh)
+            a[f][kh] = *reinterpret_cast<const double*>(st + offA[f & 1][kh] + (f >> 1) * g::BOX_BYTES + grp * 8 * 128);
+#pragma unroll
+        for (int f = 0; f < g::WN / 8; ++f)
+#pragma unroll
+          for (int kh = 0; kh < 2; ++kh)
+            b[f][kh] = *reinterpret_cast<const double*>(st + offB[f & 1][kh] + (f >> 1) * g::BOX_BYTES + grp * 8 * 128);
+#pragma unroll
+        for (int kh = 0; kh < 2; ++kh)
+#pragma unroll
+          for (int i = 0; i < g::WM / 8; ++i)
+#pragma unroll
+            for (int j = 0; j < g::WN / 8; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i][kh], b[j][kh]);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);
+    // refill the stage consumed in the previous iteration (all 8 warps must have released it)
+    if (threadIdx.x == 0 && kt >= 1) {
+      const int kr = kt - 1 + g::STAGES;
+      if (kr < KT) {
+        const int sr = (kt - 1) % g::STAGES;
+        mbar_wait(&empty[sr], ((kt - 1) / g::STAGES) & 1);
+        load_stage(smem, sr, &tmA, &tmB, m0, n0, kr, full);
+      }
+    }
+  }
+
+  if (warp_dead) return;
+  // ---------------- epilogue: C -= acc
+#pragma unroll
+  for (int i = 0; i < g::WM / 8; ++i) {
+    const int m = m0 + wm0 + 8 * i + gq;
+#pragma unroll
+    for (int j = 0; j < g::WN / 8; ++j) {
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int n = n0 + wn0 + 8 * j + 2 * tq + h;
+        if (m < M && n < N && (!lower || m >= n)) {
+          double* p = C + (int64_t)n * ldc + m;
+          *p = *p - acc[i][j][h];
+        }
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ host side
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+// rows x cols column-major FP64 operand, box {16 rows, BK cols}, 128B swizzle, OOB -> 0.
+static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(double)};
+  cuuint32_t box[2] = {(cuuint32_t)g::BOX, (cuuint32_t)g::BK};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(ptr), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
+                    const double* B, int64_t ldb, double* C, int64_t ldc, int lower) {
+  if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
+  if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
+    return cudaErrorMisalignedAddress;
+  CUtensorMap tmA, tmB;
+  if (!make_operand_map(&tmA, A, M, K, lda) || !make_operand_map(&tmB, B, N, K, ldb)) return cudaErrorInvalidValue;
+  const int tM = (M + g::BM - 1) / g::BM, tN = (N + g::BN - 1) / g::BN;
+  cudaLaunchConfig_t cfg = {};
+  if (lower) {
+    cfg.gridDim = dim3(tM * (tM + 1) / 2, 1, 1);
+  } else {
+    cfg.gridDim = dim3(tM, tN, 1);
+  }
+  cfg.blockDim = dim3(g::NTHREADS, 1, 1);
+  cfg.dynamicSmemBytes = g::SMEM_BYTES;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributePriority;
+  attr[0].val.priority = prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  ++launch_count();
+  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel, tmA, tmB, C, ldc, M, N, K, lower);
+}
+
+cudaError_t gemm_init_attrs() {
+  return cudaFuncSetAttribute(gemm_nt_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g::SMEM_BYTES);
+}
+
+}  // namespace stfk

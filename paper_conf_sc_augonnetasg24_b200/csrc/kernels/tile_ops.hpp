@@ -1,0 +1,54 @@
+// Host-side launchers of the sm_100a FP64 tile kernels.
+//
+// All matrices are column-major FP64 with an explicit leading dimension (in
+// elements).  Every launcher enqueues on `stream` and returns a cudaError_t of
+// the launch (asynchronous errors surface at the next synchronisation).
+// `prio` is the CUDA stream-priority value recorded on the launch (and on the
+// graph node when captured); lower numbers are higher priority.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace stfk {
+
+// K1/K2: C[M x N] -= A[M x K] * B[N x K]^T.  lower != 0 (SYRK, requires M == N
+// and A == B) updates only the elements with row >= col of C; the strictly upper
+// part of C is neither read nor written.  Requirements: A, B 16-byte aligned,
+// lda, ldb even (TMA global strides are multiples of 16 bytes).
+cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
+                    const double* B, int64_t ldb, double* C, int64_t ldc, int lower);
+
+// K3: B[M x n] <- B * L^-T with L[n x n] lower triangular, non-unit diagonal
+// (side = right, lower, transposed).  Recursive: base blocks of <= 64 columns
+// are solved by substitution, the off-diagonal blocks by gemm_nt.
+cudaError_t trsm_rlt(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                     int64_t ldb);
+
+// K4: in-place lower Cholesky of A[n x n] (lower triangle referenced, strictly
+// upper untouched).  Recursive: POTRF(A11); TRSM(A21); SYRK(A22); POTRF(A22),
+// base blocks of <= 64 solved by one CTA.  A non-positive or NaN pivot in local
+// column j does atomicMin(info, col0 + j + 1); the factorisation then continues
+// with NaN (results unspecified, LAPACK convention).
+cudaError_t potrf_lower(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
+                        unsigned long long* info);
+
+// K8: fill rows r0.., cols c0.. (global indices) of the seeded SPD metric matrix
+// of order n into dst[rows x cols] (ld).  Same SplitMix64 spec as synth/spd.py.
+cudaError_t fill_spd(cudaStream_t stream, double* dst, int64_t ld, int64_t n, int64_t r0, int64_t c0, int rows,
+                     int cols, uint64_t seed);
+
+// K7: dst[rows x cols] (ldd) = transpose(src[cols x rows] (lds)).
+cudaError_t transpose_copy(cudaStream_t stream, double* dst, int64_t ldd, const double* src, int64_t lds, int rows,
+                           int cols);
+
+// Fill a device int64 sentinel used by potrf_lower's info.
+cudaError_t info_reset(cudaStream_t stream, unsigned long long* info);
+
+// Number of kernels enqueued by the launchers above on this host thread
+// (monotonic; the runtime reports per-call deltas as gpu_launches).
+int64_t& launch_count();
+
+// Device attributes / one-time function attribute setup (max dynamic smem).
+cudaError_t kernels_init(int device);
+
+}  // namespace stfk

@@ -1,0 +1,157 @@
+// Cholesky plan construction; see plan.hpp for the model and citations.
+#include "plan.hpp"
+
+#include <algorithm>
+
+namespace stf {
+
+int streams_per_slot(const PlanOptions& opt) {
+  if (opt.serial) return 1 + opt.copy_streams;
+  return opt.crit_streams + opt.bulk_streams + opt.copy_streams;
+}
+
+namespace {
+
+struct Builder {
+  Plan& p;
+  const int64_t T;
+  const int G;
+  std::vector<int64_t> version;      // per home tile
+  std::vector<int64_t> rep_buffer;   // (tile * G + slot) -> buffer id or -1
+  std::vector<int64_t> rep_version;  // version the replica holds
+
+  Builder(Plan& plan, int64_t T_) : p(plan), T(T_), G(plan.opt.nslots) {
+    const int64_t NT = p.ntiles();
+    version.assign((size_t)NT, 0);
+    rep_buffer.assign((size_t)(NT * G), -1);
+    rep_version.assign((size_t)(NT * G), -1);
+  }
+
+  int copy_stream(int dst_slot) const {
+    const int base = p.opt.serial ? 1 : p.opt.crit_streams + p.opt.bulk_streams;
+    return base + dst_slot % p.opt.copy_streams;
+  }
+
+  int compute_stream(const Task& t) const {
+    if (p.opt.serial) return 0;
+    if (p.opt.priority && t.prio) {
+      if (t.kind == K_POTRF) return 0;
+      return (int)(t.i % p.opt.crit_streams);
+    }
+    return p.opt.crit_streams + (int)((t.i * T + t.j) % p.opt.bulk_streams);
+  }
+
+  void submit(Task t, const Access* acc, int nacc) {
+    p.graph.submit(acc, nacc);
+    p.tasks.push_back(t);
+  }
+
+  // buffer to read tile (i,j) from on `slot`, emitting a COPY if needed
+  int64_t read_buffer(int64_t i, int64_t j, int slot) {
+    const int64_t d = Plan::tile_id(i, j);
+    const int own = p.owner(i, j);
+    if (own == slot) return d;
+    const size_t r = (size_t)(d * G + slot);
+    if (rep_buffer[r] < 0) {
+      rep_buffer[r] = (int64_t)p.buffers.size();
+      p.buffers.push_back(Buffer{(int32_t)i, (int32_t)j, slot, true});
+      p.replicas_per_slot[(size_t)slot]++;
+    }
+    if (rep_version[r] != version[(size_t)d]) {
+      Task c{K_COPY, (int32_t)i, (int32_t)j, slot, own, 1, copy_stream(slot), {d, -1}, rep_buffer[r]};
+      Access acc[2] = {{d, READ}, {rep_buffer[r], WRITE}};
+      submit(c, acc, 2);
+      p.ntransfers++;
+      rep_version[r] = version[(size_t)d];
+    }
+    return rep_buffer[r];
+  }
+
+  void compute(int32_t kind, int64_t i, int64_t j, int64_t k, int prio, int64_t ra, int64_t rb, int64_t wi,
+               int64_t wj) {
+    const int slot = p.owner(wi, wj);
+    const int64_t w = Plan::tile_id(wi, wj);
+    int64_t in0 = ra >= 0 ? read_buffer(ra / T, ra % T, slot) : -1;
+    int64_t in1 = rb >= 0 ? read_buffer(rb / T, rb % T, slot) : -1;
+    Task t{kind, (int32_t)i, (int32_t)j, (int32_t)k, slot, prio, 0, {in0, in1}, w};
+    t.stream = compute_stream(t);
+    Access acc[3];
+    int n = 0;
+    if (in0 >= 0) acc[n++] = {in0, READ};
+    if (in1 >= 0) acc[n++] = {in1, READ};
+    acc[n++] = {w, RW};
+    submit(t, acc, n);
+    version[(size_t)w]++;
+  }
+
+  void run() {
+    const int64_t NT = p.ntiles();
+    p.buffers.clear();
+    for (int64_t i = 0; i < T; ++i)
+      for (int64_t j = 0; j <= i; ++j) p.buffers.push_back(Buffer{(int32_t)i, (int32_t)j, p.owner(i, j), false});
+    (void)NT;
+    if (p.opt.with_load) {
+      for (int64_t j = 0; j < T; ++j)
+        for (int64_t i = j; i < T; ++i) {
+          const int own = p.owner(i, j);
+          const int64_t w = Plan::tile_id(i, j);
+          Task t{K_LOAD, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own), {-1, -1}, w};
+          Access acc[1] = {{w, WRITE}};
+          submit(t, acc, 1);
+          version[(size_t)w]++;
+        }
+    }
+    auto key = [&](int64_t i, int64_t j) { return i * T + j; };
+    const bool prio = p.opt.priority;
+    for (int64_t k = 0; k < T; ++k) {
+      compute(K_POTRF, k, k, k, 1, -1, -1, k, k);
+      for (int64_t i = k + 1; i < T; ++i) compute(K_TRSM, i, k, k, 1, key(k, k), -1, i, k);
+      for (int64_t i = k + 1; i < T; ++i) {
+        compute(K_SYRK, i, i, k, prio && i == k + 1, key(i, k), -1, i, i);
+        for (int64_t j = k + 1; j < i; ++j) compute(K_GEMM, i, j, k, prio && j == k + 1, key(i, k), key(j, k), i, j);
+      }
+    }
+    if (p.opt.with_store) {
+      for (int64_t j = 0; j < T; ++j)
+        for (int64_t i = j; i < T; ++i) {
+          const int own = p.owner(i, j);
+          const int64_t d = Plan::tile_id(i, j);
+          Task t{K_STORE, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own), {d, -1}, -1};
+          Access acc[1] = {{d, READ}};
+          submit(t, acc, 1);
+        }
+    }
+  }
+};
+
+}  // namespace
+
+void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
+  plan.T = T;
+  plan.opt = opt;
+  if (plan.opt.crit_streams < 1) plan.opt.crit_streams = 1;
+  if (plan.opt.bulk_streams < 1) plan.opt.bulk_streams = 1;
+  if (plan.opt.copy_streams < 1) plan.opt.copy_streams = 1;
+  plan.tasks.clear();
+  plan.ntransfers = 0;
+  plan.replicas_per_slot.assign((size_t)opt.nslots, 0);
+  // dense datum ids: home tiles + at most one replica per (tile, slot)
+  const int64_t NT = T * (T + 1) / 2;
+  plan.graph = TaskGraph(NT + NT * opt.nslots + 1);
+  Builder b(plan, T);
+  b.run();
+  // longest chain of compute tasks (COPY/LOAD/STORE weigh 0)
+  std::vector<int64_t> depth(plan.tasks.size(), 0);
+  int64_t best = 0;
+  for (size_t t = 0; t < plan.tasks.size(); ++t) {
+    int64_t d = 0;
+    for (const int64_t* q = plan.graph.preds_begin((int64_t)t); q != plan.graph.preds_end((int64_t)t); ++q)
+      d = std::max(d, depth[(size_t)*q]);
+    const int32_t kd = plan.tasks[t].kind;
+    depth[t] = d + ((kd <= K_GEMM) ? 1 : 0);
+    best = std::max(best, depth[t]);
+  }
+  plan.critical_path = best;
+}
+
+}  // namespace stf

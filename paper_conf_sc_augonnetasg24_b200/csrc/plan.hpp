@@ -1,0 +1,82 @@
+// Cholesky task generator + 2D block-cyclic placement + MSI-lite replicas +
+// stream assignment (§8 rows a1-a3, a5, a7).
+//
+// Program order (right-looking tiled Cholesky, ref. [17] PAPER.md:495; one
+// logical datum per tile):
+//   for k: POTRF(k)                      A_kk:rw
+//          for i>k: TRSM(i,k)            A_kk:r  A_ik:rw
+//          for i>k: SYRK(i,k)            A_ik:r  A_ii:rw
+//                   for k<j<i: GEMM(i,j,k)  A_ik:r  A_jk:r  A_ij:rw
+// Placement (owner computes): the task runs on the owner
+// of the tile it writes; owner(i,j) = (i mod P)*Q + (j mod Q).
+// Coherency (asynchronous MSI): every tile has a home
+// instance on its owner; a read on another slot needs a valid replica there.
+// If the replica is missing or stale (tile version changed), a COPY task is
+// emitted in program order just before the reader: it reads the home tile and
+// writes the replica datum, so the same STF rule orders it after the tile's
+// last writer and before every later writer of the replica (WAR).  Cholesky
+// tiles are final when first read remotely, so each replica is copied once.
+// Optional LOAD (tile <- caller matrix) and STORE (caller matrix <- tile) tasks
+// implement the COLMAJOR descriptors and the write-back of PAPER.md:146-148.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "stf_core.hpp"
+
+namespace stf {
+
+enum Kind : int32_t { K_POTRF = 0, K_TRSM = 1, K_SYRK = 2, K_GEMM = 3, K_COPY = 4, K_LOAD = 5, K_STORE = 6 };
+
+struct Task {
+  int32_t kind;
+  int32_t i, j, k;   // tile indices (COPY/LOAD/STORE: tile (i,j); COPY: k = destination slot)
+  int32_t slot;      // executing slot (COPY: source slot, push model)
+  int32_t prio;      // 1 = critical path (high-priority stream), 0 = bulk
+  int32_t stream;    // index into the slot's stream pool (see Lowering in runtime.cpp)
+  int64_t in[2];     // buffer ids read (-1 if unused)
+  int64_t out;       // buffer id written
+};
+
+struct PlanOptions {
+  int P = 1, Q = 1;
+  int nslots = 1;
+  int bulk_streams = 8;
+  int crit_streams = 2;
+  int copy_streams = 2;
+  bool serial = false;     // all tasks of all slots on stream 0 (program order)
+  bool priority = true;
+  bool with_load = false;  // LOAD tasks first (COLMAJOR descriptors)
+  bool with_store = false; // STORE tasks (write-back) at the end of program order
+};
+
+// A "buffer" is one physical nb x nb tile instance: home tiles are buffers
+// 0..NT-1 (lower tile (i,j) -> i*(i+1)/2 + j), replicas follow.
+struct Buffer {
+  int32_t i, j, slot;
+  bool replica;
+};
+
+struct Plan {
+  int64_t T = 0;
+  PlanOptions opt;
+  std::vector<Task> tasks;
+  std::vector<Buffer> buffers;
+  TaskGraph graph;
+  int64_t ntransfers = 0;
+  int64_t critical_path = 0;  // longest chain counted in compute tasks
+  std::vector<int64_t> replicas_per_slot;
+
+  int owner(int64_t i, int64_t j) const { return (int)((i % opt.P) * opt.Q + (j % opt.Q)); }
+  static int64_t tile_id(int64_t i, int64_t j) { return i * (i + 1) / 2 + j; }
+  int64_t ntiles() const { return T * (T + 1) / 2; }
+};
+
+// Build the full plan (tasks, DAG, replicas, stream assignment).  Pure host code.
+void build_plan(Plan& plan, int64_t T, const PlanOptions& opt);
+
+// Number of pool streams a slot needs for `opt`.
+int streams_per_slot(const PlanOptions& opt);
+
+}  // namespace stf

@@ -1,0 +1,986 @@
+// Runtime: context, per-slot stream pools, lowering of the STF plan onto CUDA
+// streams + events (eager) or into one CUDA graph per call configuration
+// (memoised), and the C ABI of include/stf_cholesky.h.
+//
+// Paper mechanisms realised here:
+//   A4  Algorithm 2 prologue: for each task, wait on the
+//       events of its STF predecessors that ran on other streams (enforce_stf),
+//       allocation is done once per plan (replica arenas), update = COPY tasks.
+//   A8  stream pools per device.
+//   A9  stream backend: ordering with cudaStreamWaitEvent.
+//   A10 graph backend: the whole DAG of one stf_potrf call (one epoch,
+//       PAPER.md:166-172) captured into a CUDA graph; multi-stream capture keeps
+//       the DAG's concurrency, and per-node priorities keep the look-ahead.
+//   A11 memoisation of executable graphs across calls, keyed by the call
+//       configuration.
+//   A12 abstract events: a task's completion is an event only when a successor
+//       runs on another stream; in a graph these become plain edges.
+//   A13 finalize: synchronous completion + write-back.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <climits>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <list>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/stf_cholesky.h"
+#include "kernels/tile_ops.hpp"
+#include "plan.hpp"
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+int cuda_fail(cudaError_t e, const char* what) {
+  cudaGetLastError();  // clear sticky-free errors
+  if (e == cudaErrorMemoryAllocation) return fail(-103, "%s: %s", what, cudaGetErrorString(e));
+  return fail(-101, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CUDA_TRY(expr, what)                 \
+  do {                                       \
+    cudaError_t e_ = (expr);                 \
+    if (e_ != cudaSuccess) return cuda_fail(e_, what); \
+  } while (0)
+
+int64_t env_int(const char* name, int64_t dflt) {
+  const char* v = getenv(name);
+  if (!v || !*v) return dflt;
+  return strtoll(v, nullptr, 10);
+}
+
+struct Slot {
+  int device = 0;
+  std::vector<cudaStream_t> streams;
+  unsigned long long* d_info = nullptr;
+};
+
+struct Options {
+  int64_t graph = 1;
+  int64_t streams = 8;
+  int64_t serial = 0;
+  int64_t priority = 1;
+  int64_t grid_p = 0;
+};
+
+// A plan bound to physical buffers, plus its lowering artefacts.
+struct Exec {
+  // key
+  int64_t n = 0, nb = 0;
+  char uplo = 'L';
+  int kind = 0, ngpus = 0, P = 1, Q = 1;
+  Options opt;
+  std::vector<uintptr_t> key_ptrs;
+  int64_t key_ld = 0;
+  int key_dev = 0;
+
+  stf::Plan plan;
+  std::vector<double*> buf;           // buffer id -> device pointer
+  std::vector<std::pair<int, void*>> allocs;  // (device, ptr) library-owned
+  std::vector<double*> scratch;       // per (slot, copy stream): staging tile for 'U'
+  std::vector<cudaEvent_t> events;    // per task, null if not needed
+  std::vector<int> events_dev;
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+  int64_t graph_nodes = 0;
+  int64_t launches = 0;
+  double build_ms = 0;
+  // caller matrix for COLMAJOR kinds
+  double* mat = nullptr;
+  int64_t ld = 0;
+  int mat_dev = -1;  // -1: host
+
+  ~Exec() {
+    if (gexec) cudaGraphExecDestroy(gexec);
+    if (graph) cudaGraphDestroy(graph);
+    for (size_t t = 0; t < events.size(); ++t)
+      if (events[t]) {
+        cudaSetDevice(events_dev[t]);
+        cudaEventDestroy(events[t]);
+      }
+    for (auto& a : allocs) {
+      cudaSetDevice(a.first);
+      cudaFree(a.second);
+    }
+  }
+};
+
+struct Context {
+  std::mutex mu;
+  bool inited = false;
+  std::vector<Slot> slots;
+  std::vector<int> devices;  // distinct physical devices
+  Options opt;
+  std::list<std::unique_ptr<Exec>> cache;  // MRU first
+  stf_plan_stats last{};
+  cudaStream_t origin = nullptr;  // capture / launch stream on slot 0's device
+  int origin_dev = 0;
+  std::vector<cudaEvent_t> fork_join;  // per slot-stream, for fork/join around a call
+  cudaEvent_t t_start = nullptr, t_end = nullptr;  // timing events on `origin`
+  double device_ms = 0;
+};
+
+Context& ctx() {
+  static Context c;
+  return c;
+}
+
+constexpr int kCritStreams = 4;
+constexpr int kCopyStreams = 2;
+constexpr size_t kCacheMax = 4;
+
+stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool load, bool store) {
+  stf::PlanOptions po;
+  po.P = P;
+  po.Q = Q;
+  po.nslots = nslots;
+  po.bulk_streams = (int)std::max<int64_t>(1, o.streams);
+  po.crit_streams = kCritStreams;
+  po.copy_streams = kCopyStreams;
+  po.serial = o.serial != 0;
+  po.priority = o.priority != 0;
+  po.with_load = load;
+  po.with_store = store;
+  return po;
+}
+
+// ------------------------------------------------------------------ lowering
+struct Lowerer {
+  Context& C;
+  Exec& X;
+  int cur_dev = -1;
+
+  void set_dev(int d) {
+    if (d != cur_dev) {
+      cudaSetDevice(d);
+      cur_dev = d;
+    }
+  }
+  cudaStream_t stream_of(const stf::Task& t) { return C.slots[(size_t)t.slot].streams[(size_t)t.stream]; }
+  int prio_of(const stf::Task& t) {
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    return (X.opt.priority && t.prio) ? hi : lo;
+  }
+
+  int body(const stf::Task& t, cudaStream_t s, int prio) {
+    const int64_t nb = X.nb;
+    const size_t tile_bytes = (size_t)(nb * nb) * sizeof(double);
+    Slot& S = C.slots[(size_t)t.slot];
+    switch (t.kind) {
+      case stf::K_POTRF:
+        CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
+                 "POTRF launch");
+        return 0;
+      case stf::K_TRSM:
+        CUDA_TRY(stfk::trsm_rlt(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb),
+                 "TRSM launch");
+        return 0;
+      case stf::K_SYRK:
+        CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[0]],
+                               nb, X.buf[(size_t)t.out], nb, 1),
+                 "SYRK launch");
+        return 0;
+      case stf::K_GEMM:
+        CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[1]],
+                               nb, X.buf[(size_t)t.out], nb, 0),
+                 "GEMM launch");
+        return 0;
+      case stf::K_COPY: {
+        const int dst_dev = C.slots[(size_t)t.k].device, src_dev = S.device;
+        if (dst_dev == src_dev)
+          CUDA_TRY(cudaMemcpyAsync(X.buf[(size_t)t.out], X.buf[(size_t)t.in[0]], tile_bytes, cudaMemcpyDeviceToDevice, s),
+                   "replica copy");
+        else
+          CUDA_TRY(cudaMemcpyPeerAsync(X.buf[(size_t)t.out], dst_dev, X.buf[(size_t)t.in[0]], src_dev, tile_bytes, s),
+                   "replica peer copy");
+        return 0;
+      }
+      case stf::K_LOAD:
+      case stf::K_STORE: {
+        const bool load = t.kind == stf::K_LOAD;
+        double* tile = X.buf[(size_t)(load ? t.out : t.in[0])];
+        const int64_t i = t.i, j = t.j;
+        const bool upper = (X.uplo == 'U');
+        // block of the caller matrix holding tile (i,j) of L: (i,j) for 'L', (j,i) transposed for 'U'
+        double* blk = upper ? X.mat + (j * nb) + (i * nb) * X.ld : X.mat + (i * nb) + (j * nb) * X.ld;
+        if (!upper) {
+          if (load)
+            CUDA_TRY(cudaMemcpy2DAsync(tile, nb * 8, blk, X.ld * 8, nb * 8, nb, cudaMemcpyDefault, s), "load tile");
+          else
+            CUDA_TRY(cudaMemcpy2DAsync(blk, X.ld * 8, tile, nb * 8, nb * 8, nb, cudaMemcpyDefault, s), "store tile");
+          return 0;
+        }
+        const size_t scr_idx = (size_t)t.slot * kCopyStreams + (size_t)(t.stream % kCopyStreams);
+        if (X.mat_dev >= 0 && X.mat_dev == S.device) {
+          if (load)
+            CUDA_TRY(stfk::transpose_copy(s, tile, nb, blk, X.ld, (int)nb, (int)nb), "load transpose");
+          else
+            CUDA_TRY(stfk::transpose_copy(s, blk, X.ld, tile, nb, (int)nb, (int)nb), "store transpose");
+          return 0;
+        }
+        double* scr = X.scratch[scr_idx];
+        if (load) {
+          CUDA_TRY(cudaMemcpy2DAsync(scr, nb * 8, blk, X.ld * 8, nb * 8, nb, cudaMemcpyDefault, s), "load stage");
+          CUDA_TRY(stfk::transpose_copy(s, tile, nb, scr, nb, (int)nb, (int)nb), "load transpose");
+        } else {
+          CUDA_TRY(stfk::transpose_copy(s, scr, nb, tile, nb, (int)nb, (int)nb), "store transpose");
+          CUDA_TRY(cudaMemcpy2DAsync(blk, X.ld * 8, scr, nb * 8, nb * 8, nb, cudaMemcpyDefault, s), "store stage");
+        }
+        return 0;
+      }
+    }
+    return fail(-101, "unknown task kind %d", t.kind);
+  }
+
+  // Enqueue every task in program order.  Assumes all pool streams are ready
+  // (forked from the origin when capturing).
+  int issue() {
+    const stf::Plan& P = X.plan;
+    const int64_t launches0 = stfk::launch_count();
+    // info reset on each slot's first stream
+    for (size_t s = 0; s < C.slots.size() && s < (size_t)X.ngpus; ++s) {
+      set_dev(C.slots[s].device);
+      CUDA_TRY(stfk::info_reset(C.slots[s].streams[0], C.slots[s].d_info), "info reset");
+    }
+    // info reset must precede POTRFs on other streams of the slot: make every
+    // stream of the slot wait for it
+    for (size_t s = 0; s < C.slots.size() && s < (size_t)X.ngpus; ++s) {
+      Slot& S = C.slots[s];
+      set_dev(S.device);
+      cudaEvent_t ev = C.fork_join[s * S.streams.size()];
+      CUDA_TRY(cudaEventRecord(ev, S.streams[0]), "record info event");
+      for (size_t k = 1; k < S.streams.size(); ++k) CUDA_TRY(cudaStreamWaitEvent(S.streams[k], ev, 0), "wait info event");
+    }
+    for (size_t t = 0; t < P.tasks.size(); ++t) {
+      const stf::Task& task = P.tasks[t];
+      set_dev(C.slots[(size_t)task.slot].device);
+      cudaStream_t s = stream_of(task);
+      for (const int64_t* q = P.graph.preds_begin((int64_t)t); q != P.graph.preds_end((int64_t)t); ++q) {
+        const stf::Task& pt = P.tasks[(size_t)*q];
+        if (pt.slot == task.slot && pt.stream == task.stream) continue;  // stream order suffices
+        CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
+      }
+      int r = body(task, s, prio_of(task));
+      if (r) return r;
+      if (X.events[t]) CUDA_TRY(cudaEventRecord(X.events[t], s), "event record");
+    }
+    X.launches = stfk::launch_count() - launches0;
+    return 0;
+  }
+};
+
+// fork all pool streams of the first ngpus slots from `origin` / join them back
+int fork_streams(Context& C, int ngpus) {
+  cudaSetDevice(C.origin_dev);
+  cudaEvent_t fork = C.fork_join.back();
+  CUDA_TRY(cudaEventRecord(fork, C.origin), "fork record");
+  for (int s = 0; s < ngpus; ++s) {
+    Slot& S = C.slots[(size_t)s];
+    cudaSetDevice(S.device);
+    for (cudaStream_t st : S.streams) CUDA_TRY(cudaStreamWaitEvent(st, fork, 0), "fork wait");
+  }
+  return 0;
+}
+
+int join_streams(Context& C, int ngpus) {
+  for (int s = 0; s < ngpus; ++s) {
+    Slot& S = C.slots[(size_t)s];
+    cudaSetDevice(S.device);
+    for (size_t k = 0; k < S.streams.size(); ++k) {
+      cudaEvent_t ev = C.fork_join[(size_t)s * S.streams.size() + k];
+      CUDA_TRY(cudaEventRecord(ev, S.streams[k]), "join record");
+      cudaSetDevice(C.origin_dev);
+      CUDA_TRY(cudaStreamWaitEvent(C.origin, ev, 0), "join wait");
+      cudaSetDevice(S.device);
+    }
+  }
+  cudaSetDevice(C.origin_dev);
+  return 0;
+}
+
+int alloc_on(Exec& X, int dev, size_t bytes, double** out) {
+  cudaSetDevice(dev);
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (plan workspace)");
+  X.allocs.push_back({dev, p});
+  *out = static_cast<double*>(p);
+  return 0;
+}
+
+// Build plan + buffers + events (+ graph) for X (key fields already set).
+int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
+  auto t0 = std::chrono::steady_clock::now();
+  const int64_t T = X.n / X.nb;
+  const bool colmajor = X.kind != STF_DESC_TILED_2DBC;
+  stf::build_plan(X.plan, T, plan_options(X.opt, X.P, X.Q, X.ngpus, colmajor, colmajor));
+  const stf::Plan& P = X.plan;
+  const size_t tile_bytes = (size_t)(X.nb * X.nb) * sizeof(double);
+  X.buf.assign(P.buffers.size(), nullptr);
+  // home tiles
+  if (!colmajor) {
+    for (size_t b = 0; b < (size_t)P.ntiles(); ++b) {
+      const stf::Buffer& B = P.buffers[b];
+      X.buf[b] = desc->tiles[(size_t)B.i + (size_t)B.j * (size_t)T];
+    }
+  } else {
+    X.mat = desc->ptr;
+    X.ld = desc->ld;
+    X.mat_dev = (X.kind == STF_DESC_DEVICE_COLMAJOR) ? desc->device : -1;
+  }
+  // library-owned storage: per slot one arena for (COLMAJOR) home tiles + replicas
+  for (int s = 0; s < X.ngpus; ++s) {
+    size_t count = 0;
+    for (size_t b = 0; b < P.buffers.size(); ++b) {
+      const stf::Buffer& B = P.buffers[b];
+      if (B.slot == s && (B.replica || colmajor)) count++;
+    }
+    const size_t nscr = (colmajor && X.uplo == 'U') ? kCopyStreams : 0;
+    if (count + nscr == 0) continue;
+    double* arena = nullptr;
+    int r = alloc_on(X, C.slots[(size_t)s].device, (count + nscr) * tile_bytes, &arena);
+    if (r) return r;
+    size_t used = 0;
+    for (size_t b = 0; b < P.buffers.size(); ++b) {
+      const stf::Buffer& B = P.buffers[b];
+      if (B.slot == s && (B.replica || colmajor)) X.buf[b] = arena + (used++) * (size_t)(X.nb * X.nb);
+    }
+    if (nscr) {
+      X.scratch.resize((size_t)X.ngpus * kCopyStreams, nullptr);
+      for (size_t k = 0; k < nscr; ++k) X.scratch[(size_t)s * kCopyStreams + k] = arena + (used++) * (size_t)(X.nb * X.nb);
+    }
+  }
+  // events only where a successor runs on another stream
+  std::vector<int64_t> soff, succ;
+  P.graph.build_successors(soff, succ);
+  X.events.assign(P.tasks.size(), nullptr);
+  X.events_dev.assign(P.tasks.size(), 0);
+  for (size_t t = 0; t < P.tasks.size(); ++t) {
+    const stf::Task& a = P.tasks[t];
+    bool need = false;
+    for (int64_t e = soff[t]; e < soff[t + 1] && !need; ++e) {
+      const stf::Task& b = P.tasks[(size_t)succ[(size_t)e]];
+      need = !(b.slot == a.slot && b.stream == a.stream);
+    }
+    if (need) {
+      const int dev = C.slots[(size_t)a.slot].device;
+      cudaSetDevice(dev);
+      CUDA_TRY(cudaEventCreateWithFlags(&X.events[t], cudaEventDisableTiming), "cudaEventCreate");
+      X.events_dev[t] = dev;
+    }
+  }
+  if (X.opt.graph) {
+    cudaSetDevice(C.origin_dev);
+    CUDA_TRY(cudaStreamBeginCapture(C.origin, cudaStreamCaptureModeThreadLocal), "begin capture");
+    int r = fork_streams(C, X.ngpus);
+    Lowerer L{C, X};
+    if (!r) r = L.issue();
+    if (!r) r = join_streams(C, X.ngpus);
+    cudaSetDevice(C.origin_dev);
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(C.origin, &g);
+    if (r) {
+      if (g) cudaGraphDestroy(g);
+      return r;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "end capture");
+    X.graph = g;
+    size_t nn = 0;
+    cudaGraphGetNodes(g, nullptr, &nn);
+    X.graph_nodes = (int64_t)nn;
+    CUDA_TRY(cudaGraphInstantiateWithFlags(&X.gexec, g, cudaGraphInstantiateFlagUseNodePriority), "graph instantiate");
+  }
+  X.build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return 0;
+}
+
+int run(Context& C, Exec& X) {
+  cudaSetDevice(C.origin_dev);
+  CUDA_TRY(cudaEventRecord(C.t_start, C.origin), "timing start");
+  if (X.opt.graph) {
+    CUDA_TRY(cudaGraphLaunch(X.gexec, C.origin), "graph launch");
+  } else {
+    int r = fork_streams(C, X.ngpus);
+    Lowerer L{C, X};
+    if (!r) r = L.issue();
+    if (!r) r = join_streams(C, X.ngpus);
+    if (r) return r;
+  }
+  cudaSetDevice(C.origin_dev);
+  CUDA_TRY(cudaEventRecord(C.t_end, C.origin), "timing end");
+  CUDA_TRY(cudaStreamSynchronize(C.origin), "factorisation sync");
+  float ms = 0.f;
+  CUDA_TRY(cudaEventElapsedTime(&ms, C.t_start, C.t_end), "timing elapsed");
+  C.device_ms = ms;
+  // info = min over slots (0 if none failed)
+  unsigned long long best = ULLONG_MAX;
+  for (int s = 0; s < X.ngpus; ++s) {
+    unsigned long long v = 0;
+    cudaSetDevice(C.slots[(size_t)s].device);
+    CUDA_TRY(cudaMemcpy(&v, C.slots[(size_t)s].d_info, sizeof v, cudaMemcpyDeviceToHost), "info readback");
+    best = std::min(best, v);
+  }
+  cudaSetDevice(C.origin_dev);
+  return best == ULLONG_MAX ? 0 : (int)std::min<unsigned long long>(best, INT_MAX);
+}
+
+void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
+  const stf::Plan& P = X.plan;
+  int64_t compute = 0;
+  for (const auto& t : P.tasks) compute += (t.kind <= stf::K_GEMM);
+  s->tasks = compute;
+  s->transfers = P.ntransfers;
+  s->edges = P.graph.nedges();
+  s->transfer_bytes = P.ntransfers * X.nb * X.nb * 8;
+  s->critical_path = P.critical_path;
+  s->graph_nodes = X.graph_nodes;
+  s->kernel_launches = X.launches;
+  s->build_ms = hit ? 0.0 : X.build_ms;
+}
+
+int choose_grid(int ngpus, int64_t grid_p, int* P, int* Q) {
+  if (grid_p > 0) {
+    if (ngpus % grid_p) return -1;
+    *P = (int)grid_p;
+    *Q = ngpus / (int)grid_p;
+    return 0;
+  }
+  int best = 1;
+  for (int p = 1; p * p <= ngpus; ++p)
+    if (ngpus % p == 0) best = p;
+  *P = best;
+  *Q = ngpus / best;
+  return 0;
+}
+
+bool device_of(const void* ptr, int* dev) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  if (a.type != cudaMemoryTypeDevice && a.type != cudaMemoryTypeManaged) return false;
+  *dev = a.device;
+  return true;
+}
+
+// page-locked (or registered) host memory: capturable async copies
+bool host_pinned(const void* ptr) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost;
+}
+
+int ensure_kernel_attrs(int dev) {
+  static std::mutex m;
+  static std::vector<int> done;
+  std::lock_guard<std::mutex> g(m);
+  if (std::find(done.begin(), done.end(), dev) != done.end()) return 0;
+  cudaError_t e = stfk::kernels_init(dev);
+  if (e != cudaSuccess) return cuda_fail(e, "kernel attributes");
+  done.push_back(dev);
+  return 0;
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+const char* stf_last_error(void) { return g_err.c_str(); }
+
+int stf_cholesky_init(int ngpus, const int* device_ids) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (C.inited) return fail(-104, "stf_cholesky_init called twice without stf_finalize");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(-101, "no CUDA device available (%s)", cudaGetErrorString(e));
+  }
+  if (ngpus < 1 || ngpus > 64) return fail(-5, "ngpus=%d out of range", ngpus);
+  C.opt.graph = env_int("STF_GRAPH", 1);
+  C.opt.streams = env_int("STF_STREAMS", 8);
+  C.opt.serial = env_int("STF_SERIAL", 0);
+  C.opt.priority = env_int("STF_PRIO", 1);
+  C.opt.grid_p = 0;
+  if (const char* gs = getenv("STF_GRID")) C.opt.grid_p = atoi(gs);
+  C.slots.assign((size_t)ngpus, Slot{});
+  C.devices.clear();
+  for (int s = 0; s < ngpus; ++s) {
+    const int d = device_ids ? device_ids[s] : s;
+    if (d < 0 || d >= ndev) {
+      C.slots.clear();
+      return fail(-5, "device id %d of slot %d out of range (have %d)", d, s, ndev);
+    }
+    C.slots[(size_t)s].device = d;
+    if (std::find(C.devices.begin(), C.devices.end(), d) == C.devices.end()) C.devices.push_back(d);
+  }
+  // peer access between distinct devices
+  for (int a : C.devices)
+    for (int b : C.devices) {
+      if (a == b) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, a, b);
+      if (can) {
+        cudaSetDevice(a);
+        cudaError_t pe = cudaDeviceEnablePeerAccess(b, 0);
+        if (pe != cudaSuccess && pe != cudaErrorPeerAccessAlreadyEnabled) {
+          cudaGetLastError();
+          return cuda_fail(pe, "enable peer access");
+        }
+        cudaGetLastError();
+      }
+    }
+  for (int d : C.devices) {
+    int r = ensure_kernel_attrs(d);
+    if (r) return r;
+  }
+  // stream pools: sized for the largest configuration (crit + bulk + copy)
+  const int nstreams = kCritStreams + (int)std::max<int64_t>(1, C.opt.streams) + kCopyStreams;
+  int lo = 0, hi = 0;
+  for (auto& S : C.slots) {
+    cudaSetDevice(S.device);
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    S.streams.resize((size_t)nstreams);
+    for (int k = 0; k < nstreams; ++k) {
+      const int pr = (k < kCritStreams) ? hi : lo;
+      CUDA_TRY(cudaStreamCreateWithPriority(&S.streams[(size_t)k], cudaStreamNonBlocking, pr), "stream create");
+    }
+    CUDA_TRY(cudaMalloc(&S.d_info, sizeof(unsigned long long)), "info alloc");
+  }
+  C.origin_dev = C.slots[0].device;
+  cudaSetDevice(C.origin_dev);
+  CUDA_TRY(cudaStreamCreateWithFlags(&C.origin, cudaStreamNonBlocking), "origin stream");
+  C.fork_join.assign((size_t)ngpus * (size_t)nstreams + 1, nullptr);
+  for (size_t k = 0; k < C.fork_join.size(); ++k) {
+    const int dev = (k + 1 == C.fork_join.size()) ? C.origin_dev : C.slots[k / (size_t)nstreams].device;
+    cudaSetDevice(dev);
+    CUDA_TRY(cudaEventCreateWithFlags(&C.fork_join[k], cudaEventDisableTiming), "fork/join event");
+  }
+  cudaSetDevice(C.origin_dev);
+  CUDA_TRY(cudaEventCreate(&C.t_start), "timing event");
+  CUDA_TRY(cudaEventCreate(&C.t_end), "timing event");
+  C.inited = true;
+  return 0;
+}
+
+static void release_all(Context& C) {
+  C.cache.clear();
+  for (size_t k = 0; k < C.fork_join.size(); ++k)
+    if (C.fork_join[k]) cudaEventDestroy(C.fork_join[k]);
+  C.fork_join.clear();
+  for (auto& S : C.slots) {
+    cudaSetDevice(S.device);
+    for (auto st : S.streams) cudaStreamDestroy(st);
+    if (S.d_info) cudaFree(S.d_info);
+  }
+  C.slots.clear();
+  if (C.t_start) cudaEventDestroy(C.t_start);
+  if (C.t_end) cudaEventDestroy(C.t_end);
+  C.t_start = C.t_end = nullptr;
+  if (C.origin) {
+    cudaSetDevice(C.origin_dev);
+    cudaStreamDestroy(C.origin);
+    C.origin = nullptr;
+  }
+  C.inited = false;
+}
+
+int stf_finalize(void) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (!C.inited) return fail(-100, "stf_finalize: library not initialised");
+  for (int d : C.devices) {
+    cudaSetDevice(d);
+    cudaDeviceSynchronize();
+  }
+  release_all(C);
+  return 0;
+}
+
+int stf_set_option(const char* name, int64_t value) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (!name) return fail(-105, "option name is NULL");
+  std::string n(name);
+  if (n == "graph") C.opt.graph = value != 0;
+  else if (n == "streams") {
+    if (value < 1 || value > 64) return fail(-105, "streams must be in [1, 64]");
+    const int have = C.inited ? (int)C.slots[0].streams.size() - kCritStreams - kCopyStreams : 64;
+    if (value > have) return fail(-105, "streams=%lld exceeds the pool created at init (%d)", (long long)value, have);
+    C.opt.streams = value;
+  } else if (n == "serial") C.opt.serial = value != 0;
+  else if (n == "priority") C.opt.priority = value != 0;
+  else if (n == "grid_p") {
+    if (value < 0) return fail(-105, "grid_p must be >= 0");
+    C.opt.grid_p = value;
+  } else return fail(-105, "unknown option '%s'", name);
+  return 0;
+}
+
+int stf_get_option(const char* name, int64_t* value) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (!name || !value) return fail(-105, "NULL argument");
+  std::string n(name);
+  if (n == "graph") *value = C.opt.graph;
+  else if (n == "streams") *value = C.opt.streams;
+  else if (n == "serial") *value = C.opt.serial;
+  else if (n == "priority") *value = C.opt.priority;
+  else if (n == "grid_p") *value = C.opt.grid_p;
+  else return fail(-105, "unknown option '%s'", name);
+  return 0;
+}
+
+int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngpus) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  // argument checks first (LAPACK order), then runtime state
+  if (n < 0) return fail(-1, "n=%lld < 0", (long long)n);
+  if (nb < 2 || (nb & 1) || (n > 0 && n % nb != 0) || nb > 16384)
+    return fail(-2, "nb=%lld must be even, >= 2, <= 16384 and divide n=%lld", (long long)nb, (long long)n);
+  const char up = (uplo == 'l') ? 'L' : (uplo == 'u') ? 'U' : uplo;
+  if (up != 'L' && up != 'U') return fail(-3, "uplo='%c' must be 'L' or 'U'", uplo);
+  if (!A_desc) return fail(-4, "A_desc is NULL");
+  if (A_desc->kind != STF_DESC_TILED_2DBC && A_desc->kind != STF_DESC_DEVICE_COLMAJOR &&
+      A_desc->kind != STF_DESC_HOST_COLMAJOR)
+    return fail(-4, "unknown descriptor kind %d", A_desc->kind);
+  if (A_desc->kind == STF_DESC_TILED_2DBC && up != 'L') return fail(-3, "uplo='U' requires a COLMAJOR descriptor");
+  if (A_desc->kind != STF_DESC_TILED_2DBC) {
+    if (!A_desc->ptr && n > 0) return fail(-4, "descriptor ptr is NULL");
+    if (A_desc->ld < std::max<int64_t>(1, n)) return fail(-4, "ld=%lld < max(1,n)", (long long)A_desc->ld);
+  } else {
+    if (!A_desc->tiles && n > 0) return fail(-4, "descriptor tiles table is NULL");
+    if (A_desc->p < 1 || A_desc->q < 1 || (int64_t)A_desc->p * A_desc->q != ngpus)
+      return fail(-4, "grid %dx%d does not match ngpus=%d", A_desc->p, A_desc->q, ngpus);
+  }
+  if (ngpus < 1) return fail(-5, "ngpus=%d < 1", ngpus);
+  if (!C.inited) return fail(-100, "stf_potrf: call stf_cholesky_init first");
+  if (ngpus > (int)C.slots.size()) return fail(-5, "ngpus=%d exceeds the %zu initialised slots", ngpus, C.slots.size());
+  if (n == 0) return 0;
+
+  int P = A_desc->p, Q = A_desc->q;
+  if (A_desc->kind != STF_DESC_TILED_2DBC) {
+    if (choose_grid(ngpus, C.opt.grid_p, &P, &Q)) return fail(-4, "grid_p does not divide ngpus");
+    if (A_desc->kind == STF_DESC_DEVICE_COLMAJOR) {
+      int d = -1;
+      if (!device_of(A_desc->ptr, &d) || d != A_desc->device)
+        return fail(-4, "DEVICE_COLMAJOR ptr is not device memory of device %d", A_desc->device);
+    }
+  }
+  const int64_t T = n / nb;
+  // tile residency check (TILED_2DBC): every lower tile on its owner's device
+  std::vector<uintptr_t> ptrs;
+  if (A_desc->kind == STF_DESC_TILED_2DBC) {
+    ptrs.reserve((size_t)(T * (T + 1) / 2));
+    for (int64_t j = 0; j < T; ++j)
+      for (int64_t i = j; i < T; ++i) {
+        const double* tp = A_desc->tiles[(size_t)(i + j * T)];
+        const int own = (int)((i % P) * Q + (j % Q));
+        int d = -1;
+        if (!tp || !device_of(tp, &d) || d != C.slots[(size_t)own].device)
+          return fail(-4, "tile (%lld,%lld) is not device memory on slot %d (device %d)", (long long)i, (long long)j,
+                      own, C.slots[(size_t)own].device);
+        if (reinterpret_cast<uintptr_t>(tp) & 15) return fail(-4, "tile (%lld,%lld) not 16-byte aligned", (long long)i, (long long)j);
+        ptrs.push_back(reinterpret_cast<uintptr_t>(tp));
+      }
+  }
+  // memo lookup
+  Exec* X = nullptr;
+  bool hit = false;
+  for (auto it = C.cache.begin(); it != C.cache.end(); ++it) {
+    Exec& e = **it;
+    if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
+        e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
+        (e.opt.graph == C.opt.graph || A_desc->kind == STF_DESC_HOST_COLMAJOR) &&
+        e.opt.priority == C.opt.priority && e.key_ptrs == ptrs &&
+        (A_desc->kind == STF_DESC_TILED_2DBC ||
+         (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
+      C.cache.splice(C.cache.begin(), C.cache, it);
+      X = C.cache.front().get();
+      hit = true;
+      break;
+    }
+  }
+  if (!X) {
+    while (C.cache.size() >= kCacheMax) C.cache.pop_back();
+    std::unique_ptr<Exec> e(new Exec());
+    e->n = n;
+    e->nb = nb;
+    e->uplo = up;
+    e->kind = A_desc->kind;
+    e->ngpus = ngpus;
+    e->P = P;
+    e->Q = Q;
+    e->opt = C.opt;
+    e->key_ptrs = ptrs;
+    e->key_ld = A_desc->ld;
+    e->key_dev = A_desc->device;
+    if (A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr)) e->opt.graph = 0;  // pageable: no capture
+    int r = prepare(C, *e, A_desc);
+    if (r == -103 && !C.cache.empty()) {  // out of memory: drop memoised plans and retry once
+      C.cache.clear();
+      e.reset(new Exec());
+      e->n = n; e->nb = nb; e->uplo = up; e->kind = A_desc->kind; e->ngpus = ngpus; e->P = P; e->Q = Q;
+      e->opt = C.opt; e->key_ptrs = ptrs; e->key_ld = A_desc->ld; e->key_dev = A_desc->device;
+      if (A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr)) e->opt.graph = 0;
+      g_err.clear();
+      r = prepare(C, *e, A_desc);
+    }
+    if (r) return r;
+    C.cache.push_front(std::move(e));
+    X = C.cache.front().get();
+  }
+  int info = run(C, *X);
+  fill_stats(*X, hit, &C.last);
+  C.last.device_ms = C.device_ms;
+  if (info < 0) {
+    // a failed call leaves device state unknown: drop the plan
+    C.cache.remove_if([&](const std::unique_ptr<Exec>& p) { return p.get() == X; });
+  }
+  return info;
+}
+
+int stf_last_stats(stf_plan_stats* out) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  if (!out) return fail(-105, "NULL stats pointer");
+  *out = C.last;
+  return 0;
+}
+
+int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t cap_tasks, int32_t* kinds,
+                  int64_t* ijk, stf_plan_stats* stats) {
+  g_err.clear();
+  if (T < 0) return fail(-1, "T < 0");
+  if (p < 1 || q < 1) return fail(-4, "bad grid %dx%d", p, q);
+  Options o;
+  o.priority = 1;
+  stf::Plan plan;
+  auto t0 = std::chrono::steady_clock::now();
+  stf::build_plan(plan, T, plan_options(o, p, q, p * q, false, false));
+  double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  int64_t e = 0;
+  for (int64_t t = 0; t < plan.graph.ntasks(); ++t)
+    for (const int64_t* x = plan.graph.preds_begin(t); x != plan.graph.preds_end(t); ++x, ++e)
+      if (edges && e < cap) {
+        edges[2 * e] = *x;
+        edges[2 * e + 1] = t;
+      }
+  for (size_t t = 0; t < plan.tasks.size() && (int64_t)t < cap_tasks; ++t) {
+    if (kinds) kinds[t] = plan.tasks[t].kind;
+    if (ijk) {
+      ijk[3 * t] = plan.tasks[t].i;
+      ijk[3 * t + 1] = plan.tasks[t].j;
+      ijk[3 * t + 2] = plan.tasks[t].k;
+    }
+  }
+  if (stats) {
+    int64_t compute = 0;
+    for (const auto& t : plan.tasks) compute += (t.kind <= stf::K_GEMM);
+    stats->tasks = compute;
+    stats->transfers = plan.ntransfers;
+    stats->edges = plan.graph.nedges();
+    stats->transfer_bytes = 0;
+    stats->critical_path = plan.critical_path;
+    stats->graph_nodes = 0;
+    stats->kernel_launches = 0;
+    stats->build_ms = ms;
+    stats->device_ms = 0;
+  }
+  return 0;
+}
+
+int64_t stf_infer_edges(int64_t ntasks, const int32_t* nacc, const int64_t* data, const int32_t* modes, int64_t cap,
+                        int64_t* edges) {
+  g_err.clear();
+  if (ntasks < 0 || (ntasks > 0 && (!nacc || !data || !modes))) return fail(-4, "bad arguments");
+  stf::TaskGraph G(0);
+  int64_t off = 0;
+  std::vector<stf::Access> acc;
+  for (int64_t t = 0; t < ntasks; ++t) {
+    acc.clear();
+    for (int32_t a = 0; a < nacc[t]; ++a) {
+      const int32_t m = modes[off + a];
+      if (m < 1 || m > 3) return fail(-4, "bad access mode %d", m);
+      acc.push_back(stf::Access{data[off + a], (uint8_t)m});
+    }
+    off += nacc[t];
+    G.submit(acc.data(), (int)acc.size());
+  }
+  int64_t e = 0;
+  for (int64_t t = 0; t < ntasks; ++t)
+    for (const int64_t* x = G.preds_begin(t); x != G.preds_end(t); ++x, ++e)
+      if (edges && e < cap) {
+        edges[2 * e] = *x;
+        edges[2 * e + 1] = t;
+      }
+  return e;
+}
+
+int stf_fill_spd_tiles(int64_t n, int64_t nb, const stf_matrix_desc* A_desc, int ngpus, uint64_t seed) {
+  g_err.clear();
+  if (!A_desc || A_desc->kind != STF_DESC_TILED_2DBC || nb < 1 || n % nb || !A_desc->tiles)
+    return fail(-4, "stf_fill_spd_tiles needs a TILED_2DBC descriptor");
+  const int64_t T = n / nb;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  std::vector<int> devs;
+  for (int64_t j = 0; j < T; ++j)
+    for (int64_t i = j; i < T; ++i) {
+      double* tp = A_desc->tiles[(size_t)(i + j * T)];
+      int d = 0;
+      if (!device_of(tp, &d)) return fail(-4, "tile (%lld,%lld) is not device memory", (long long)i, (long long)j);
+      cudaSetDevice(d);
+      CUDA_TRY(stfk::fill_spd(0, tp, nb, n, i * nb, j * nb, (int)nb, (int)nb, seed), "fill_spd");
+      if (std::find(devs.begin(), devs.end(), d) == devs.end()) devs.push_back(d);
+    }
+  for (int d : devs) {
+    cudaSetDevice(d);
+    CUDA_TRY(cudaDeviceSynchronize(), "fill_spd sync");
+  }
+  cudaSetDevice(cur);
+  (void)ngpus;
+  return 0;
+}
+
+int stf_fill_spd_block(double* dst, int64_t ld, int64_t n, int64_t r0, int64_t c0, int64_t rows, int64_t cols,
+                       uint64_t seed) {
+  g_err.clear();
+  if (!dst || ld < rows || rows < 0 || cols < 0) return fail(-4, "bad block arguments");
+  CUDA_TRY(stfk::fill_spd(0, dst, ld, n, r0, c0, (int)rows, (int)cols, seed), "fill_spd");
+  CUDA_TRY(cudaStreamSynchronize(0), "fill_spd sync");
+  return 0;
+}
+
+int stf_kernel_gemm_nt(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B, int64_t ldb,
+                       double* C, int64_t ldc, int lower) {
+  g_err.clear();
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int r = ensure_kernel_attrs(dev);
+  if (r) return r;
+  if (lower && M != N) return fail(-4, "lower (SYRK) mode needs M == N");
+  CUDA_TRY(stfk::gemm_nt(0, 0, (int)M, (int)N, (int)K, A, lda, B, ldb, C, ldc, lower), "gemm_nt");
+  CUDA_TRY(cudaStreamSynchronize(0), "gemm_nt sync");
+  return 0;
+}
+
+int stf_kernel_trsm(int64_t M, int64_t n, const double* L, int64_t ldl, double* B, int64_t ldb) {
+  g_err.clear();
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int r = ensure_kernel_attrs(dev);
+  if (r) return r;
+  CUDA_TRY(stfk::trsm_rlt(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm");
+  CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
+  return 0;
+}
+
+int stf_kernel_potrf(int64_t n, double* A, int64_t lda, int64_t* info) {
+  g_err.clear();
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int r = ensure_kernel_attrs(dev);
+  if (r) return r;
+  unsigned long long* d_info = nullptr;
+  CUDA_TRY(cudaMalloc(&d_info, sizeof *d_info), "info alloc");
+  cudaError_t e = stfk::info_reset(0, d_info);
+  if (e == cudaSuccess) e = stfk::potrf_lower(0, 0, (int)n, A, lda, 0, d_info);
+  unsigned long long v = ULLONG_MAX;
+  if (e == cudaSuccess) e = cudaMemcpy(&v, d_info, sizeof v, cudaMemcpyDeviceToHost);
+  cudaFree(d_info);
+  if (e != cudaSuccess) return cuda_fail(e, "potrf");
+  if (info) *info = (v == ULLONG_MAX) ? 0 : (int64_t)v;
+  return 0;
+}
+
+int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double* avg_ms) {
+  g_err.clear();
+  if (kind < 0 || kind > 3 || M < 1 || reps < 1 || !avg_ms) return fail(-4, "bad stf_bench_kernel arguments");
+  if (kind == 1 || kind == 3) N = M;
+  if (kind == 2) K = N;
+  if (kind == 3) K = M;
+  if (N < 1 || K < 1) return fail(-4, "bad sizes");
+  const int64_t ldm = M + (M & 1), ldn = N + (N & 1);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int r = ensure_kernel_attrs(dev);
+  if (r) return r;
+  double *A = nullptr, *B = nullptr, *Cm = nullptr, *Src = nullptr;
+  unsigned long long* info = nullptr;
+  cudaStream_t s = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  double total = 0;
+  cudaError_t e = cudaSuccess;
+  auto step = [&](cudaError_t x) { if (e == cudaSuccess) e = x; };
+  step(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  step(cudaEventCreate(&e0));
+  step(cudaEventCreate(&e1));
+  step(cudaMalloc(&A, (size_t)(ldm * K) * 8));
+  step(cudaMalloc(&B, (size_t)(ldn * std::max(K, N)) * 8));
+  step(cudaMalloc(&Cm, (size_t)(ldm * N) * 8));
+  step(cudaMalloc(&Src, (size_t)(ldm * N) * 8));
+  step(cudaMalloc(&info, sizeof *info));
+  if (e == cudaSuccess) {
+    // operands: SPD generator blocks (well scaled); L for TRSM = the lower part of an SPD block is fine
+    step(stfk::fill_spd(s, A, ldm, M + K, 0, 0, (int)M, (int)K, 11));
+    step(stfk::fill_spd(s, B, ldn, std::max(N, K), 0, 0, (int)N, (int)std::max(K, N), 12));
+    step(stfk::fill_spd(s, Src, ldm, M, 0, 0, (int)M, (int)N, 13));
+    step(cudaMemcpyAsync(Cm, Src, (size_t)(ldm * N) * 8, cudaMemcpyDeviceToDevice, s));
+    step(stfk::info_reset(s, info));
+    for (int it = 0; it < reps + 1 && e == cudaSuccess; ++it) {  // first launch = warm-up
+      if (kind == 3 || kind == 2) step(cudaMemcpyAsync(Cm, Src, (size_t)(ldm * N) * 8, cudaMemcpyDeviceToDevice, s));
+      step(cudaEventRecord(e0, s));
+      switch (kind) {
+        case 0: step(stfk::gemm_nt(s, 0, (int)M, (int)N, (int)K, A, ldm, B, ldn, Cm, ldm, 0)); break;
+        case 1: step(stfk::gemm_nt(s, 0, (int)M, (int)M, (int)K, A, ldm, A, ldm, Cm, ldm, 1)); break;
+        case 2: step(stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)); break;
+        case 3: step(stfk::potrf_lower(s, 0, (int)M, Cm, ldm, 0, info)); break;
+      }
+      step(cudaEventRecord(e1, s));
+      step(cudaEventSynchronize(e1));
+      float ms = 0;
+      step(cudaEventElapsedTime(&ms, e0, e1));
+      if (it > 0) total += ms;
+    }
+  }
+  cudaFree(A); cudaFree(B); cudaFree(Cm); cudaFree(Src); cudaFree(info);
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (s) cudaStreamDestroy(s);
+  if (e != cudaSuccess) return cuda_fail(e, "stf_bench_kernel");
+  *avg_ms = total / reps;
+  return 0;
+}
+
+}  // extern "C"

@@ -1,0 +1,91 @@
+"""C-ABI boundary checks that need no GPU: the library loads, exports every
+symbol include/stf_cholesky.h declares, and validates arguments LAPACK-style
+before touching any device."""
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+import paper_conf_sc_augonnetasg24_b200 as stf
+from paper_conf_sc_augonnetasg24_b200 import _abi
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "stf_cholesky.h")
+
+
+def header_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(stf_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_header_declares_the_planned_boundary():
+    fns = header_functions()
+    for f in ("stf_cholesky_init", "stf_potrf", "stf_finalize", "stf_last_error"):
+        assert f in fns
+
+
+def test_library_exports_every_declared_symbol():
+    out = subprocess.run(["nm", "-D", "--defined-only", _abi.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (stf_[a-z_0-9]+)", out))
+    missing = [f for f in header_functions() if f not in exported]
+    assert not missing, missing
+    assert sorted(_abi.EXPORTS) == header_functions()
+
+
+def test_library_has_sm100a_code():
+    out = subprocess.run(["cuobjdump", "--list-elf", _abi.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def _desc_host(ptr=None, ld=4):
+    return _abi.stf_matrix_desc(stf.STF_DESC_HOST_COLMAJOR, 0, ld, ptr, 0, 0, None)
+
+
+@pytest.mark.parametrize(
+    "n,nb,uplo,code",
+    [(-1, 2, b"L", -1), (4, 0, b"L", -2), (4, 3, b"L", -2), (6, 4, b"L", -2), (4, 2, b"X", -3)],
+)
+def test_argument_validation_without_gpu(n, nb, uplo, code):
+    buf = (ctypes.c_double * 64)()
+    d = _desc_host(ctypes.cast(buf, ctypes.c_void_p), ld=8)
+    assert _abi.stf_potrf(n, nb, uplo, ctypes.byref(d), 1) == code
+    assert len(_abi.stf_last_error()) > 0
+
+
+def test_bad_descriptor_codes():
+    assert _abi.stf_potrf(4, 2, b"L", None, 1) == -4
+    buf = (ctypes.c_double * 64)()
+    d = _desc_host(ctypes.cast(buf, ctypes.c_void_p), ld=2)  # ld < n
+    assert _abi.stf_potrf(4, 2, b"L", ctypes.byref(d), 1) == -4
+    d = _abi.stf_matrix_desc(7, 0, 4, None, 0, 0, None)
+    assert _abi.stf_potrf(4, 2, b"L", ctypes.byref(d), 1) == -4
+    # TILED requires uplo L and p*q == ngpus
+    d = _abi.stf_matrix_desc(stf.STF_DESC_TILED_2DBC, 0, 0, None, 1, 2, None)
+    assert _abi.stf_potrf(4, 2, b"U", ctypes.byref(d), 2) == -3
+    assert _abi.stf_potrf(4, 2, b"L", ctypes.byref(d), 1) == -4
+
+
+def test_not_initialised_and_n_zero_order():
+    buf = (ctypes.c_double * 64)()
+    d = _desc_host(ctypes.cast(buf, ctypes.c_void_p), ld=8)
+    assert _abi.stf_potrf(4, 2, b"L", ctypes.byref(d), 0) == -5
+    assert _abi.stf_finalize() == -100
+
+
+def test_init_without_gpu_fails_cleanly():
+    from conftest import gpu_available
+    if gpu_available():
+        pytest.skip("GPU present")
+    assert _abi.stf_cholesky_init(1, None) == -101
+    assert b"CUDA" in _abi.stf_last_error() or b"device" in _abi.stf_last_error()
+
+
+def test_options_roundtrip_without_gpu():
+    stf.set_option("serial", 1)
+    assert stf.get_option("serial") == 1
+    stf.set_option("serial", 0)
+    with pytest.raises(stf.StfError):
+        stf.set_option("nonsense", 1)

@@ -1,0 +1,244 @@
+"""Parity of the full STF Cholesky path (stf_potrf through the C ABI) against
+the CPU oracle, plus the exact pins of SURVEY.md §8(c) through the GPU
+pipeline, determinism across schedules / grids, COLMAJOR descriptors and info.
+
+Gate (north_star): ||L_gpu - L_ref||_F / ||L_ref||_F <= 1e-10 and backward
+error ||A - L L^T||_F / (||A||_F n eps) <= 10."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from gpu_util import backward_ratio, relF
+
+pytestmark = pytest.mark.gpu
+
+NSLOTS = 8  # slots 0..7 all on cuda:0 ("virtual GPUs")
+
+
+@pytest.fixture(scope="module")
+def stf():
+    import paper_conf_sc_augonnetasg24_b200 as s
+    s.init(NSLOTS, [0] * NSLOTS)
+    yield s
+    s.finalize()
+
+
+def _options(stf, **kw):
+    for k, v in kw.items():
+        stf.set_option(k, v)
+
+
+@pytest.fixture(autouse=True)
+def _reset_options(request):
+    yield
+    if "stf" in request.fixturenames:
+        s = request.getfixturevalue("stf")
+        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0)
+
+
+def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
+    M = stf.TiledMatrix(n, nb, p, q, devices=[0] * (p * q))
+    M.fill_spd(seed)
+    info = M.potrf()
+    return M, info
+
+
+# ---------------------------------------------------------------- parity vs oracle
+@pytest.mark.parametrize("n,nb", [(1024, 256), (576, 192), (480, 96), (200, 100), (2048, 512), (256, 256)])
+def test_parity_metric_inputs(stf, n, nb):
+    M, info = _factor_spd(stf, n, nb, seed=1)
+    assert info == 0
+    L = M.to_dense().numpy()
+    A = synth.spd_matrix(1, n)
+    Lo, oinfo = oracle.potrf(A)
+    assert oinfo == 0
+    assert relF(L, Lo) <= 1e-10
+    assert backward_ratio(A, L) <= 10
+
+
+@pytest.fixture(scope="module")
+def oracle_8192():
+    A = synth.spd_matrix(1, 8192)
+    L, info = oracle.potrf(A)
+    assert info == 0
+    return A, L
+
+
+@pytest.mark.parametrize("nb", [256, 512, 1024])
+def test_parity_cfg1_nb_sweep(stf, oracle_8192, nb):
+    A, Lo = oracle_8192
+    M, info = _factor_spd(stf, 8192, nb, seed=1)
+    assert info == 0
+    L = M.to_dense().numpy()
+    assert relF(L, Lo) <= 1e-10
+    assert backward_ratio(A, L) <= 10
+
+
+# ---------------------------------------------------------------- exact pins through the GPU path
+def _factor_dense(stf, A, nb, p=1, q=1):
+    import torch
+
+    n = A.shape[0]
+    M = stf.TiledMatrix(n, nb, p, q, devices=[0] * (p * q))
+    M.load_dense(torch.from_numpy(np.ascontiguousarray(A)))
+    info = M.potrf()
+    return M.to_dense().numpy(), info
+
+
+@pytest.mark.parametrize("n,nb", [(512, 128), (1024, 256), (384, 96)])
+def test_p1_min_matrix_bit_exact(stf, n, nb):
+    L, info = _factor_dense(stf, synth.min_matrix(n), nb)
+    assert info == 0 and np.array_equal(L, np.tril(np.ones((n, n))))
+
+
+@pytest.mark.parametrize("n,nb,p,q", [(1024, 256, 1, 1), (2048, 256, 2, 2), (1024, 128, 1, 2)])
+def test_p2_dyadic_bit_exact(stf, n, nb, p, q):
+    A, L0 = synth.dyadic_spd(101, n)
+    L, info = _factor_dense(stf, A, nb, p, q)
+    assert info == 0 and np.array_equal(L, L0)
+
+
+def test_p3_diagonal_bit_exact(stf):
+    A = synth.diag_matrix(5, 768)
+    L, info = _factor_dense(stf, A, 256)
+    assert info == 0 and np.array_equal(L, np.diag(np.sqrt(np.diag(A))))
+
+
+@pytest.mark.parametrize("rho,tol", [(0.5, 1e-13), (0.9, 1e-12)])
+def test_p6_kms(stf, rho, tol):
+    n = 1024
+    L, info = _factor_dense(stf, synth.kms_matrix(n, rho), 256)
+    assert info == 0
+    i = np.arange(n)
+    Lref = np.where(i[:, None] >= i[None, :], rho ** (i[:, None] - i[None, :]).clip(0).astype(float), 0.0)
+    Lref[1:, 1:] *= np.sqrt(1 - rho * rho)
+    assert relF(L, Lref) <= tol
+
+
+@pytest.mark.parametrize("j", [0, 255, 256, 1023])
+def test_p10_info_at_tile_boundaries(stf, j):
+    A = synth.spd_matrix(1, 1024)
+    A[j, j] = -1.0
+    _, info = _factor_dense(stf, A, 256)
+    assert info == j + 1
+
+
+def test_info_on_other_grid_slot(stf):
+    A = synth.spd_matrix(1, 1024)
+    A[700, 700] = -1.0  # tile (2,2) -> slot 0 on 2x2... and column 700 on slot (2%2)*2+2%2
+    _, info = _factor_dense(stf, A, 256, 2, 2)
+    assert info == 701
+
+
+# ---------------------------------------------------------------- determinism / race checks (P9)
+def _bits(stf, n, nb, p=1, q=1, seed=3, **opts):
+    _options(stf, **opts)
+    M, info = _factor_spd(stf, n, nb, p, q, seed)
+    assert info == 0
+    out = M.to_dense().numpy().copy()
+    _options(stf, graph=1, serial=0, priority=1, streams=8)
+    return out
+
+
+def test_bit_stable_runs_and_schedules(stf):
+    n, nb = 2048, 256
+    ref = _bits(stf, n, nb)
+    assert np.array_equal(ref, _bits(stf, n, nb))
+    assert np.array_equal(ref, _bits(stf, n, nb, serial=1))
+    assert np.array_equal(ref, _bits(stf, n, nb, graph=0))
+    assert np.array_equal(ref, _bits(stf, n, nb, priority=0, streams=3))
+
+
+@pytest.mark.parametrize("p,q", [(1, 2), (2, 1), (2, 2), (2, 4)])
+def test_bit_equal_across_virtual_grids(stf, p, q):
+    n, nb = 2048, 256
+    ref = _bits(stf, n, nb, 1, 1)
+    assert np.array_equal(ref, _bits(stf, n, nb, p, q))
+    assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0))
+
+
+def test_repeated_calls_reuse_graph(stf):
+    M = stf.TiledMatrix(1024, 256)
+    M.fill_spd(2)
+    assert M.potrf() == 0
+    s1 = stf.last_stats()
+    M.fill_spd(2)
+    assert M.potrf() == 0
+    s2 = stf.last_stats()
+    assert s1["build_ms"] > 0 and s2["build_ms"] == 0
+    assert s2["graph_nodes"] > 0 and s2["kernel_launches"] > 0
+    assert s2["tasks"] == 20 and s2["edges"] == 30
+
+
+# ---------------------------------------------------------------- COLMAJOR descriptors
+@pytest.mark.parametrize("where", ["device", "host_pinned", "host_pageable"])
+@pytest.mark.parametrize("order", ["F", "C"])
+@pytest.mark.parametrize("ngpus", [1, 4])
+def test_colmajor_descriptors(stf, where, order, ngpus):
+    import torch
+
+    n, nb = 768, 128
+    A = synth.spd_matrix(4, n)
+    A[np.triu_indices(n, 1)] = 12345.0  # the other triangle: must come back untouched
+    if order == "F":
+        base = np.asfortranarray(A)
+    else:
+        base = np.ascontiguousarray(A)
+    if where == "device":
+        t = torch.from_numpy(np.ascontiguousarray(base.T if order == "F" else base)).cuda()
+        if order == "F":
+            t = t.t()  # column-major view of A
+    else:
+        t = torch.from_numpy(np.ascontiguousarray(base.T if order == "F" else base))
+        if where == "host_pinned":
+            t = t.pin_memory()
+        if order == "F":
+            t = t.t()
+    info = stf.potrf(t, nb, ngpus=ngpus)
+    assert info == 0
+    got = t.cpu().numpy()
+    Lo, _ = oracle.potrf(synth.spd_matrix(4, n))
+    assert relF(np.tril(got), Lo) <= 1e-10
+    assert np.all(got[np.triu_indices(n, 1)] == 12345.0)
+
+
+def test_n_zero(stf):
+    import torch
+
+    t = torch.zeros((1, 1), dtype=torch.float64, device="cuda")
+    assert stf.potrf_colmajor(t.data_ptr(), 0, 1, 2, "L", 0) == 0
+
+
+# ---------------------------------------------------------------- full-size sampled parity
+@pytest.mark.parametrize("n,nb,m", [(32768, 1024, 4096)])
+def test_bench_config_leading_block_and_residual(stf, n, nb, m):
+    """At the bench's full size: the leading m x m block of L is the Cholesky
+    factor of A[:m,:m] (oracle computes it), and sampled rows of L L^T match A."""
+    import torch
+
+    M, info = _factor_spd(stf, n, nb, seed=1)
+    assert info == 0
+    T = n // nb
+    mb = m // nb
+    Llead = np.zeros((m, m))
+    for (i, j), t in M.tiles.items():
+        if i < mb and j < mb:
+            Llead[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb] = t.T.cpu().numpy()
+    Llead = np.tril(Llead)
+    Lo, _ = oracle.potrf(synth.spd_block(1, n, 0, 0, m, m))
+    assert relF(Llead, Lo) <= 1e-10
+    # sampled rows: (L L^T)[r, :] = sum_k L[r, k] L[:, k]  vs  A[r, :]   (torch fp64 on GPU, harness only)
+    rng = np.random.default_rng(0)
+    rows = sorted(rng.choice(n, size=8, replace=False).tolist())
+    Ld = torch.zeros((n, n), dtype=torch.float64, device="cuda")
+    for (i, j), t in M.tiles.items():
+        Ld[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb] = t.T
+    Ld = torch.tril(Ld)
+    for r in rows:
+        got = (Ld[r:r + 1, :] @ Ld.T).cpu().numpy()[0]
+        Arow = synth.spd_block(1, n, r, 0, 1, n)[0]
+        err = np.linalg.norm(got - Arow) / (np.linalg.norm(Arow) * n * np.finfo(float).eps)
+        assert err <= 10
+    del Ld
+    assert T == n // nb
