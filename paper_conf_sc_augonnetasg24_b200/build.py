@@ -25,6 +25,7 @@ COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler",
 SOURCES = [
     "kernels/gemm_dmma.cu",
     "kernels/panel.cu",
+    "kernels/dataflow.cu",
     "plan.cpp",
     "runtime.cpp",
 ]

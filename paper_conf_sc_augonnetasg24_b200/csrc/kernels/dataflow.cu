@@ -1,0 +1,430 @@
+// K3 TRSM and K4 POTRF of one tile as single-launch, device-side dataflow
+// kernels (the STF idea of PAPER.md:144 applied inside a
+// tile: block tasks run as soon as the blocks they read are final).
+//
+// Task definitions (right-looking tiled Cholesky of [17]):
+//   POTRF on an n x n tile, 64 x 64 blocks (ib, jb), ib >= jb:
+//     P(kb)        X_kk <- chol(X_kk)                         (block Cholesky, in smem)
+//     S(ib,kb)     X_ik <- X_ik X_kk^-T                      (substitution, in smem)
+//     U(ib,jb,kb)  X_ij <- X_ij - X_ik X_jk^T                (DMMA, lower part only if ib == jb)
+//   TRSM X[m x n] <- X L^-T, L n x n lower:
+//     S(ib,jb)     X_ij <- X_ij L_jj^-T
+//     U(ib,jb,pb)  X_ij <- X_ij - X_ip L_jp^T   (pb < jb)
+//
+// Scheduling: the host writes the task list once per block-grid shape, in a
+// topological order with a look-ahead of one column (the next panel's column
+// is updated first).  Every CTA repeatedly takes the next ticket from an atomic
+// counter, waits (acquire) until the progress counters of the blocks the task
+// reads have reached the required values, runs the task, and publishes
+// (release) the new progress of the block it wrote.  A CTA only ever waits for
+// tasks with smaller tickets, which were claimed by CTAs that are already
+// running, so the scheme cannot deadlock whatever the grid size or how many
+// CTAs are co-resident.  Progress of block (ib,jb) = number of operations
+// completed on it; it is final when progress == jb + 1.
+//
+// Operations on every block happen in a fixed order (updates by increasing k,
+// then the final P/S), so results are bit-identical run to run.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstdint>
+#include <map>
+#include <mutex>
+#include <tuple>
+#include <vector>
+
+#include "ptx.cuh"
+#include "tile_ops.hpp"
+
+namespace stfk {
+
+namespace df {
+constexpr int W = 64;       // block order
+constexpr int LDO = 68;     // smem stride of DMMA operand blocks [k][row] (68 = 4 mod 16: conflict-free)
+constexpr int LDB = 65;     // smem stride of substitution / Cholesky blocks [row][col]
+constexpr int NT = 256;
+constexpr int SMEM_BYTES = 2 * W * LDO * 8;  // 69,632 B
+enum : uint32_t { T_P = 0, T_S = 1, T_U = 2 };
+
+__host__ __device__ inline uint32_t enc(uint32_t t, uint32_t i, uint32_t j, uint32_t k) {
+  return (t << 30) | (i << 20) | (j << 10) | k;
+}
+}  // namespace df
+
+struct DfParams {
+  double* X;
+  int64_t ldx;
+  const double* L;  // TRSM: the triangular factor; POTRF: unused (X itself)
+  int64_t ldl;
+  int m, n;    // X is m x n
+  int Mb, Nb;  // block grid of X
+  const uint32_t* tasks;
+  int ntasks;
+  int* ws;  // ws[0] ticket, ws[1 + ib * Nb + jb] progress
+  int64_t col0;
+  unsigned long long* info;
+  int potrf;
+};
+
+__device__ __forceinline__ int ld_acquire(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(int* p, int v) {
+  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void wait_geq(const int* p, int v) {
+  int ns = 32;
+  while (ld_acquire(p) < v) {
+    __nanosleep(ns);
+    if (ns < 256) ns <<= 1;
+  }
+}
+
+// smem S[c * ld + r] = G(r0 + r, c0 + c) for r < rows, c < cols; zero elsewhere (W x W)
+__device__ __forceinline__ void load_block_cm(double* S, int ld, const double* G, int64_t ldg, int rows, int cols) {
+  for (int idx = threadIdx.x; idx < df::W * df::W; idx += df::NT) {
+    const int r = idx & (df::W - 1), c = idx >> 6;
+    S[c * ld + r] = (r < rows && c < cols) ? __ldcg(G + (int64_t)c * ldg + r) : 0.0;
+  }
+}
+// smem S[r * ld + c] = G(r, c)  (row-major in smem)
+__device__ __forceinline__ void load_block_rm(double* S, int ld, const double* G, int64_t ldg, int rows, int cols,
+                                              bool lower_only) {
+  for (int idx = threadIdx.x; idx < df::W * df::W; idx += df::NT) {
+    const int r = idx & (df::W - 1), c = idx >> 6;
+    double v = 0.0;
+    if (r < rows && c < cols && (!lower_only || r >= c)) v = __ldcg(G + (int64_t)c * ldg + r);
+    S[r * ld + c] = v;
+  }
+}
+__device__ __forceinline__ void store_block_rm(const double* S, int ld, double* G, int64_t ldg, int rows, int cols,
+                                               bool lower_only) {
+  for (int idx = threadIdx.x; idx < df::W * df::W; idx += df::NT) {
+    const int r = idx & (df::W - 1), c = idx >> 6;
+    if (r < rows && c < cols && (!lower_only || r >= c)) G[(int64_t)c * ldg + r] = S[r * ld + c];
+  }
+}
+
+__device__ __forceinline__ double negd(double x) {
+  return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
+}
+
+// U: C[rows x cols] -= A[rows x K] * B[cols x K]^T, K <= 64; lower: keep r >= c only
+__device__ void task_update(double* sm, double* C, int64_t ldc, const double* A, int64_t lda, const double* B,
+                            int64_t ldb, int rows, int cols, int K, bool lower) {
+  double* As = sm;
+  double* Bs = sm + df::W * df::LDO;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const int wm0 = (warp & 1) * 32, wn0 = (warp >> 1) * 16;
+  double acc[4][2][2];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 2; ++j)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int r = wm0 + 8 * i + g, c = wn0 + 8 * j + 2 * t + h;
+        acc[i][j][h] = (r < rows && c < cols && (!lower || r >= c)) ? __ldcg(C + (int64_t)c * ldc + r) : 0.0;
+      }
+  load_block_cm(As, df::LDO, A, lda, rows, K);   // As[k][r]
+  load_block_cm(Bs, df::LDO, B, ldb, cols, K);   // Bs[k][c]
+  __syncthreads();
+#pragma unroll 4
+  for (int k0 = 0; k0 < df::W; k0 += 4) {
+    double a[4], b[2];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) a[i] = As[(k0 + t) * df::LDO + wm0 + 8 * i + g];
+#pragma unroll
+    for (int j = 0; j < 2; ++j) b[j] = negd(Bs[(k0 + t) * df::LDO + wn0 + 8 * j + g]);
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i], b[j]);
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 2; ++j)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int r = wm0 + 8 * i + g, c = wn0 + 8 * j + 2 * t + h;
+        if (r < rows && c < cols && (!lower || r >= c)) C[(int64_t)c * ldc + r] = acc[i][j][h];
+      }
+}
+
+// S: X[rows x nc] <- X L^-T, L nc x nc lower (substitution, column by column)
+__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc) {
+  double* Bs = sm;                    // Bs[r][c]
+  double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
+  load_block_rm(Bs, df::LDB, X, ldx, rows, nc, false);
+  load_block_rm(Ls, df::LDB, L, ldl, nc, nc, true);
+  __syncthreads();
+  const int r = threadIdx.x & (df::W - 1), ty = threadIdx.x >> 6;
+  for (int c = 0; c < nc; ++c) {
+    if (threadIdx.x < rows) Bs[threadIdx.x * df::LDB + c] = Bs[threadIdx.x * df::LDB + c] / Ls[c * df::LDB + c];
+    __syncthreads();
+    if (r < rows) {
+      const double x = Bs[r * df::LDB + c];
+      for (int c2 = c + 1 + ty; c2 < nc; c2 += 4)
+        Bs[r * df::LDB + c2] = fma(-x, Ls[c2 * df::LDB + c], Bs[r * df::LDB + c2]);
+    }
+    __syncthreads();
+  }
+  store_block_rm(Bs, df::LDB, X, ldx, rows, nc, false);
+}
+
+// P: in-place lower Cholesky of the nc x nc diagonal block (right-looking, in smem)
+__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
+  double* S = sm;  // S[r][c]
+  load_block_rm(S, df::LDB, X, ldx, nc, nc, true);
+  __syncthreads();
+  const int r = threadIdx.x & (df::W - 1), ty = threadIdx.x >> 6;
+  for (int j = 0; j < nc; ++j) {
+    if (threadIdx.x == 0) {
+      double s = S[j * df::LDB + j];
+      if (!(s > 0.0)) {
+        atomicMin(info, (unsigned long long)(col0 + j + 1));
+        s = __longlong_as_double(0x7ff8000000000000LL);
+      } else {
+        s = sqrt(s);
+      }
+      S[j * df::LDB + j] = s;
+    }
+    __syncthreads();
+    if (threadIdx.x > j && threadIdx.x < nc) S[threadIdx.x * df::LDB + j] = S[threadIdx.x * df::LDB + j] / S[j * df::LDB + j];
+    __syncthreads();
+    if (r > j && r < nc) {
+      const double l = S[r * df::LDB + j];
+      for (int c = j + 1 + ty; c <= r; c += 4) S[r * df::LDB + c] = fma(-l, S[c * df::LDB + j], S[r * df::LDB + c]);
+    }
+    __syncthreads();
+  }
+  store_block_rm(S, df::LDB, X, ldx, nc, nc, true);
+}
+
+__global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
+  extern __shared__ __align__(16) double sm[];
+  __shared__ int s_task;
+  const int W = df::W;
+  for (;;) {
+    if (threadIdx.x == 0) s_task = atomicAdd(&p.ws[0], 1);
+    __syncthreads();
+    const int ticket = s_task;
+    if (ticket >= p.ntasks) return;
+    const uint32_t code = p.tasks[ticket];
+    const uint32_t type = code >> 30;
+    const int ib = (code >> 20) & 1023, jb = (code >> 10) & 1023, kb = code & 1023;
+    int* prog = p.ws + 1;
+    const int rows = min(W, p.m - ib * W);
+    if (threadIdx.x == 0) {
+      if (p.potrf) {
+        if (type == df::T_P) {
+          wait_geq(&prog[kb * p.Nb + kb], kb);
+        } else if (type == df::T_S) {
+          wait_geq(&prog[kb * p.Nb + kb], kb + 1);
+          wait_geq(&prog[ib * p.Nb + kb], kb);
+        } else {
+          wait_geq(&prog[ib * p.Nb + kb], kb + 1);
+          wait_geq(&prog[jb * p.Nb + kb], kb + 1);
+          wait_geq(&prog[ib * p.Nb + jb], kb);
+        }
+      } else {
+        if (type == df::T_S) {
+          wait_geq(&prog[ib * p.Nb + jb], jb);
+        } else {
+          wait_geq(&prog[ib * p.Nb + kb], kb + 1);
+          wait_geq(&prog[ib * p.Nb + jb], kb);
+        }
+      }
+    }
+    __syncthreads();
+    if (p.potrf) {
+      double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
+      const int nk = min(W, p.n - kb * W);
+      if (type == df::T_P) {
+        task_chol(sm, Xkk, p.ldx, nk, p.col0 + (int64_t)kb * W, p.info);
+      } else if (type == df::T_S) {
+        task_solve(sm, p.X + (int64_t)kb * W * p.ldx + ib * W, p.ldx, Xkk, p.ldx, rows, nk);
+      } else {
+        const int cols = min(W, p.n - jb * W);
+        task_update(sm, p.X + (int64_t)jb * W * p.ldx + ib * W, p.ldx, p.X + (int64_t)kb * W * p.ldx + ib * W, p.ldx,
+                    p.X + (int64_t)kb * W * p.ldx + jb * W, p.ldx, rows, cols, nk, ib == jb);
+      }
+    } else {
+      if (type == df::T_S) {
+        const int nc = min(W, p.n - jb * W);
+        task_solve(sm, p.X + (int64_t)jb * W * p.ldx + ib * W, p.ldx, p.L + (int64_t)jb * W * p.ldl + jb * W, p.ldl,
+                   rows, nc);
+      } else {
+        const int cols = min(W, p.n - jb * W), K = min(W, p.n - kb * W);
+        task_update(sm, p.X + (int64_t)jb * W * p.ldx + ib * W, p.ldx, p.X + (int64_t)kb * W * p.ldx + ib * W, p.ldx,
+                    p.L + (int64_t)kb * W * p.ldl + jb * W, p.ldl, rows, cols, K, false);
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      const int tgt = p.potrf ? (type == df::T_U ? ib * p.Nb + jb : ib * p.Nb + kb) : (ib * p.Nb + jb);
+      st_release(&prog[tgt], kb + 1);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ host side
+namespace {
+
+std::vector<uint32_t> build_tasks(bool potrf, int Mb, int Nb) {
+  std::vector<uint32_t> t;
+  using df::enc;
+  if (potrf) {
+    const int T = Nb;
+    // look-ahead-1 topological order (see header comment)
+    t.push_back(enc(df::T_P, 0, 0, 0));
+    for (int i = 1; i < T; ++i) t.push_back(enc(df::T_S, i, 0, 0));
+    for (int i = 1; i < T; ++i) t.push_back(enc(df::T_U, i, 1, 0));
+    for (int kb = 0; kb + 1 < T; ++kb) {
+      t.push_back(enc(df::T_P, kb + 1, kb + 1, kb + 1));
+      for (int i = kb + 2; i < T; ++i) t.push_back(enc(df::T_S, i, kb + 1, kb + 1));
+      for (int j = kb + 2; j < T; ++j)
+        for (int i = j; i < T; ++i) t.push_back(enc(df::T_U, i, j, kb));
+      if (kb + 2 < T)
+        for (int i = kb + 2; i < T; ++i) t.push_back(enc(df::T_U, i, kb + 2, kb + 1));
+    }
+  } else {
+    for (int i = 0; i < Mb; ++i) t.push_back(enc(df::T_S, i, 0, 0));
+    if (Nb > 1)
+      for (int i = 0; i < Mb; ++i) t.push_back(enc(df::T_U, i, 1, 0));
+    for (int pb = 0; pb + 1 < Nb; ++pb) {
+      for (int i = 0; i < Mb; ++i) t.push_back(enc(df::T_S, i, pb + 1, pb + 1));
+      for (int j = pb + 2; j < Nb; ++j)
+        for (int i = 0; i < Mb; ++i) t.push_back(enc(df::T_U, i, j, pb));
+      if (pb + 2 < Nb)
+        for (int i = 0; i < Mb; ++i) t.push_back(enc(df::T_U, i, pb + 2, pb + 1));
+    }
+  }
+  return t;
+}
+
+std::mutex g_mu;
+std::map<std::tuple<int, int, int, int>, std::pair<uint32_t*, int>> g_tables;  // (dev, potrf, Mb, Nb)
+int g_num_sms[64];
+
+cudaError_t get_table(bool potrf, int Mb, int Nb, const uint32_t** out, int* count) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> g(g_mu);
+  auto key = std::make_tuple(dev, (int)potrf, Mb, Nb);
+  auto it = g_tables.find(key);
+  if (it != g_tables.end()) {
+    *out = it->second.first;
+    *count = it->second.second;
+    return cudaSuccess;
+  }
+  // Must not be called while a stream is being captured (cudaMemcpy); the runtime
+  // calls dataflow_prepare() before capture.
+  std::vector<uint32_t> t = build_tasks(potrf, Mb, Nb);
+  uint32_t* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, t.size() * sizeof(uint32_t));
+  if (e != cudaSuccess) return e;
+  e = cudaMemcpy(d, t.data(), t.size() * sizeof(uint32_t), cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return e;
+  g_tables[key] = {d, (int)t.size()};
+  *out = d;
+  *count = (int)t.size();
+  return cudaSuccess;
+}
+
+int num_sms() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 64 && g_num_sms[dev]) return g_num_sms[dev];
+  int n = 148;
+  cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+  if (dev < 64) g_num_sms[dev] = n;
+  return n;
+}
+
+cudaError_t launch_df(cudaStream_t s, int prio, DfParams& p, int max_ctas) {
+  cudaError_t e = cudaMemsetAsync(p.ws, 0, dataflow_ws_bytes(p.m, p.n), s);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  int grid = p.ntasks < max_ctas ? p.ntasks : max_ctas;
+  if (grid < 1) grid = 1;
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(df::NT);
+  cfg.dynamicSmemBytes = df::SMEM_BYTES;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributePriority;
+  attr[0].val.priority = prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  ++launch_count();
+  return cudaLaunchKernelEx(&cfg, dataflow_kernel, p);
+}
+
+}  // namespace
+
+size_t dataflow_ws_bytes(int m, int n) {
+  const int Mb = (m + df::W - 1) / df::W, Nb = (n + df::W - 1) / df::W;
+  return ((size_t)(1 + Mb * Nb) * sizeof(int) + 255) / 256 * 256;
+}
+
+cudaError_t dataflow_prepare(int m, int n, bool potrf) {
+  const int Mb = (m + df::W - 1) / df::W, Nb = (n + df::W - 1) / df::W;
+  const uint32_t* t;
+  int c;
+  return get_table(potrf, Mb, Nb, &t, &c);
+}
+
+cudaError_t dataflow_init_attrs() {
+  return cudaFuncSetAttribute(dataflow_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, df::SMEM_BYTES);
+}
+
+cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
+                       unsigned long long* info, int* ws) {
+  if (n <= 0) return cudaSuccess;
+  DfParams p{};
+  p.X = A;
+  p.ldx = lda;
+  p.L = nullptr;
+  p.ldl = 0;
+  p.m = p.n = n;
+  p.Mb = p.Nb = (n + df::W - 1) / df::W;
+  cudaError_t e = get_table(true, p.Mb, p.Nb, &p.tasks, &p.ntasks);
+  if (e != cudaSuccess) return e;
+  p.ws = ws;
+  p.col0 = col0;
+  p.info = info;
+  p.potrf = 1;
+  const int T = p.Nb;
+  const int par = T * (T - 1) / 2 > 0 ? T * (T - 1) / 2 : 1;  // widest update wave
+  return launch_df(stream, prio, p, std::min(par, num_sms() / 2));
+}
+
+cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                      int64_t ldb, int* ws) {
+  if (M <= 0 || n <= 0) return cudaSuccess;
+  DfParams p{};
+  p.X = B;
+  p.ldx = ldb;
+  p.L = L;
+  p.ldl = ldl;
+  p.m = M;
+  p.n = n;
+  p.Mb = (M + df::W - 1) / df::W;
+  p.Nb = (n + df::W - 1) / df::W;
+  cudaError_t e = get_table(false, p.Mb, p.Nb, &p.tasks, &p.ntasks);
+  if (e != cudaSuccess) return e;
+  p.ws = ws;
+  p.col0 = 0;
+  p.info = nullptr;
+  p.potrf = 0;
+  const int par = p.Mb * (p.Nb > 1 ? p.Nb - 1 : 1);
+  return launch_df(stream, prio, p, std::min(par, num_sms() / 2));
+}
+
+}  // namespace stfk

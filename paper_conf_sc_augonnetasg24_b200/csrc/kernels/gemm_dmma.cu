@@ -27,6 +27,7 @@
 #include <cudaTypedefs.h>
 
 #include <cstdio>
+#include <cstdlib>
 #include <mutex>
 
 #include "ptx.cuh"
@@ -36,9 +37,6 @@ namespace stfk {
 
 namespace g {
 constexpr int BM = 128, BN = 128, BK = 16, STAGES = 4;
-constexpr int WM = 64, WN = 32;
-constexpr int NCW = (BM / WM) * (BN / WN);  // consumer warps = 8
-constexpr int NTHREADS = NCW * 32;
 constexpr int BOX = 16;                      // doubles per 128-byte swizzle row
 constexpr int BOX_BYTES = BOX * BK * 8;      // 2 KB
 constexpr int A_BYTES = BM * BK * 8;         // 16 KB
@@ -46,6 +44,11 @@ constexpr int B_BYTES = BN * BK * 8;         // 16 KB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 2 * STAGES * 8;
 }  // namespace g
+
+// Exact negation as a sign-bit flip on the integer pipe (keeps the FP64/DMMA pipe free).
+__device__ __forceinline__ double neg(double x) {
+  return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
+}
 
 // Byte offset of element (row r in [0,128), k in [0,16)) inside one operand stage.
 __device__ __forceinline__ uint32_t swz_off(int r, int k) {
@@ -68,11 +71,15 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
 // so the refill of the stage consumed at kt-1 rarely waits).  8 warps keep the
 // register cap at 255/thread (a 9th producer warp would cap it at 168: the
 // register file is split per SM sub-partition and 9 warps round up to 12).
-__global__ void __launch_bounds__(g::NTHREADS, 1)
+template <int WM, int WN>
+__global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         double* __restrict__ C, int64_t ldc, int M, int N, int K, int lower) {
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  constexpr int NCW = (g::BM / WM) * (g::BN / WN);
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  // keep the pointer derived from the __shared__ array (integer offset only) so
+  // the compiler emits LDS, not generic LD, for the fragment loads
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + g::STAGES * g::STAGE_BYTES);
   uint64_t* empty = full + g::STAGES;
 
@@ -98,25 +105,36 @@ __global__ void __launch_bounds__(g::NTHREADS, 1)
     tma_prefetch_desc(&tmB);
     for (int s = 0; s < g::STAGES; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], g::NCW);
+      mbar_init(&empty[s], NCW);
     }
     fence_barrier_init();
     for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage(smem, kt, &tmA, &tmB, m0, n0, kt, full);
   }
   __syncthreads();
 
-  const int wm0 = (warp % (g::BM / g::WM)) * g::WM;
-  const int wn0 = (warp / (g::BM / g::WM)) * g::WN;
+  const int wm0 = (warp % (g::BM / WM)) * WM;
+  const int wn0 = (warp / (g::BM / WM)) * WN;
   const int gq = lane >> 2, tq = lane & 3;
 
   // In lower mode, warps of a diagonal CTA whose warp tile is strictly upper idle.
-  const bool warp_dead = lower && (m0 == n0) && (wm0 + g::WM <= wn0);
+  const bool warp_dead = lower && (m0 == n0) && (wm0 + WM <= wn0);
 
-  double acc[g::WM / 8][g::WN / 8][2];
+  // acc = C, loaded straight into the accumulators (64 independent loads in
+  // flight, latency hidden behind the first TMA wait); the mainloop adds
+  // A * (-B)^T with the B fragments sign-flipped (exact), so acc = C - A B^T.
+  double acc[WM / 8][WN / 8][2];
 #pragma unroll
-  for (int i = 0; i < g::WM / 8; ++i)
+  for (int i = 0; i < WM / 8; ++i) {
+    const int m = m0 + wm0 + 8 * i + gq;
 #pragma unroll
-    for (int j = 0; j < g::WN / 8; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+    for (int j = 0; j < WN / 8; ++j)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int n = n0 + wn0 + 8 * j + 2 * tq + h;
+        const bool in = !warp_dead && m < M && n < N && (!lower || m >= n);
+        acc[i][j][h] = in ? __ldg(C + (int64_t)n * ldc + m) : 0.0;
+      }
+  }
 
   // Per-lane fragment offsets: swz_off(w0 + 8f + gq, 2tq + kh) depends on f only
   // through the box (f >> 1, an immediate) and the chunk bit 2 (f & 1).
@@ -136,23 +154,23 @@ __global__ void __launch_bounds__(g::NTHREADS, 1)
     if (!warp_dead) {
 #pragma unroll
       for (int grp = 0; grp < g::BK / 8; ++grp) {
-        double a[g::WM / 8][2], b[g::WN / 8][2];
+        double a[WM / 8][2], b[WN / 8][2];
 #pragma unroll
-        for (int f = 0; f < g::WM / 8; ++f)
+        for (int f = 0; f < WM / 8; ++f)
 #pragma unroll
           for (int kh = 0; kh < 2; ++kh)
             a[f][kh] = *reinterpret_cast<const double*>(st + offA[f & 1][kh] + (f >> 1) * g::BOX_BYTES + grp * 8 * 128);
 #pragma unroll
-        for (int f = 0; f < g::WN / 8; ++f)
+        for (int f = 0; f < WN / 8; ++f)
 #pragma unroll
           for (int kh = 0; kh < 2; ++kh)
-            b[f][kh] = *reinterpret_cast<const double*>(st + offB[f & 1][kh] + (f >> 1) * g::BOX_BYTES + grp * 8 * 128);
+            b[f][kh] = neg(*reinterpret_cast<const double*>(st + offB[f & 1][kh] + (f >> 1) * g::BOX_BYTES + grp * 8 * 128));
 #pragma unroll
         for (int kh = 0; kh < 2; ++kh)
 #pragma unroll
-          for (int i = 0; i < g::WM / 8; ++i)
+          for (int i = 0; i < WM / 8; ++i)
 #pragma unroll
-            for (int j = 0; j < g::WN / 8; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i][kh], b[j][kh]);
+            for (int j = 0; j < WN / 8; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i][kh], b[j][kh]);
       }
     }
     __syncwarp();
@@ -171,17 +189,14 @@ __global__ void __launch_bounds__(g::NTHREADS, 1)
   if (warp_dead) return;
   // ---------------- epilogue: C -= acc
 #pragma unroll
-  for (int i = 0; i < g::WM / 8; ++i) {
+  for (int i = 0; i < WM / 8; ++i) {
     const int m = m0 + wm0 + 8 * i + gq;
 #pragma unroll
-    for (int j = 0; j < g::WN / 8; ++j) {
+    for (int j = 0; j < WN / 8; ++j) {
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const int n = n0 + wn0 + 8 * j + 2 * tq + h;
-        if (m < M && n < N && (!lower || m >= n)) {
-          double* p = C + (int64_t)n * ldc + m;
-          *p = *p - acc[i][j][h];
-        }
+        if (m < M && n < N && (!lower || m >= n)) C[(int64_t)n * ldc + m] = acc[i][j][h];
       }
     }
   }
@@ -215,6 +230,16 @@ static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int c
   return r == CUDA_SUCCESS;
 }
 
+// 8 warps of 64x32 (224 regs, 2 warps / SM sub-partition) or 16 warps of 32x32
+// (<= 128 regs, 4 warps / sub-partition).  STF_GEMM_WARPS selects; default 16.
+static int gemm_variant() {
+  static int v = [] {
+    const char* e = getenv("STF_GEMM_WARPS");
+    return (e && atoi(e) == 8) ? 8 : 16;
+  }();
+  return v;
+}
+
 cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
                     const double* B, int64_t ldb, double* C, int64_t ldc, int lower) {
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
@@ -229,7 +254,8 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   } else {
     cfg.gridDim = dim3(tM, tN, 1);
   }
-  cfg.blockDim = dim3(g::NTHREADS, 1, 1);
+  const int variant = gemm_variant();
+  cfg.blockDim = dim3(variant == 16 ? 512 : 256, 1, 1);
   cfg.dynamicSmemBytes = g::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
@@ -238,11 +264,16 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   ++launch_count();
-  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel, tmA, tmB, C, ldc, M, N, K, lower);
+  if (variant == 16) return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32>, tmA, tmB, C, ldc, M, N, K, lower);
+  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32>, tmA, tmB, C, ldc, M, N, K, lower);
 }
 
 cudaError_t gemm_init_attrs() {
-  return cudaFuncSetAttribute(gemm_nt_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g::SMEM_BYTES);
+  cudaError_t e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<64, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       g::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, g::SMEM_BYTES);
+  return e;
 }
 
 }  // namespace stfk

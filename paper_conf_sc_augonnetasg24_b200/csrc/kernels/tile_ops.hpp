@@ -32,6 +32,18 @@ cudaError_t trsm_rlt(cudaStream_t stream, int prio, int M, int n, const double* 
 cudaError_t potrf_lower(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                         unsigned long long* info);
 
+// K3/K4 as single-launch device-side dataflow kernels over 64 x 64 blocks
+// (dataflow.cu).  `ws` is a device workspace of dataflow_ws_bytes(m, n) bytes,
+// private to the launch (zeroed by the launcher with a memset on `stream`).
+// dataflow_prepare() uploads the task table for the shape; it must be called
+// once before the first launch of that shape inside a stream capture.
+cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
+                       unsigned long long* info, int* ws);
+cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                      int64_t ldb, int* ws);
+size_t dataflow_ws_bytes(int m, int n);
+cudaError_t dataflow_prepare(int m, int n, bool potrf);
+
 // K8: fill rows r0.., cols c0.. (global indices) of the seeded SPD metric matrix
 // of order n into dst[rows x cols] (ld).  Same SplitMix64 spec as synth/spd.py.
 cudaError_t fill_spd(cudaStream_t stream, double* dst, int64_t ld, int64_t n, int64_t r0, int64_t c0, int rows,

@@ -74,6 +74,7 @@ struct Slot {
 };
 
 struct Options {
+  int64_t dataflow = 1;  // 1: single-launch dataflow POTRF/TRSM tile kernels; 0: recursive (GEMM-based)
   int64_t graph = 1;
   int64_t streams = 8;
   int64_t serial = 0;
@@ -96,6 +97,7 @@ struct Exec {
   std::vector<double*> buf;           // buffer id -> device pointer
   std::vector<std::pair<int, void*>> allocs;  // (device, ptr) library-owned
   std::vector<double*> scratch;       // per (slot, copy stream): staging tile for 'U'
+  std::vector<int*> task_ws;          // per task: dataflow-kernel workspace (POTRF/TRSM), else null
   std::vector<cudaEvent_t> events;    // per task, null if not needed
   std::vector<int> events_dev;
   cudaGraph_t graph = nullptr;
@@ -181,18 +183,27 @@ struct Lowerer {
     return (X.opt.priority && t.prio) ? hi : lo;
   }
 
-  int body(const stf::Task& t, cudaStream_t s, int prio) {
+  int body(const stf::Task& t, size_t tidx, cudaStream_t s, int prio) {
     const int64_t nb = X.nb;
+    int* ws = X.task_ws.empty() ? nullptr : X.task_ws[tidx];
     const size_t tile_bytes = (size_t)(nb * nb) * sizeof(double);
     Slot& S = C.slots[(size_t)t.slot];
     switch (t.kind) {
       case stf::K_POTRF:
-        CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
-                 "POTRF launch");
+        if (X.opt.dataflow)
+          CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws),
+                   "POTRF launch");
+        else
+          CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
+                   "POTRF launch");
         return 0;
       case stf::K_TRSM:
-        CUDA_TRY(stfk::trsm_rlt(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb),
-                 "TRSM launch");
+        if (X.opt.dataflow)
+          CUDA_TRY(stfk::trsm_tile(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, ws),
+                   "TRSM launch");
+        else
+          CUDA_TRY(stfk::trsm_rlt(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb),
+                   "TRSM launch");
         return 0;
       case stf::K_SYRK:
         CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[0]],
@@ -279,7 +290,7 @@ struct Lowerer {
         if (pt.slot == task.slot && pt.stream == task.stream) continue;  // stream order suffices
         CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
       }
-      int r = body(task, s, prio_of(task));
+      int r = body(task, t, s, prio_of(task));
       if (r) return r;
       if (X.events[t]) CUDA_TRY(cudaEventRecord(X.events[t], s), "event record");
     }
@@ -367,6 +378,29 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
     if (nscr) {
       X.scratch.resize((size_t)X.ngpus * kCopyStreams, nullptr);
       for (size_t k = 0; k < nscr; ++k) X.scratch[(size_t)s * kCopyStreams + k] = arena + (used++) * (size_t)(X.nb * X.nb);
+    }
+  }
+  // dataflow-kernel workspaces (one private block per POTRF/TRSM task) and task tables
+  X.task_ws.assign(P.tasks.size(), nullptr);
+  if (X.opt.dataflow) {
+    const size_t wsb = stfk::dataflow_ws_bytes((int)X.nb, (int)X.nb);
+    for (int s = 0; s < X.ngpus; ++s) {
+      size_t cnt = 0;
+      for (const auto& t : P.tasks) cnt += (t.slot == s && (t.kind == stf::K_POTRF || t.kind == stf::K_TRSM));
+      if (!cnt) continue;
+      double* arena = nullptr;
+      int r = alloc_on(X, C.slots[(size_t)s].device, cnt * wsb, &arena);
+      if (r) return r;
+      char* base = reinterpret_cast<char*>(arena);
+      size_t used = 0;
+      for (size_t t = 0; t < P.tasks.size(); ++t) {
+        const stf::Task& tk = P.tasks[t];
+        if (tk.slot == s && (tk.kind == stf::K_POTRF || tk.kind == stf::K_TRSM))
+          X.task_ws[t] = reinterpret_cast<int*>(base + (used++) * wsb);
+      }
+      cudaSetDevice(C.slots[(size_t)s].device);
+      CUDA_TRY(stfk::dataflow_prepare((int)X.nb, (int)X.nb, true), "dataflow tables");
+      CUDA_TRY(stfk::dataflow_prepare((int)X.nb, (int)X.nb, false), "dataflow tables");
     }
   }
   // events only where a successor runs on another stream
@@ -524,6 +558,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   }
   if (ngpus < 1 || ngpus > 64) return fail(-5, "ngpus=%d out of range", ngpus);
   C.opt.graph = env_int("STF_GRAPH", 1);
+  C.opt.dataflow = env_int("STF_DATAFLOW", 1);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.priority = env_int("STF_PRIO", 1);
@@ -631,6 +666,7 @@ int stf_set_option(const char* name, int64_t value) {
   if (!name) return fail(-105, "option name is NULL");
   std::string n(name);
   if (n == "graph") C.opt.graph = value != 0;
+  else if (n == "dataflow") C.opt.dataflow = value != 0;
   else if (n == "streams") {
     if (value < 1 || value > 64) return fail(-105, "streams must be in [1, 64]");
     const int have = C.inited ? (int)C.slots[0].streams.size() - kCritStreams - kCopyStreams : 64;
@@ -652,6 +688,7 @@ int stf_get_option(const char* name, int64_t* value) {
   if (!name || !value) return fail(-105, "NULL argument");
   std::string n(name);
   if (n == "graph") *value = C.opt.graph;
+  else if (n == "dataflow") *value = C.opt.dataflow;
   else if (n == "streams") *value = C.opt.streams;
   else if (n == "serial") *value = C.opt.serial;
   else if (n == "priority") *value = C.opt.priority;
@@ -722,7 +759,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
         e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
         (e.opt.graph == C.opt.graph || A_desc->kind == STF_DESC_HOST_COLMAJOR) &&
-        e.opt.priority == C.opt.priority && e.key_ptrs == ptrs &&
+        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
       C.cache.splice(C.cache.begin(), C.cache, it);
@@ -901,6 +938,15 @@ int stf_kernel_trsm(int64_t M, int64_t n, const double* L, int64_t ldl, double* 
   cudaGetDevice(&dev);
   int r = ensure_kernel_attrs(dev);
   if (r) return r;
+  if (ctx().opt.dataflow) {
+    int* ws = nullptr;
+    CUDA_TRY(cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)M, (int)n)), "ws alloc");
+    cudaError_t e = stfk::trsm_tile(0, 0, (int)M, (int)n, L, ldl, B, ldb, ws);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(0);
+    cudaFree(ws);
+    CUDA_TRY(e, "trsm (dataflow)");
+    return 0;
+  }
   CUDA_TRY(stfk::trsm_rlt(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm");
   CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
   return 0;
@@ -914,11 +960,16 @@ int stf_kernel_potrf(int64_t n, double* A, int64_t lda, int64_t* info) {
   if (r) return r;
   unsigned long long* d_info = nullptr;
   CUDA_TRY(cudaMalloc(&d_info, sizeof *d_info), "info alloc");
-  cudaError_t e = stfk::info_reset(0, d_info);
-  if (e == cudaSuccess) e = stfk::potrf_lower(0, 0, (int)n, A, lda, 0, d_info);
+  int* ws = nullptr;
+  cudaError_t e = cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)n, (int)n));
+  if (e == cudaSuccess) e = stfk::info_reset(0, d_info);
+  if (e == cudaSuccess)
+    e = ctx().opt.dataflow ? stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws)
+                           : stfk::potrf_lower(0, 0, (int)n, A, lda, 0, d_info);
   unsigned long long v = ULLONG_MAX;
   if (e == cudaSuccess) e = cudaMemcpy(&v, d_info, sizeof v, cudaMemcpyDeviceToHost);
   cudaFree(d_info);
+  cudaFree(ws);
   if (e != cudaSuccess) return cuda_fail(e, "potrf");
   if (info) *info = (v == ULLONG_MAX) ? 0 : (int64_t)v;
   return 0;
@@ -951,6 +1002,8 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
   step(cudaMalloc(&Cm, (size_t)(ldm * N) * 8));
   step(cudaMalloc(&Src, (size_t)(ldm * N) * 8));
   step(cudaMalloc(&info, sizeof *info));
+  int* ws = nullptr;
+  step(cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)M, (int)N)));
   if (e == cudaSuccess) {
     // operands: SPD generator blocks (well scaled); L for TRSM = the lower part of an SPD block is fine
     step(stfk::fill_spd(s, A, ldm, M + K, 0, 0, (int)M, (int)K, 11));
@@ -964,8 +1017,14 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
       switch (kind) {
         case 0: step(stfk::gemm_nt(s, 0, (int)M, (int)N, (int)K, A, ldm, B, ldn, Cm, ldm, 0)); break;
         case 1: step(stfk::gemm_nt(s, 0, (int)M, (int)M, (int)K, A, ldm, A, ldm, Cm, ldm, 1)); break;
-        case 2: step(stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)); break;
-        case 3: step(stfk::potrf_lower(s, 0, (int)M, Cm, ldm, 0, info)); break;
+        case 2:
+          step(ctx().opt.dataflow ? stfk::trsm_tile(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm, ws)
+                                  : stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm));
+          break;
+        case 3:
+          step(ctx().opt.dataflow ? stfk::potrf_tile(s, 0, (int)M, Cm, ldm, 0, info, ws)
+                                  : stfk::potrf_lower(s, 0, (int)M, Cm, ldm, 0, info));
+          break;
       }
       step(cudaEventRecord(e1, s));
       step(cudaEventSynchronize(e1));
@@ -974,7 +1033,7 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
       if (it > 0) total += ms;
     }
   }
-  cudaFree(A); cudaFree(B); cudaFree(Cm); cudaFree(Src); cudaFree(info);
+  cudaFree(A); cudaFree(B); cudaFree(Cm); cudaFree(Src); cudaFree(info); cudaFree(ws);
   if (e0) cudaEventDestroy(e0);
   if (e1) cudaEventDestroy(e1);
   if (s) cudaStreamDestroy(s);

@@ -21,6 +21,15 @@ def abi():
     return _abi
 
 
+@pytest.fixture(params=[1, 0], ids=["dataflow", "recursive"])
+def variant(request, abi):
+    """TRSM/POTRF implementation: single-launch dataflow kernel (product
+    default) or the recursive GEMM-based driver."""
+    abi.stf_set_option(b"dataflow", request.param)
+    yield request.param
+    abi.stf_set_option(b"dataflow", 1)
+
+
 def _even(x):
     return x + (x & 1)
 
@@ -77,8 +86,9 @@ def test_syrk_lower(abi, N, K):
     _gemm_case(abi, N, N, K, True)
 
 
-@pytest.mark.parametrize("M,n", [(64, 64), (100, 70), (1024, 1024), (300, 200), (1, 1), (512, 129)])
-def test_trsm(abi, M, n):
+@pytest.mark.parametrize("M,n", [(64, 64), (100, 70), (1024, 1024), (300, 200), (1, 1), (512, 129), (2048, 2048),
+                                 (130, 1000)])
+def test_trsm(abi, variant, M, n):
     rng = np.random.default_rng(M + n)
     Lfull = np.tril(rng.standard_normal((n, n))) * 0.1 + np.diag(1.0 + rng.random(n))
     B = rng.standard_normal((M, n))
@@ -94,8 +104,8 @@ def test_trsm(abi, M, n):
     assert np.linalg.norm(X - ref) <= 1e-12 * np.linalg.norm(ref)
 
 
-@pytest.mark.parametrize("n", [1, 2, 17, 64, 65, 100, 256, 1024])
-def test_potrf_tile(abi, n):
+@pytest.mark.parametrize("n", [1, 2, 17, 64, 65, 100, 256, 1024, 2048])
+def test_potrf_tile(abi, variant, n):
     import synth
 
     A = synth.spd_matrix(20 + n, n)
@@ -113,7 +123,7 @@ def test_potrf_tile(abi, n):
 
 
 @pytest.mark.parametrize("n,j", [(64, 0), (64, 63), (200, 64), (200, 199), (1024, 511)])
-def test_potrf_tile_info(abi, n, j):
+def test_potrf_tile_info(abi, variant, n, j):
     import synth
 
     A = synth.spd_matrix(3, n)
