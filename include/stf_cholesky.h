@@ -95,6 +95,8 @@ const char *stf_last_error(void);
 
 /* ---------------------------------------------------------------- options
  * Execution options (defaults from the environment at init):
+ *   "dataflow" STF_DATAFLOW POTRF tile kernel: 1 single-launch dataflow (default), 0 recursive
+ *   "trsm"     STF_TRSM     TRSM tile kernel: 2 row-panel (default), 1 dataflow, 0 recursive
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA
  *                           graph, memoised per (n, nb, grid, tiles) (default);
  *                           0: eager lowering on streams + events

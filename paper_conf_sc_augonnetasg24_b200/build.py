@@ -26,6 +26,7 @@ SOURCES = [
     "kernels/gemm_dmma.cu",
     "kernels/panel.cu",
     "kernels/dataflow.cu",
+    "kernels/trsm_panel.cu",
     "plan.cpp",
     "runtime.cpp",
 ]

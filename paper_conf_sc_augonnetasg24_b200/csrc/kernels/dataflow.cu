@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <climits>
 #include <cstdint>
 #include <map>
@@ -155,54 +156,122 @@ __device__ void task_update(double* sm, double* C, int64_t ldc, const double* A,
       }
 }
 
-// S: X[rows x nc] <- X L^-T, L nc x nc lower (substitution, column by column)
-__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc) {
-  double* Bs = sm;                    // Bs[r][c]
-  double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
-  load_block_rm(Bs, df::LDB, X, ldx, rows, nc, false);
-  load_block_rm(Ls, df::LDB, L, ldl, nc, nc, true);
-  __syncthreads();
-  const int r = threadIdx.x & (df::W - 1), ty = threadIdx.x >> 6;
-  for (int c = 0; c < nc; ++c) {
-    if (threadIdx.x < rows) Bs[threadIdx.x * df::LDB + c] = Bs[threadIdx.x * df::LDB + c] / Ls[c * df::LDB + c];
-    __syncthreads();
-    if (r < rows) {
-      const double x = Bs[r * df::LDB + c];
-      for (int c2 = c + 1 + ty; c2 < nc; c2 += 4)
-        Bs[r * df::LDB + c2] = fma(-x, Ls[c2 * df::LDB + c], Bs[r * df::LDB + c2]);
-    }
-    __syncthreads();
-  }
-  store_block_rm(Bs, df::LDB, X, ldx, rows, nc, false);
+__device__ __forceinline__ void named_bar(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// P: in-place lower Cholesky of the nc x nc diagonal block (right-looking, in smem)
-__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
-  double* S = sm;  // S[r][c]
-  load_block_rm(S, df::LDB, X, ldx, nc, nc, true);
-  __syncthreads();
-  const int r = threadIdx.x & (df::W - 1), ty = threadIdx.x >> 6;
-  for (int j = 0; j < nc; ++j) {
-    if (threadIdx.x == 0) {
-      double s = S[j * df::LDB + j];
-      if (!(s > 0.0)) {
-        atomicMin(info, (unsigned long long)(col0 + j + 1));
-        s = __longlong_as_double(0x7ff8000000000000LL);
-      } else {
-        s = sqrt(s);
-      }
-      S[j * df::LDB + j] = s;
-    }
-    __syncthreads();
-    if (threadIdx.x > j && threadIdx.x < nc) S[threadIdx.x * df::LDB + j] = S[threadIdx.x * df::LDB + j] / S[j * df::LDB + j];
-    __syncthreads();
-    if (r > j && r < nc) {
-      const double l = S[r * df::LDB + j];
-      for (int c = j + 1 + ty; c <= r; c += 4) S[r * df::LDB + c] = fma(-l, S[c * df::LDB + j], S[r * df::LDB + c]);
-    }
-    __syncthreads();
+// S: X[rows x nc] <- X L^-T, L nc x nc lower.  Thread (r = tid & 63, q = tid >> 6)
+// holds X[r, 16q .. 16q+15] in registers.  Chunk q solves its 16 columns by
+// substitution (divisions by L_cc), publishes x to smem, later chunks subtract
+// x L^T; every element accumulates its terms in increasing column order.
+__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc) {
+  double* Xs = sm;                    // Xs[r][c]
+  double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
+  double b[16];
+#pragma unroll
+  for (int c = 0; c < 16; ++c) {
+    const int col = 16 * q + c;
+    b[c] = (r < rows && col < nc) ? __ldcg(X + (int64_t)col * ldx + r) : 0.0;
   }
-  store_block_rm(S, df::LDB, X, ldx, nc, nc, true);
+  load_block_rm(Ls, df::LDB, L, ldl, nc, nc, true);
+  __syncthreads();
+  for (int qq = 0; qq < 4 && 16 * qq < nc; ++qq) {
+    if (q == qq) {
+#pragma unroll
+      for (int c = 0; c < 16; ++c) {
+        const int col = 16 * qq + c;
+        if (col < nc) {
+          b[c] = b[c] / Ls[col * df::LDB + col];
+#pragma unroll
+          for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], Ls[(16 * qq + c2) * df::LDB + col], b[c2]);
+        }
+      }
+#pragma unroll
+      for (int c = 0; c < 16; ++c) Xs[r * df::LDB + 16 * qq + c] = b[c];
+    }
+    __syncthreads();
+    if (q > qq) {
+#pragma unroll
+      for (int cc = 0; cc < 16; ++cc)
+#pragma unroll
+        for (int c = 0; c < 16; ++c)
+          b[cc] = fma(-Xs[r * df::LDB + 16 * qq + c], Ls[(16 * q + cc) * df::LDB + 16 * qq + c], b[cc]);
+    }
+  }
+  if (r < rows) {
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      const int col = 16 * q + c;
+      if (col < nc) X[(int64_t)col * ldx + r] = b[c];
+    }
+  }
+}
+
+// P: in-place lower Cholesky of the nc x nc diagonal block.  Thread (r, q) holds
+// A[r, 16q .. 16q+15]; chunk q (two warps, named barrier 1+q) factors its 16
+// columns (pivot sqrt by the owner of row col, column scaled by division,
+// in-chunk rank-1 updates), publishes them, and later chunks apply the
+// chunk's update.  Element updates run in increasing column order (Crout order).
+__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
+  double* S = sm;  // S[r][c]: published L values
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
+  double a[16];
+#pragma unroll
+  for (int c = 0; c < 16; ++c) {
+    const int col = 16 * q + c;
+    a[c] = (r < nc && col < nc && r >= col) ? __ldcg(X + (int64_t)col * ldx + r) : 0.0;
+  }
+  for (int qq = 0; qq < 4 && 16 * qq < nc; ++qq) {
+    if (q == qq) {
+#pragma unroll
+      for (int c = 0; c < 16; ++c) {
+        const int col = 16 * qq + c;
+        if (col < nc) {
+          if (r == col) {
+            double s = a[c];
+            if (!(s > 0.0)) {
+              atomicMin(info, (unsigned long long)(col0 + col + 1));
+              s = __longlong_as_double(0x7ff8000000000000LL);
+            } else {
+              s = sqrt(s);
+            }
+            a[c] = s;
+            S[col * df::LDB + col] = s;
+          }
+          named_bar(1 + qq, 64);
+          if (r > col && r < nc) {
+            a[c] = a[c] / S[col * df::LDB + col];
+            S[r * df::LDB + col] = a[c];
+          }
+          named_bar(1 + qq, 64);
+          if (r > col && r < nc) {
+#pragma unroll
+            for (int c2 = c + 1; c2 < 16; ++c2)
+              if (16 * qq + c2 <= r) a[c2] = fma(-a[c], S[(16 * qq + c2) * df::LDB + col], a[c2]);
+          }
+        }
+      }
+    }
+    __syncthreads();
+    if (q > qq && r < nc) {
+#pragma unroll
+      for (int cc = 0; cc < 16; ++cc) {
+        if (16 * q + cc <= r) {
+#pragma unroll
+          for (int c = 0; c < 16; ++c)
+            a[cc] = fma(-S[r * df::LDB + 16 * qq + c], S[(16 * q + cc) * df::LDB + 16 * qq + c], a[cc]);
+        }
+      }
+    }
+  }
+  if (r < nc) {
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      const int col = 16 * q + c;
+      if (col < nc && r >= col) X[(int64_t)col * ldx + r] = a[c];
+    }
+  }
 }
 
 __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
@@ -337,6 +406,14 @@ cudaError_t get_table(bool potrf, int Mb, int Nb, const uint32_t** out, int* cou
   return cudaSuccess;
 }
 
+int df_max_ctas() {
+  static int v = [] {
+    const char* e = getenv("STF_DF_CTAS");
+    return e ? atoi(e) : 16;
+  }();
+  return v;
+}
+
 int num_sms() {
   int dev = 0;
   cudaGetDevice(&dev);
@@ -402,7 +479,7 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   p.potrf = 1;
   const int T = p.Nb;
   const int par = T * (T - 1) / 2 > 0 ? T * (T - 1) / 2 : 1;  // widest update wave
-  return launch_df(stream, prio, p, std::min(par, num_sms() / 2));
+  return launch_df(stream, prio, p, std::min(par, std::min(df_max_ctas(), num_sms())));
 }
 
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
@@ -424,7 +501,7 @@ cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double*
   p.info = nullptr;
   p.potrf = 0;
   const int par = p.Mb * (p.Nb > 1 ? p.Nb - 1 : 1);
-  return launch_df(stream, prio, p, std::min(par, num_sms() / 2));
+  return launch_df(stream, prio, p, std::min(par, std::min(4 * df_max_ctas(), num_sms())));
 }
 
 }  // namespace stfk

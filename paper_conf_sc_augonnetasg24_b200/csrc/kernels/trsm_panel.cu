@@ -1,0 +1,204 @@
+// K3 TRSM tile kernel, row-panel form (north_star "TRSM as
+// a blocked triangular solve that calls those same tensor-core tiles").
+//
+//   TRSM(i,k):  X <- B L^-T   (X L^T = B),  B: M x n,  L: n x n lower
+//
+// Rows of X are independent, so each CTA owns 32 rows and sweeps the 64-wide
+// column blocks left to right (left-looking):
+//   for jb:  acc = B[rows, jb] - sum_{pb<jb} X[rows, pb] L[jb, pb]^T   (DMMA, operands
+//            staged by cp.async into padded smem, two stages)
+//            X[rows, jb] = acc L[jb, jb]^-T                              (substitution)
+// No cross-CTA dependencies: no flags, no waiting, every SM-cycle is work.  The
+// k-order of every sum is fixed, so results are bit-identical run to run; the
+// diagonal solve divides by L_cc (no reciprocal), so unit-diagonal dyadic inputs
+// stay exact (pin P2).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "tile_ops.hpp"
+
+namespace stfk {
+
+namespace tp {
+constexpr int BM = 32, W = 64, NT = 256;
+constexpr int SA = 36;  // As[k][m] stride (36 = 4 mod 16 -> conflict-free fragment loads)
+constexpr int SB = 68;  // Bs[k][n] stride
+constexpr int SS = 65;  // solve scratch stride
+constexpr int STAGE = W * SA + W * SB;  // doubles
+constexpr int SMEM_BYTES = 2 * STAGE * 8;
+}  // namespace tp
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ double negd_tp(double x) {
+  return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
+}
+
+// dst[k * ld + r] = G(r, k) for r < rows (<= R), k < kc (<= W); zero-filled otherwise.
+// Fast path (full block, 16-byte aligned columns) uses cp.async; else scalar loads.
+template <int R>
+__device__ __forceinline__ void stage_block(double* dst, int ld, const double* G, int64_t ldg, int rows, int kc,
+                                            bool fast) {
+  if (fast) {
+    constexpr int CH = R / 2;  // 16-byte chunks per column
+    for (int idx = threadIdx.x; idx < CH * tp::W; idx += tp::NT) {
+      const int k = idx / CH, c = idx % CH;
+      cp_async16(dst + k * ld + 2 * c, G + (int64_t)k * ldg + 2 * c);
+    }
+  } else {
+    for (int idx = threadIdx.x; idx < R * tp::W; idx += tp::NT) {
+      const int k = idx / R, r = idx % R;
+      dst[k * ld + r] = (r < rows && k < kc) ? __ldcg(G + (int64_t)k * ldg + r) : 0.0;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __restrict__ L, int64_t ldl, int n,
+                                                                double* __restrict__ X, int64_t ldx, int M) {
+  extern __shared__ __align__(16) double smt[];
+  const int r0 = blockIdx.x * tp::BM;
+  const int rows = min(tp::BM, M - r0);
+  const int Nb = (n + tp::W - 1) / tp::W;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const int wm0 = (warp & 1) * 16, wn0 = (warp >> 1) * 16;
+  double* Xr = X + r0;  // this CTA's rows
+  const bool rows_fast = (rows == tp::BM) && ((ldx & 1) == 0) && ((reinterpret_cast<uintptr_t>(Xr) & 15) == 0);
+
+  for (int jb = 0; jb < Nb; ++jb) {
+    const int c0 = jb * tp::W;
+    const int nc = min(tp::W, n - c0);
+    const bool l_fast = (nc == tp::W) && ((ldl & 1) == 0) && ((reinterpret_cast<uintptr_t>(L) & 15) == 0);
+    // acc = B[rows, jb-block]
+    double acc[2][2][2];
+#pragma unroll
+    for (int i = 0; i < 2; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int r = wm0 + 8 * i + g, c = wn0 + 8 * j + 2 * t + h;
+          acc[i][j][h] = (r < rows && c < nc) ? __ldcg(Xr + (int64_t)(c0 + c) * ldx + r) : 0.0;
+        }
+    // left-looking update over pb < jb, two-stage cp.async pipeline
+    if (jb > 0) {
+      auto issue = [&](int pb, int st) {
+        double* As = smt + st * tp::STAGE;
+        double* Bs = As + tp::W * tp::SA;
+        stage_block<tp::BM>(As, tp::SA, Xr + (int64_t)pb * tp::W * ldx, ldx, rows, tp::W, rows_fast);
+        stage_block<tp::W>(Bs, tp::SB, L + (int64_t)pb * tp::W * ldl + c0, ldl, nc, tp::W, l_fast);
+        cp_async_commit();
+      };
+      issue(0, 0);
+      for (int pb = 0; pb < jb; ++pb) {
+        const int st = pb & 1;
+        if (pb + 1 < jb) {
+          issue(pb + 1, st ^ 1);
+          cp_async_wait<1>();
+        } else {
+          cp_async_wait<0>();
+        }
+        __syncthreads();
+        const double* As = smt + st * tp::STAGE;
+        const double* Bs = As + tp::W * tp::SA;
+#pragma unroll 4
+        for (int k0 = 0; k0 < tp::W; k0 += 4) {
+          double a[2], b[2];
+#pragma unroll
+          for (int i = 0; i < 2; ++i) a[i] = As[(k0 + t) * tp::SA + wm0 + 8 * i + g];
+#pragma unroll
+          for (int j = 0; j < 2; ++j) b[j] = negd_tp(Bs[(k0 + t) * tp::SB + wn0 + 8 * j + g]);
+#pragma unroll
+          for (int i = 0; i < 2; ++i)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i], b[j]);
+        }
+        __syncthreads();  // stage st may be refilled next iteration
+      }
+    }
+    // ---- diagonal solve: S[r][c] = acc, Ld[c][p] = L(c0 + c, c0 + p)
+    double* S = smt;
+    double* Ld = smt + tp::BM * tp::SS;
+#pragma unroll
+    for (int i = 0; i < 2; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) S[(wm0 + 8 * i + g) * tp::SS + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
+    for (int idx = threadIdx.x; idx < tp::W * tp::W; idx += tp::NT) {
+      const int c = idx % tp::W, p = idx / tp::W;
+      Ld[c * tp::SS + p] = (c < nc && p <= c) ? __ldg(L + (int64_t)(c0 + p) * ldl + c0 + c) : 0.0;
+    }
+    __syncthreads();
+    // warps 0..3 own 16-column chunks; lane = row.  Chunk q solves its columns in
+    // registers, publishes x to S, later chunks subtract its contribution.
+    const int q = warp, r = lane;
+    double b[16];
+    if (q < 4) {
+#pragma unroll
+      for (int c = 0; c < 16; ++c) b[c] = S[r * tp::SS + 16 * q + c];
+    }
+    for (int qq = 0; qq < 4; ++qq) {
+      if (q == qq) {
+#pragma unroll
+        for (int c = 0; c < 16; ++c) {
+          const int col = 16 * qq + c;
+          if (col < nc) {
+            b[c] = b[c] / Ld[col * tp::SS + col];
+#pragma unroll
+            for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], Ld[(16 * qq + c2) * tp::SS + col], b[c2]);
+          }
+        }
+#pragma unroll
+        for (int c = 0; c < 16; ++c) S[r * tp::SS + 16 * qq + c] = b[c];
+      }
+      __syncthreads();
+      if (q > qq && q < 4) {
+#pragma unroll
+        for (int cc = 0; cc < 16; ++cc)
+#pragma unroll
+          for (int c = 0; c < 16; ++c)
+            b[cc] = fma(-S[r * tp::SS + 16 * qq + c], Ld[(16 * q + cc) * tp::SS + 16 * qq + c], b[cc]);
+      }
+    }
+    if (q < 4 && r < rows) {
+#pragma unroll
+      for (int c = 0; c < 16; ++c) {
+        const int col = 16 * q + c;
+        if (col < nc) Xr[(int64_t)(c0 + col) * ldx + r] = b[c];
+      }
+    }
+    __threadfence();  // X[rows, jb] is re-read (cp.async.cg, L2) by later jb iterations
+    __syncthreads();
+  }
+}
+
+cudaError_t trsm_panel_init_attrs() {
+  return cudaFuncSetAttribute(trsm_panel_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, tp::SMEM_BYTES);
+}
+
+cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                       int64_t ldb) {
+  if (M <= 0 || n <= 0) return cudaSuccess;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((M + tp::BM - 1) / tp::BM);
+  cfg.blockDim = dim3(tp::NT);
+  cfg.dynamicSmemBytes = tp::SMEM_BYTES;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributePriority;
+  attr[0].val.priority = prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  ++launch_count();
+  return cudaLaunchKernelEx(&cfg, trsm_panel_kernel, L, ldl, n, B, ldb, M);
+}
+
+}  // namespace stfk

@@ -74,7 +74,8 @@ struct Slot {
 };
 
 struct Options {
-  int64_t dataflow = 1;  // 1: single-launch dataflow POTRF/TRSM tile kernels; 0: recursive (GEMM-based)
+  int64_t dataflow = 1;  // POTRF tile kernel: 1 single-launch dataflow, 0 recursive (GEMM-based)
+  int64_t trsm = 2;      // TRSM tile kernel: 2 row-panel, 1 dataflow, 0 recursive
   int64_t graph = 1;
   int64_t streams = 8;
   int64_t serial = 0;
@@ -198,7 +199,10 @@ struct Lowerer {
                    "POTRF launch");
         return 0;
       case stf::K_TRSM:
-        if (X.opt.dataflow)
+        if (X.opt.trsm == 2)
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb),
+                   "TRSM launch");
+        else if (X.opt.trsm == 1)
           CUDA_TRY(stfk::trsm_tile(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, ws),
                    "TRSM launch");
         else
@@ -382,7 +386,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   }
   // dataflow-kernel workspaces (one private block per POTRF/TRSM task) and task tables
   X.task_ws.assign(P.tasks.size(), nullptr);
-  if (X.opt.dataflow) {
+  if (X.opt.dataflow || X.opt.trsm == 1) {
     const size_t wsb = stfk::dataflow_ws_bytes((int)X.nb, (int)X.nb);
     for (int s = 0; s < X.ngpus; ++s) {
       size_t cnt = 0;
@@ -559,6 +563,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   if (ngpus < 1 || ngpus > 64) return fail(-5, "ngpus=%d out of range", ngpus);
   C.opt.graph = env_int("STF_GRAPH", 1);
   C.opt.dataflow = env_int("STF_DATAFLOW", 1);
+  C.opt.trsm = env_int("STF_TRSM", 2);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.priority = env_int("STF_PRIO", 1);
@@ -667,6 +672,10 @@ int stf_set_option(const char* name, int64_t value) {
   std::string n(name);
   if (n == "graph") C.opt.graph = value != 0;
   else if (n == "dataflow") C.opt.dataflow = value != 0;
+  else if (n == "trsm") {
+    if (value < 0 || value > 2) return fail(-105, "trsm must be 0 (recursive), 1 (dataflow) or 2 (row panel)");
+    C.opt.trsm = value;
+  }
   else if (n == "streams") {
     if (value < 1 || value > 64) return fail(-105, "streams must be in [1, 64]");
     const int have = C.inited ? (int)C.slots[0].streams.size() - kCritStreams - kCopyStreams : 64;
@@ -689,6 +698,7 @@ int stf_get_option(const char* name, int64_t* value) {
   std::string n(name);
   if (n == "graph") *value = C.opt.graph;
   else if (n == "dataflow") *value = C.opt.dataflow;
+  else if (n == "trsm") *value = C.opt.trsm;
   else if (n == "streams") *value = C.opt.streams;
   else if (n == "serial") *value = C.opt.serial;
   else if (n == "priority") *value = C.opt.priority;
@@ -759,7 +769,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
         e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
         (e.opt.graph == C.opt.graph || A_desc->kind == STF_DESC_HOST_COLMAJOR) &&
-        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.key_ptrs == ptrs &&
+        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
       C.cache.splice(C.cache.begin(), C.cache, it);
@@ -938,7 +948,12 @@ int stf_kernel_trsm(int64_t M, int64_t n, const double* L, int64_t ldl, double* 
   cudaGetDevice(&dev);
   int r = ensure_kernel_attrs(dev);
   if (r) return r;
-  if (ctx().opt.dataflow) {
+  if (ctx().opt.trsm == 2) {
+    CUDA_TRY(stfk::trsm_panel(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm (row panel)");
+    CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
+    return 0;
+  }
+  if (ctx().opt.trsm == 1) {
     int* ws = nullptr;
     CUDA_TRY(cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)M, (int)n)), "ws alloc");
     cudaError_t e = stfk::trsm_tile(0, 0, (int)M, (int)n, L, ldl, B, ldb, ws);
@@ -1018,8 +1033,9 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
         case 0: step(stfk::gemm_nt(s, 0, (int)M, (int)N, (int)K, A, ldm, B, ldn, Cm, ldm, 0)); break;
         case 1: step(stfk::gemm_nt(s, 0, (int)M, (int)M, (int)K, A, ldm, A, ldm, Cm, ldm, 1)); break;
         case 2:
-          step(ctx().opt.dataflow ? stfk::trsm_tile(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm, ws)
-                                  : stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm));
+          step(ctx().opt.trsm == 2   ? stfk::trsm_panel(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)
+               : ctx().opt.trsm == 1 ? stfk::trsm_tile(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm, ws)
+                                     : stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm));
           break;
         case 3:
           step(ctx().opt.dataflow ? stfk::potrf_tile(s, 0, (int)M, Cm, ldm, 0, info, ws)

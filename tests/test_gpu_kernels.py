@@ -21,13 +21,15 @@ def abi():
     return _abi
 
 
-@pytest.fixture(params=[1, 0], ids=["dataflow", "recursive"])
+@pytest.fixture(params=[(1, 2), (1, 1), (0, 0)], ids=["dataflow+rowpanel", "dataflow", "recursive"])
 def variant(request, abi):
-    """TRSM/POTRF implementation: single-launch dataflow kernel (product
-    default) or the recursive GEMM-based driver."""
-    abi.stf_set_option(b"dataflow", request.param)
+    """(POTRF, TRSM) implementations: POTRF dataflow (1) / recursive (0);
+    TRSM row panel (2, product default) / dataflow (1) / recursive (0)."""
+    abi.stf_set_option(b"dataflow", request.param[0])
+    abi.stf_set_option(b"trsm", request.param[1])
     yield request.param
     abi.stf_set_option(b"dataflow", 1)
+    abi.stf_set_option(b"trsm", 2)
 
 
 def _even(x):

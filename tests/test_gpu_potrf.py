@@ -24,11 +24,21 @@ def stf():
     s.finalize()
 
 
+@pytest.mark.parametrize("trsm", [1, 2])
+def test_parity_trsm_variants(stf, trsm):
+    _options(stf, trsm=trsm)
+    M, info = _factor_spd(stf, 1536, 512, seed=2)
+    _options(stf, trsm=2)
+    assert info == 0
+    Lo, _ = oracle.potrf(synth.spd_matrix(2, 1536))
+    assert relF(M.to_dense().numpy(), Lo) <= 1e-10
+
+
 def test_parity_recursive_panel_kernels(stf):
     """The recursive (GEMM-based) POTRF/TRSM variant through the whole path."""
-    _options(stf, dataflow=0)
+    _options(stf, dataflow=0, trsm=0)
     M, info = _factor_spd(stf, 2048, 512, seed=1)
-    _options(stf, dataflow=1)
+    _options(stf, dataflow=1, trsm=2)
     assert info == 0
     Lo, _ = oracle.potrf(synth.spd_matrix(1, 2048))
     assert relF(M.to_dense().numpy(), Lo) <= 1e-10
@@ -44,7 +54,7 @@ def _reset_options(request):
     yield
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
-        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1)
+        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):

@@ -11,6 +11,8 @@ kind, M, N, K, reps = (int(x) for x in sys.argv[1:6])
 import os
 if os.environ.get("STF_DATAFLOW") == "0":
     _abi.stf_set_option(b"dataflow", 0)
+if os.environ.get("STF_TRSM"):
+    _abi.stf_set_option(b"trsm", int(os.environ["STF_TRSM"]))
 ms = ctypes.c_double()
 rc = _abi.stf_bench_kernel(kind, M, N, K, reps, ctypes.byref(ms))
 print("rc", rc, "avg_ms", ms.value, _abi.stf_last_error())
