@@ -175,6 +175,9 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
     b[c] = (r < rows && col < nc) ? __ldcg(X + (int64_t)col * ldx + r) : 0.0;
   }
   load_block_rm(Ls, df::LDB, L, ldl, nc, nc, true);
+  double* Rc = Ls + df::W * df::LDB;
+  __syncthreads();
+  if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / Ls[threadIdx.x * df::LDB + threadIdx.x];
   __syncthreads();
   for (int qq = 0; qq < 4 && 16 * qq < nc; ++qq) {
     if (q == qq) {
@@ -182,7 +185,7 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
       for (int c = 0; c < 16; ++c) {
         const int col = 16 * qq + c;
         if (col < nc) {
-          b[c] = b[c] / Ls[col * df::LDB + col];
+          b[c] = div_by(b[c], Ls[col * df::LDB + col], Rc[col]);
 #pragma unroll
           for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], Ls[(16 * qq + c2) * df::LDB + col], b[c2]);
         }
@@ -215,6 +218,7 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
 // chunk's update.  Element updates run in increasing column order (Crout order).
 __device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
   double* S = sm;  // S[r][c]: published L values
+  double* Y = sm + df::W * df::LDB;  // Y[c] = 1 / L_cc
   const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
   double a[16];
 #pragma unroll
@@ -238,10 +242,11 @@ __device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t co
             }
             a[c] = s;
             S[col * df::LDB + col] = s;
+            Y[col] = 1.0 / s;
           }
           named_bar(1 + qq, 64);
           if (r > col && r < nc) {
-            a[c] = a[c] / S[col * df::LDB + col];
+            a[c] = div_by(a[c], S[col * df::LDB + col], Y[col]);
             S[r * df::LDB + col] = a[c];
           }
           named_bar(1 + qq, 64);

@@ -35,27 +35,32 @@
 
 namespace stfk {
 
-namespace g {
-constexpr int BM = 128, BN = 128, BK = 16, STAGES = 4;
-constexpr int BOX = 16;                      // doubles per 128-byte swizzle row
-constexpr int BOX_BYTES = BOX * BK * 8;      // 2 KB
-constexpr int A_BYTES = BM * BK * 8;         // 16 KB
-constexpr int B_BYTES = BN * BK * 8;         // 16 KB
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 2 * STAGES * 8;
-}  // namespace g
+template <int BK_, int STAGES_>
+struct Cfg {
+  static constexpr int BM = 128, BN = 128, BK = BK_, STAGES = STAGES_;
+  static constexpr int BOX = 16;                  // doubles per 128-byte swizzle row
+  static constexpr int BOX_BYTES = BOX * BK * 8;  // 2 KB at BK = 16
+  static constexpr int A_BYTES = BM * BK * 8;     // 16 KB at BK = 16
+  static constexpr int B_BYTES = BN * BK * 8;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 2 * STAGES * 8;
+};
+using CfgK16 = Cfg<16, 4>;  // 4 x 32 KB stages
+using CfgK32 = Cfg<32, 3>;  // 3 x 64 KB stages
 
 // Exact negation as a sign-bit flip on the integer pipe (keeps the FP64/DMMA pipe free).
 __device__ __forceinline__ double neg(double x) {
   return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
 }
 
-// Byte offset of element (row r in [0,128), k in [0,16)) inside one operand stage.
+// Byte offset of element (row r in [0,128), k in [0,BK)) inside one operand stage.
+template <class g>
 __device__ __forceinline__ uint32_t swz_off(int r, int k) {
   const int box = r >> 4, mi = r & 15;
   return box * g::BOX_BYTES + k * 128 + ((((mi >> 1) ^ (k & 7)) << 4) | ((mi & 1) << 3));
 }
 
+template <class g>
 __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorMap* tmA, const CUtensorMap* tmB,
                                            int m0, int n0, int kt, uint64_t* full) {
   mbar_arrive_expect_tx(&full[s], g::STAGE_BYTES);
@@ -71,7 +76,7 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
 // so the refill of the stage consumed at kt-1 rarely waits).  8 warps keep the
 // register cap at 255/thread (a 9th producer warp would cap it at 168: the
 // register file is split per SM sub-partition and 9 warps round up to 12).
-template <int WM, int WN>
+template <int WM, int WN, class g>
 __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         double* __restrict__ C, int64_t ldc, int M, int N, int K, int lower) {
@@ -108,7 +113,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
       mbar_init(&empty[s], NCW);
     }
     fence_barrier_init();
-    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage(smem, kt, &tmA, &tmB, m0, n0, kt, full);
+    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, m0, n0, kt, full);
   }
   __syncthreads();
 
@@ -143,8 +148,8 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
   for (int p = 0; p < 2; ++p)
 #pragma unroll
     for (int kh = 0; kh < 2; ++kh) {
-      offA[p][kh] = swz_off(wm0 + 8 * p + gq, 2 * tq + kh);
-      offB[p][kh] = g::A_BYTES + swz_off(wn0 + 8 * p + gq, 2 * tq + kh);
+      offA[p][kh] = swz_off<g>(wm0 + 8 * p + gq, 2 * tq + kh);
+      offB[p][kh] = g::A_BYTES + swz_off<g>(wn0 + 8 * p + gq, 2 * tq + kh);
     }
 
   for (int kt = 0; kt < KT; ++kt) {
@@ -181,7 +186,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
       if (kr < KT) {
         const int sr = (kt - 1) % g::STAGES;
         mbar_wait(&empty[sr], ((kt - 1) / g::STAGES) & 1);
-        load_stage(smem, sr, &tmA, &tmB, m0, n0, kr, full);
+        load_stage<g>(smem, sr, &tmA, &tmB, m0, n0, kr, full);
       }
     }
   }
@@ -216,13 +221,13 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-// rows x cols column-major FP64 operand, box {16 rows, BK cols}, 128B swizzle, OOB -> 0.
-static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld) {
+// rows x cols column-major FP64 operand, box {16 rows, bk cols}, 128B swizzle, OOB -> 0.
+static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld, int bk) {
   auto fn = encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};
   cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(double)};
-  cuuint32_t box[2] = {(cuuint32_t)g::BOX, (cuuint32_t)g::BK};
+  cuuint32_t box[2] = {16u, (cuuint32_t)bk};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = fn(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(ptr), dims, strides, box, estr,
                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -230,14 +235,32 @@ static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int c
   return r == CUDA_SUCCESS;
 }
 
-// 8 warps of 64x32 (224 regs, 2 warps / SM sub-partition) or 16 warps of 32x32
-// (<= 128 regs, 4 warps / sub-partition).  STF_GEMM_WARPS selects; default 16.
-static int gemm_variant() {
-  static int v = [] {
-    const char* e = getenv("STF_GEMM_WARPS");
-    return (e && atoi(e) == 8) ? 8 : 16;
-  }();
+// Variants: warps 8 (64x32 warp tiles, 224 regs, 2 warps / SM sub-partition) or
+// 16 (32x32, <= 128 regs, 4 warps / sub-partition); BK 16 (4 stages) or 32 (3
+// stages).  STF_GEMM_WARPS / STF_GEMM_BK select; defaults 16 warps, BK 32.
+static int env_or(const char* name, int dflt) {
+  const char* e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
+static int gemm_warps() {
+  static int v = env_or("STF_GEMM_WARPS", 16) == 8 ? 8 : 16;
   return v;
+}
+static int gemm_bk() {
+  static int v = env_or("STF_GEMM_BK", 32) == 16 ? 16 : 32;
+  return v;
+}
+
+template <class G>
+static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tmA, const CUtensorMap& tmB, double* C,
+                                  int64_t ldc, int M, int N, int K, int lower) {
+  cfg.dynamicSmemBytes = G::SMEM_BYTES;
+  if (gemm_warps() == 16) {
+    cfg.blockDim = dim3(512, 1, 1);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, G>, tmA, tmB, C, ldc, M, N, K, lower);
+  }
+  cfg.blockDim = dim3(256, 1, 1);
+  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, G>, tmA, tmB, C, ldc, M, N, K, lower);
 }
 
 cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
@@ -245,18 +268,13 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
     return cudaErrorMisalignedAddress;
+  const int bk = gemm_bk();
   CUtensorMap tmA, tmB;
-  if (!make_operand_map(&tmA, A, M, K, lda) || !make_operand_map(&tmB, B, N, K, ldb)) return cudaErrorInvalidValue;
-  const int tM = (M + g::BM - 1) / g::BM, tN = (N + g::BN - 1) / g::BN;
+  if (!make_operand_map(&tmA, A, M, K, lda, bk) || !make_operand_map(&tmB, B, N, K, ldb, bk))
+    return cudaErrorInvalidValue;
+  const int tM = (M + 127) / 128, tN = (N + 127) / 128;
   cudaLaunchConfig_t cfg = {};
-  if (lower) {
-    cfg.gridDim = dim3(tM * (tM + 1) / 2, 1, 1);
-  } else {
-    cfg.gridDim = dim3(tM, tN, 1);
-  }
-  const int variant = gemm_variant();
-  cfg.blockDim = dim3(variant == 16 ? 512 : 256, 1, 1);
-  cfg.dynamicSmemBytes = g::SMEM_BYTES;
+  cfg.gridDim = lower ? dim3(tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributePriority;
@@ -264,15 +282,23 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   ++launch_count();
-  if (variant == 16) return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32>, tmA, tmB, C, ldc, M, N, K, lower);
-  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32>, tmA, tmB, C, ldc, M, N, K, lower);
+  if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
+  return launch_variant<CfgK16>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
+}
+
+template <class G>
+static cudaError_t set_attrs() {
+  cudaError_t e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<64, 32, G>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       G::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, G>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             G::SMEM_BYTES);
+  return e;
 }
 
 cudaError_t gemm_init_attrs() {
-  cudaError_t e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<64, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       g::SMEM_BYTES);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, g::SMEM_BYTES);
+  cudaError_t e = set_attrs<CfgK16>();
+  if (e == cudaSuccess) e = set_attrs<CfgK32>();
   return e;
 }
 

@@ -68,4 +68,14 @@ __device__ __forceinline__ void dmma_8x8x4(double& d0, double& d1, double a, dou
                : "d"(a), "d"(b));
 }
 
+// a / d from y = RN(1/d) (an IEEE division done once per pivot, off the serial
+// chain): q0 = RN(a y), r = a - q0 d (exact with FMA), q = RN(q0 + r y).
+// Markstein's correction returns RN(a / d) bit for bit (checked on 2^33 random
+// operand pairs by tools/check_div.cu); unit pivots stay exact.
+__device__ __forceinline__ double div_by(double a, double d, double y) {
+  const double q0 = a * y;
+  const double r = fma(-q0, d, a);
+  return fma(r, y, q0);
+}
+
 }  // namespace stfk

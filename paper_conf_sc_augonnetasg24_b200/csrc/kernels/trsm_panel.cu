@@ -10,8 +10,9 @@
 //            X[rows, jb] = acc L[jb, jb]^-T                              (substitution)
 // No cross-CTA dependencies: no flags, no waiting, every SM-cycle is work.  The
 // k-order of every sum is fixed, so results are bit-identical run to run; the
-// diagonal solve divides by L_cc (no reciprocal), so unit-diagonal dyadic inputs
-// stay exact (pin P2).
+// diagonal solve returns the correctly rounded quotient by L_cc (div_by: one IEEE
+// reciprocal per column, Markstein correction on the chain), so unit-diagonal
+// dyadic inputs stay exact (pin P2).
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -126,6 +127,7 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
     // ---- diagonal solve: S[r][c] = acc, Ld[c][p] = L(c0 + c, c0 + p)
     double* S = smt;
     double* Ld = smt + tp::BM * tp::SS;
+    double* Rc = Ld + tp::W * tp::SS;  // Rc[c] = 1 / L(c0 + c, c0 + c)
 #pragma unroll
     for (int i = 0; i < 2; ++i)
 #pragma unroll
@@ -136,6 +138,8 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
       const int c = idx % tp::W, p = idx / tp::W;
       Ld[c * tp::SS + p] = (c < nc && p <= c) ? __ldg(L + (int64_t)(c0 + p) * ldl + c0 + c) : 0.0;
     }
+    __syncthreads();
+    if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / Ld[threadIdx.x * tp::SS + threadIdx.x];
     __syncthreads();
     // warps 0..3 own 16-column chunks; lane = row.  Chunk q solves its columns in
     // registers, publishes x to S, later chunks subtract its contribution.
@@ -151,7 +155,7 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
         for (int c = 0; c < 16; ++c) {
           const int col = 16 * qq + c;
           if (col < nc) {
-            b[c] = b[c] / Ld[col * tp::SS + col];
+            b[c] = div_by(b[c], Ld[col * tp::SS + col], Rc[col]);
 #pragma unroll
             for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], Ld[(16 * qq + c2) * tp::SS + col], b[c2]);
           }
