@@ -23,12 +23,14 @@
 namespace stfk {
 
 namespace tp {
-constexpr int BM = 32, W = 64, NT = 256;
+constexpr int BM = 32, W = 64, NT = 256, STAGES = 3;
 constexpr int SA = 36;  // As[k][m] stride (36 = 4 mod 16 -> conflict-free fragment loads)
 constexpr int SB = 68;  // Bs[k][n] stride
 constexpr int SS = 65;  // solve scratch stride
-constexpr int STAGE = W * SA + W * SB;  // doubles
-constexpr int SMEM_BYTES = 2 * STAGE * 8;
+constexpr int SL = 66;  // LdT stride (16-byte aligned columns for cp.async; accesses are warp broadcasts)
+constexpr int STAGE = W * SA + W * SB;            // doubles per pipeline stage
+constexpr int SOLVE = BM * SS + W * SL + W;       // S, LdT, Rc
+constexpr int SMEM_BYTES = (STAGES * STAGE + SOLVE) * 8;  // ~210 KB
 }  // namespace tp
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
@@ -72,11 +74,62 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
   const int wm0 = (warp & 1) * 16, wn0 = (warp >> 1) * 16;
   double* Xr = X + r0;  // this CTA's rows
   const bool rows_fast = (rows == tp::BM) && ((ldx & 1) == 0) && ((reinterpret_cast<uintptr_t>(Xr) & 15) == 0);
+  const bool lal = ((ldl & 1) == 0) && ((reinterpret_cast<uintptr_t>(L) & 15) == 0);
+  double* S = smt + tp::STAGES * tp::STAGE;  // solve scratch (never aliases the pipeline)
+  double* LdT = S + tp::BM * tp::SS;         // LdT[p * SL + c] = L(c0 + c, c0 + p); upper part unused
+  double* Rc = LdT + tp::W * tp::SL;
 
+  // Stage (jb, pb) = operands of the update of column block jb by block pb; it
+  // lives in ring slot pb % STAGES and is one cp.async group.  X block pb may be
+  // staged only after it has been solved, so the first STAGES-1 stages of jb+1
+  // are issued in two halves: those with pb < jb before the solve of jb (overlapping
+  // their latency with it), the one with pb == jb after it.  Every prologue commits
+  // exactly STAGES-1 groups and every update iteration one group.
+  auto issue = [&](int jb, int pb) {
+    const int c0 = jb * tp::W, nc = min(tp::W, n - c0);
+    double* As = smt + (pb % tp::STAGES) * tp::STAGE;
+    double* Bs = As + tp::W * tp::SA;
+    stage_block<tp::BM>(As, tp::SA, Xr + (int64_t)pb * tp::W * ldx, ldx, rows, tp::W, rows_fast);
+    stage_block<tp::W>(Bs, tp::SB, L + (int64_t)pb * tp::W * ldl + c0, ldl, nc, tp::W, lal && nc == tp::W);
+  };
+  // diagonal block L(jb, jb) -> LdT (cp.async when full and aligned)
+  auto issue_diag = [&](int jb) {
+    const int c0 = jb * tp::W, nc = min(tp::W, n - c0);
+    const double* G = L + (int64_t)c0 * ldl + c0;
+    if (lal && nc == tp::W) {
+      for (int idx = threadIdx.x; idx < 32 * tp::W; idx += tp::NT) {
+        const int p = idx / 32, ch = idx % 32;
+        cp_async16(LdT + p * tp::SL + 2 * ch, G + (int64_t)p * ldl + 2 * ch);
+      }
+    } else {
+      for (int idx = threadIdx.x; idx < tp::W * tp::W; idx += tp::NT) {
+        const int p = idx / tp::W, c = idx % tp::W;
+        LdT[p * tp::SL + c] = (c < nc && p < nc) ? __ldg(G + (int64_t)p * ldl + c) : 0.0;
+      }
+    }
+  };
+  auto prologue_pre = [&](int jn) {
+    for (int p = 0; p < tp::STAGES - 1; ++p)
+      if (p < jn - 1) {
+        issue(jn, p);
+        cp_async_commit();
+      }
+  };
+  auto prologue_post = [&](int jn) {
+    issue_diag(jn);
+    cp_async_commit();
+    for (int p = 0; p < tp::STAGES - 1; ++p)
+      if (p >= jn - 1) {
+        if (p < jn) issue(jn, p);
+        cp_async_commit();
+      }
+  };
+
+  issue_diag(0);
+  cp_async_commit();
   for (int jb = 0; jb < Nb; ++jb) {
     const int c0 = jb * tp::W;
     const int nc = min(tp::W, n - c0);
-    const bool l_fast = (nc == tp::W) && ((ldl & 1) == 0) && ((reinterpret_cast<uintptr_t>(L) & 15) == 0);
     // acc = B[rows, jb-block]
     double acc[2][2][2];
 #pragma unroll
@@ -88,58 +141,39 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
           const int r = wm0 + 8 * i + g, c = wn0 + 8 * j + 2 * t + h;
           acc[i][j][h] = (r < rows && c < nc) ? __ldcg(Xr + (int64_t)(c0 + c) * ldx + r) : 0.0;
         }
-    // left-looking update over pb < jb, two-stage cp.async pipeline
-    if (jb > 0) {
-      auto issue = [&](int pb, int st) {
-        double* As = smt + st * tp::STAGE;
-        double* Bs = As + tp::W * tp::SA;
-        stage_block<tp::BM>(As, tp::SA, Xr + (int64_t)pb * tp::W * ldx, ldx, rows, tp::W, rows_fast);
-        stage_block<tp::W>(Bs, tp::SB, L + (int64_t)pb * tp::W * ldl + c0, ldl, nc, tp::W, l_fast);
-        cp_async_commit();
-      };
-      issue(0, 0);
-      for (int pb = 0; pb < jb; ++pb) {
-        const int st = pb & 1;
-        if (pb + 1 < jb) {
-          issue(pb + 1, st ^ 1);
-          cp_async_wait<1>();
-        } else {
-          cp_async_wait<0>();
-        }
-        __syncthreads();
-        const double* As = smt + st * tp::STAGE;
-        const double* Bs = As + tp::W * tp::SA;
+    // left-looking update over pb < jb, one barrier per stage
+    for (int pb = 0; pb < jb; ++pb) {
+      cp_async_wait<tp::STAGES - 2>();
+      __syncthreads();
+      const int pf = pb + tp::STAGES - 1;  // refill the slot consumed at pb - 1
+      if (pf < jb) issue(jb, pf);
+      cp_async_commit();
+      const double* As = smt + (pb % tp::STAGES) * tp::STAGE;
+      const double* Bs = As + tp::W * tp::SA;
 #pragma unroll 4
-        for (int k0 = 0; k0 < tp::W; k0 += 4) {
-          double a[2], b[2];
+      for (int k0 = 0; k0 < tp::W; k0 += 4) {
+        double a[2], b[2];
 #pragma unroll
-          for (int i = 0; i < 2; ++i) a[i] = As[(k0 + t) * tp::SA + wm0 + 8 * i + g];
+        for (int i = 0; i < 2; ++i) a[i] = As[(k0 + t) * tp::SA + wm0 + 8 * i + g];
 #pragma unroll
-          for (int j = 0; j < 2; ++j) b[j] = negd_tp(Bs[(k0 + t) * tp::SB + wn0 + 8 * j + g]);
+        for (int j = 0; j < 2; ++j) b[j] = negd_tp(Bs[(k0 + t) * tp::SB + wn0 + 8 * j + g]);
 #pragma unroll
-          for (int i = 0; i < 2; ++i)
+        for (int i = 0; i < 2; ++i)
 #pragma unroll
-            for (int j = 0; j < 2; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i], b[j]);
-        }
-        __syncthreads();  // stage st may be refilled next iteration
+          for (int j = 0; j < 2; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i], b[j]);
       }
     }
-    // ---- diagonal solve: S[r][c] = acc, Ld[c][p] = L(c0 + c, c0 + p)
-    double* S = smt;
-    double* Ld = smt + tp::BM * tp::SS;
-    double* Rc = Ld + tp::W * tp::SS;  // Rc[c] = 1 / L(c0 + c, c0 + c)
+    cp_async_wait<0>();
+    __syncthreads();  // ring free
+    if (jb + 1 < Nb) prologue_pre(jb + 1);
+    // ---- diagonal solve: S[r][c] = acc, LdT = L(jb,jb) (landed: waited above), Rc[c] = 1 / L_cc
 #pragma unroll
     for (int i = 0; i < 2; ++i)
 #pragma unroll
       for (int j = 0; j < 2; ++j)
 #pragma unroll
         for (int h = 0; h < 2; ++h) S[(wm0 + 8 * i + g) * tp::SS + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
-    for (int idx = threadIdx.x; idx < tp::W * tp::W; idx += tp::NT) {
-      const int c = idx % tp::W, p = idx / tp::W;
-      Ld[c * tp::SS + p] = (c < nc && p <= c) ? __ldg(L + (int64_t)(c0 + p) * ldl + c0 + c) : 0.0;
-    }
-    __syncthreads();
-    if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / Ld[threadIdx.x * tp::SS + threadIdx.x];
+    if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / LdT[threadIdx.x * tp::SL + threadIdx.x];
     __syncthreads();
     // warps 0..3 own 16-column chunks; lane = row.  Chunk q solves its columns in
     // registers, publishes x to S, later chunks subtract its contribution.
@@ -155,9 +189,9 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
         for (int c = 0; c < 16; ++c) {
           const int col = 16 * qq + c;
           if (col < nc) {
-            b[c] = div_by(b[c], Ld[col * tp::SS + col], Rc[col]);
+            b[c] = div_by(b[c], LdT[col * tp::SL + col], Rc[col]);
 #pragma unroll
-            for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], Ld[(16 * qq + c2) * tp::SS + col], b[c2]);
+            for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], LdT[col * tp::SL + 16 * qq + c2], b[c2]);
           }
         }
 #pragma unroll
@@ -169,7 +203,7 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
         for (int cc = 0; cc < 16; ++cc)
 #pragma unroll
           for (int c = 0; c < 16; ++c)
-            b[cc] = fma(-S[r * tp::SS + 16 * qq + c], Ld[(16 * q + cc) * tp::SS + 16 * qq + c], b[cc]);
+            b[cc] = fma(-S[r * tp::SS + 16 * qq + c], LdT[(16 * qq + c) * tp::SL + 16 * q + cc], b[cc]);
       }
     }
     if (q < 4 && r < rows) {
@@ -179,8 +213,9 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
         if (col < nc) Xr[(int64_t)(c0 + col) * ldx + r] = b[c];
       }
     }
-    __threadfence();  // X[rows, jb] is re-read (cp.async.cg, L2) by later jb iterations
+    __threadfence();  // X[rows, jb] is re-read (cp.async.cg, L2) by the next jb iterations
     __syncthreads();
+    if (jb + 1 < Nb) prologue_post(jb + 1);
   }
 }
 
