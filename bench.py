@@ -109,7 +109,7 @@ def oracle_sample(n, seed, target_s, cap_n=None):
     oracle.potrf(A)
     tc = time.perf_counter() - t0
     m = int(cal * (target_s / max(tc, 1e-3)) ** (1.0 / 3.0))
-    m = max(cal, min(m, cap_n or n, 16384))
+    m = min(max(cal, m), cap_n or n, 16384)
     m -= m % 64
     A = synth.spd_block(seed, n, 0, 0, m, m)
     t0 = time.perf_counter()
@@ -119,12 +119,25 @@ def oracle_sample(n, seed, target_s, cap_n=None):
     return m, dt, oracle.max_threads()
 
 
+def max_over_ranks(x: float, dist_on: bool) -> float:
+    """Max of a per-rank float over all ranks (NCCL on GPU boxes, gloo on CPU)."""
+    if not dist_on:
+        return x
+    import torch
+    import torch.distributed as dist
+
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def reference_arm(args, rank, world):
     if rank != 0:
         return 0
     n, nb = args.n, args.nb
-    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
-    m, _, cores = oracle_sample(n, 1, per_step)
+    per_step = args.ref_seconds or max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    m, _, cores = oracle_sample(n, 1, per_step, cap_n=args.ref_cap)
     import oracle
     import synth
 
@@ -203,9 +216,7 @@ def run_ours(args, rank, world):
         clk = clocks.stop()
         total_ms = sum(steps_ms)
     if dist_on:
-        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
+        total_ms = max_over_ranks(total_ms, True)
         dist.barrier()
     if rank != 0:
         if dist_on:
@@ -339,6 +350,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--ref-cap", type=int, default=0, help="cap on the reference sample order (0 = none)")
+    ap.add_argument("--ref-seconds", type=float, default=0.0, help="oracle seconds per reference step (0 = auto)")
     args = ap.parse_args()
     assert args.warmup >= 1
     rank = int(os.environ.get("RANK", "0"))

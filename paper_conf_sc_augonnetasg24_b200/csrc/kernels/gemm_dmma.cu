@@ -43,7 +43,7 @@ struct Cfg {
   static constexpr int A_BYTES = BM * BK * 8;     // 16 KB at BK = 16
   static constexpr int B_BYTES = BN * BK * 8;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 2 * STAGES * 8;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + STAGES * 8 + STAGES * 4;
 };
 using CfgK16 = Cfg<16, 4>;  // 4 x 32 KB stages
 using CfgK32 = Cfg<32, 3>;  // 3 x 64 KB stages
@@ -72,10 +72,11 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
   for (int b = 0; b < g::BN / g::BOX; ++b) tma_load_2d(sb + b * g::BOX_BYTES, tmB, n0 + b * g::BOX, kt * g::BK, &full[s]);
 }
 
-// 8 warps, all consumers; thread 0 also issues the TMA loads (one stage behind,
-// so the refill of the stage consumed at kt-1 rarely waits).  8 warps keep the
-// register cap at 255/thread (a 9th producer warp would cap it at 168: the
-// register file is split per SM sub-partition and 9 warps round up to 12).
+// All warps are consumers (a dedicated producer warp would lower the register cap:
+// the register file is split per SM sub-partition, 9 warps round up to 12).  The
+// refill of a stage is issued by the LAST warp to finish reading it (shared-memory
+// arrival counter), i.e. at the earliest possible moment, with the next k-tile
+// STAGES ahead; consumers wait only on the TMA "full" mbarriers.
 template <int WM, int WN, class g>
 __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
@@ -86,7 +87,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
   // the compiler emits LDS, not generic LD, for the fragment loads
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + g::STAGES * g::STAGE_BYTES);
-  uint64_t* empty = full + g::STAGES;
+  int* released = reinterpret_cast<int*>(full + g::STAGES);  // per-stage arrival counters
 
   int tm, tn;
   if (lower) {
@@ -110,7 +111,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
     tma_prefetch_desc(&tmB);
     for (int s = 0; s < g::STAGES; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NCW);
+      released[s] = 0;
     }
     fence_barrier_init();
     for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, m0, n0, kt, full);
@@ -178,15 +179,14 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
             for (int j = 0; j < WN / 8; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i][kh], b[j][kh]);
       }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[s]);
-    // refill the stage consumed in the previous iteration (all 8 warps must have released it)
-    if (threadIdx.x == 0 && kt >= 1) {
-      const int kr = kt - 1 + g::STAGES;
-      if (kr < KT) {
-        const int sr = (kt - 1) % g::STAGES;
-        mbar_wait(&empty[sr], ((kt - 1) / g::STAGES) & 1);
-        load_stage<g>(smem, sr, &tmA, &tmB, m0, n0, kr, full);
+    __syncwarp();  // this warp's reads of stage s are complete (their values fed its DMMAs)
+    if (lane == 0 && kt + g::STAGES < KT) {
+      __threadfence_block();
+      if (atomicAdd(&released[s], 1) == NCW - 1) {  // last reader of stage s refills it
+        released[s] = 0;
+        __threadfence_block();
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        load_stage<g>(smem, s, &tmA, &tmB, m0, n0, kt + g::STAGES, full);
       }
     }
   }

@@ -16,22 +16,26 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 #include "ptx.cuh"
 #include "tile_ops.hpp"
 
 namespace stfk {
 
-namespace tp {
-constexpr int BM = 32, W = 64, NT = 256, STAGES = 3;
-constexpr int SA = 36;  // As[k][m] stride (36 = 4 mod 16 -> conflict-free fragment loads)
-constexpr int SB = 68;  // Bs[k][n] stride
-constexpr int SS = 65;  // solve scratch stride
-constexpr int SL = 66;  // LdT stride (16-byte aligned columns for cp.async; accesses are warp broadcasts)
-constexpr int STAGE = W * SA + W * SB;            // doubles per pipeline stage
-constexpr int SOLVE = BM * SS + W * SL + W;       // S, LdT, Rc
-constexpr int SMEM_BYTES = (STAGES * STAGE + SOLVE) * 8;  // ~210 KB
-}  // namespace tp
+// Rows per CTA: 32 (3 stages, latency) or 64 (2 stages, higher DMMA efficiency).
+template <int BM_>
+struct TP {
+  static constexpr int BM = BM_, W = 64, NT = 256, STAGES = (BM_ == 32) ? 3 : 2;
+  static constexpr int SA = BM + 4;  // As[k][m] stride (= 4 mod 16 -> conflict-free fragment loads)
+  static constexpr int SB = 68;      // Bs[k][n] stride
+  static constexpr int SS = 65;      // solve scratch stride
+  static constexpr int SL = 66;      // LdT stride (16-byte aligned columns for cp.async; warp-broadcast reads)
+  static constexpr int FM = BM / 16; // m-fragments per warp (2 x 4 warp grid, warp tile BM/2 x 16)
+  static constexpr int STAGE = W * SA + W * SB;                     // doubles per pipeline stage
+  static constexpr int SOLVE = BM * SS + W * SL + W;                // S, LdT, Rc
+  static constexpr int SMEM_BYTES = (STAGES * STAGE + SOLVE) * 8;  // ~210 KB / ~207 KB
+};
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
@@ -50,6 +54,7 @@ __device__ __forceinline__ double negd_tp(double x) {
 template <int R>
 __device__ __forceinline__ void stage_block(double* dst, int ld, const double* G, int64_t ldg, int rows, int kc,
                                             bool fast) {
+  using tp = TP<32>;
   if (fast) {
     constexpr int CH = R / 2;  // 16-byte chunks per column
     for (int idx = threadIdx.x; idx < CH * tp::W; idx += tp::NT) {
@@ -64,14 +69,16 @@ __device__ __forceinline__ void stage_block(double* dst, int ld, const double* G
   }
 }
 
-__global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __restrict__ L, int64_t ldl, int n,
-                                                                double* __restrict__ X, int64_t ldx, int M) {
+template <int BMT>
+__global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __restrict__ L, int64_t ldl, int n,
+                                                             double* __restrict__ X, int64_t ldx, int M) {
+  using tp = TP<BMT>;
   extern __shared__ __align__(16) double smt[];
   const int r0 = blockIdx.x * tp::BM;
   const int rows = min(tp::BM, M - r0);
   const int Nb = (n + tp::W - 1) / tp::W;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
-  const int wm0 = (warp & 1) * 16, wn0 = (warp >> 1) * 16;
+  const int wm0 = (warp & 1) * (tp::BM / 2), wn0 = (warp >> 1) * 16;
   double* Xr = X + r0;  // this CTA's rows
   const bool rows_fast = (rows == tp::BM) && ((ldx & 1) == 0) && ((reinterpret_cast<uintptr_t>(Xr) & 15) == 0);
   const bool lal = ((ldl & 1) == 0) && ((reinterpret_cast<uintptr_t>(L) & 15) == 0);
@@ -131,9 +138,9 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
     const int c0 = jb * tp::W;
     const int nc = min(tp::W, n - c0);
     // acc = B[rows, jb-block]
-    double acc[2][2][2];
+    double acc[tp::FM][2][2];
 #pragma unroll
-    for (int i = 0; i < 2; ++i)
+    for (int i = 0; i < tp::FM; ++i)
 #pragma unroll
       for (int j = 0; j < 2; ++j)
 #pragma unroll
@@ -152,13 +159,13 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
       const double* Bs = As + tp::W * tp::SA;
 #pragma unroll 4
       for (int k0 = 0; k0 < tp::W; k0 += 4) {
-        double a[2], b[2];
+        double a[tp::FM], b[2];
 #pragma unroll
-        for (int i = 0; i < 2; ++i) a[i] = As[(k0 + t) * tp::SA + wm0 + 8 * i + g];
+        for (int i = 0; i < tp::FM; ++i) a[i] = As[(k0 + t) * tp::SA + wm0 + 8 * i + g];
 #pragma unroll
         for (int j = 0; j < 2; ++j) b[j] = negd_tp(Bs[(k0 + t) * tp::SB + wn0 + 8 * j + g]);
 #pragma unroll
-        for (int i = 0; i < 2; ++i)
+        for (int i = 0; i < tp::FM; ++i)
 #pragma unroll
           for (int j = 0; j < 2; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], a[i], b[j]);
       }
@@ -168,16 +175,17 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
     if (jb + 1 < Nb) prologue_pre(jb + 1);
     // ---- diagonal solve: S[r][c] = acc, LdT = L(jb,jb) (landed: waited above), Rc[c] = 1 / L_cc
 #pragma unroll
-    for (int i = 0; i < 2; ++i)
+    for (int i = 0; i < tp::FM; ++i)
 #pragma unroll
       for (int j = 0; j < 2; ++j)
 #pragma unroll
         for (int h = 0; h < 2; ++h) S[(wm0 + 8 * i + g) * tp::SS + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
     if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / LdT[threadIdx.x * tp::SL + threadIdx.x];
     __syncthreads();
-    // warps 0..3 own 16-column chunks; lane = row.  Chunk q solves its columns in
-    // registers, publishes x to S, later chunks subtract its contribution.
-    const int q = warp, r = lane;
+    // thread (q = tid / BM, r = tid % BM), q < 4, owns row r of the 16-column chunk q.
+    // Chunk q solves its columns in registers, publishes x to S, later chunks
+    // subtract its contribution.
+    const int q = threadIdx.x / tp::BM, r = threadIdx.x % tp::BM;
     double b[16];
     if (q < 4) {
 #pragma unroll
@@ -220,16 +228,29 @@ __global__ void __launch_bounds__(tp::NT, 1) trsm_panel_kernel(const double* __r
 }
 
 cudaError_t trsm_panel_init_attrs() {
-  return cudaFuncSetAttribute(trsm_panel_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, tp::SMEM_BYTES);
+  cudaError_t e = cudaFuncSetAttribute(trsm_panel_kernel<32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       TP<32>::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(trsm_panel_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, TP<64>::SMEM_BYTES);
+  return e;
+}
+
+static int trsm_rows() {
+  static int v = [] {
+    const char* e = getenv("STF_TRSM_ROWS");
+    return (e && atoi(e) == 32) ? 32 : 64;
+  }();
+  return v;
 }
 
 cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                        int64_t ldb) {
   if (M <= 0 || n <= 0) return cudaSuccess;
+  const int bm = trsm_rows();
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((M + tp::BM - 1) / tp::BM);
-  cfg.blockDim = dim3(tp::NT);
-  cfg.dynamicSmemBytes = tp::SMEM_BYTES;
+  cfg.gridDim = dim3((M + bm - 1) / bm);
+  cfg.blockDim = dim3(256);
+  cfg.dynamicSmemBytes = bm == 32 ? TP<32>::SMEM_BYTES : TP<64>::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributePriority;
@@ -237,7 +258,8 @@ cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   ++launch_count();
-  return cudaLaunchKernelEx(&cfg, trsm_panel_kernel, L, ldl, n, B, ldb, M);
+  if (bm == 32) return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<32>, L, ldl, n, B, ldb, M);
+  return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<64>, L, ldl, n, B, ldb, M);
 }
 
 }  // namespace stfk
