@@ -93,6 +93,7 @@ struct Exec {
   std::vector<uintptr_t> key_ptrs;
   int64_t key_ld = 0;
   int key_dev = 0;
+  int64_t key_graph = 1;  // graph option requested when the plan was built (opt.graph may fall back to 0)
 
   stf::Plan plan;
   std::vector<double*> buf;           // buffer id -> device pointer
@@ -104,6 +105,7 @@ struct Exec {
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t gexec = nullptr;
   int64_t graph_nodes = 0;
+  int graph_fallback = 0;  // capture failed, eager lowering used
   int64_t launches = 0;
   double build_ms = 0;
   // caller matrix for COLMAJOR kinds
@@ -427,25 +429,43 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
     }
   }
   if (X.opt.graph) {
+    // Capture the whole DAG.  A capture the driver rejects (e.g. a multi-device
+    // topology it cannot express) falls back to the eager stream backend for
+    // this plan: same tasks, same edges, same results.
     cudaSetDevice(C.origin_dev);
-    CUDA_TRY(cudaStreamBeginCapture(C.origin, cudaStreamCaptureModeThreadLocal), "begin capture");
-    int r = fork_streams(C, X.ngpus);
-    Lowerer L{C, X};
-    if (!r) r = L.issue();
-    if (!r) r = join_streams(C, X.ngpus);
-    cudaSetDevice(C.origin_dev);
+    int r = 0;
     cudaGraph_t g = nullptr;
-    cudaError_t e = cudaStreamEndCapture(C.origin, &g);
-    if (r) {
-      if (g) cudaGraphDestroy(g);
-      return r;
+    cudaError_t e = cudaStreamBeginCapture(C.origin, cudaStreamCaptureModeThreadLocal);
+    if (e == cudaSuccess) {
+      r = fork_streams(C, X.ngpus);
+      Lowerer L{C, X};
+      if (!r) r = L.issue();
+      if (!r) r = join_streams(C, X.ngpus);
+      cudaSetDevice(C.origin_dev);
+      e = cudaStreamEndCapture(C.origin, &g);
     }
-    if (e != cudaSuccess) return cuda_fail(e, "end capture");
-    X.graph = g;
-    size_t nn = 0;
-    cudaGraphGetNodes(g, nullptr, &nn);
-    X.graph_nodes = (int64_t)nn;
-    CUDA_TRY(cudaGraphInstantiateWithFlags(&X.gexec, g, cudaGraphInstantiateFlagUseNodePriority), "graph instantiate");
+    if (r == 0 && e == cudaSuccess && g) {
+      e = cudaGraphInstantiateWithFlags(&X.gexec, g, cudaGraphInstantiateFlagUseNodePriority);
+      if (e == cudaSuccess) {
+        X.graph = g;
+        size_t nn = 0;
+        cudaGraphGetNodes(g, nullptr, &nn);
+        X.graph_nodes = (int64_t)nn;
+      }
+    }
+    if (!X.gexec) {
+      if (g) cudaGraphDestroy(g);
+      if (r == -103) return r;  // out of memory is not a capture problem
+      cudaGetLastError();
+      for (int d : C.devices) {  // drain anything a partial capture may have left behind
+        cudaSetDevice(d);
+        cudaDeviceSynchronize();
+      }
+      cudaGetLastError();
+      g_err.clear();
+      X.opt.graph = 0;
+      X.graph_fallback = 1;
+    }
   }
   X.build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return 0;
@@ -768,7 +788,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     Exec& e = **it;
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
         e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
-        (e.opt.graph == C.opt.graph || A_desc->kind == STF_DESC_HOST_COLMAJOR) &&
+        e.key_graph == C.opt.graph &&
         e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
@@ -789,6 +809,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     e->P = P;
     e->Q = Q;
     e->opt = C.opt;
+    e->key_graph = C.opt.graph;
     e->key_ptrs = ptrs;
     e->key_ld = A_desc->ld;
     e->key_dev = A_desc->device;
@@ -798,7 +819,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
       C.cache.clear();
       e.reset(new Exec());
       e->n = n; e->nb = nb; e->uplo = up; e->kind = A_desc->kind; e->ngpus = ngpus; e->P = P; e->Q = Q;
-      e->opt = C.opt; e->key_ptrs = ptrs; e->key_ld = A_desc->ld; e->key_dev = A_desc->device;
+      e->opt = C.opt; e->key_graph = C.opt.graph; e->key_ptrs = ptrs; e->key_ld = A_desc->ld; e->key_dev = A_desc->device;
       if (A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr)) e->opt.graph = 0;
       g_err.clear();
       r = prepare(C, *e, A_desc);
