@@ -255,9 +255,17 @@ def run_ours(args, rank, world):
                           "frac": round(fl / (ms.value * 1e-3) / 1e12 / FP64_PEAK_TFLOPS, 4),
                           "shape": [M_, N_, K_ if kind in (0, 1) else None]}
     roof["kernels_alone"] = kern
-    traffic = load_traffic()
-    if traffic is not None:
-        roof["traffic"] = traffic
+    # dominant kernel: the GEMM tile update (GEMM+SYRK are (T-1)(T-2)/T^2 + (T-1)/T^2 of the flops)
+    T = n // nb
+    tr = load_traffic()
+    dom = {"name": "gemm_nt_dmma (GEMM/SYRK tile update C -= A B^T)",
+           "flop_share": round(((T - 1) * (T - 2) + (T - 1)) / T ** 2, 4),
+           "launches_per_step": (T - 1) * T // 2,
+           "alone_tile": kern.get("gemm_tile"), "alone_full_occupancy": kern.get("gemm_full"),
+           "traffic_bytes_per_tile_launch": tr, "algorithmic_bytes_per_tile_launch": 4 * nb * nb * 8}
+    roof["dominant_kernel"] = dom
+    roof["traffic_note"] = ("the launch unit is the whole-DAG graph; per-kernel DRAM traffic is in "
+                            "dominant_kernel (ncu --set full, profiles/gemm_traffic.json)")
 
     cpu = None
     if N == 1 and not args.no_cpu:

@@ -104,6 +104,8 @@ const char *stf_last_error(void);
  *   "serial"   STF_SERIAL   1: every task on one stream in program order (race check)
  *   "priority" STF_PRIO     1: critical-path tasks on high-priority streams (default 1)
  *   "grid_p"   STF_GRID     rows P of the P x Q grid for COLMAJOR kinds (0 = auto)
+ *   "lookahead" STF_LOOKAHEAD 1: pure STF DAG (default); 0: a fence task closes every
+ *                           panel step (no look-ahead; ablation of PAPER.md:399)
  * Returns 0 or -105. */
 int stf_set_option(const char *name, int64_t value);
 int stf_get_option(const char *name, int64_t *value);
@@ -130,7 +132,7 @@ int stf_last_stats(stf_plan_stats *out);
 /* Build (without running) the STF DAG of a T x T tile Cholesky on a p x q grid
  * and copy up to `cap` edges (src, dst pairs of task indices in submission
  * order) into edges[2*cap].  kinds[cap_tasks] receives per-task codes
- * (0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM, 4 COPY) and ijk[3*cap_tasks] the (i, j, k)
+ * (0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM, 4 COPY, 7 FENCE) and ijk[3*cap_tasks] the (i, j, k)
  * indices (for COPY: tile i, j and destination slot k).  Any output pointer
  * may be NULL.  Fills *stats.  Needs no GPU. */
 int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t *edges, int64_t cap_tasks, int32_t *kinds,

@@ -16,7 +16,7 @@ STF_DESC_TILED_2DBC = 0
 STF_DESC_DEVICE_COLMAJOR = 1
 STF_DESC_HOST_COLMAJOR = 2
 
-KIND_NAMES = {0: "POTRF", 1: "TRSM", 2: "SYRK", 3: "GEMM", 4: "COPY", 5: "LOAD", 6: "STORE"}
+KIND_NAMES = {0: "POTRF", 1: "TRSM", 2: "SYRK", 3: "GEMM", 4: "COPY", 5: "LOAD", 6: "STORE", 7: "FENCE"}
 
 
 class stf_matrix_desc(ctypes.Structure):

@@ -62,10 +62,11 @@ struct DfParams {
   int Mb, Nb;  // block grid of X
   const uint32_t* tasks;
   int ntasks;
-  int* ws;  // ws[0] ticket, ws[1 + ib * Nb + jb] progress
+  int* ws;  // ws[0] ticket, ws[1] critical-chain role, ws[2 + ib * Nb + jb] progress
   int64_t col0;
   unsigned long long* info;
   int potrf;
+  int crit;  // POTRF: one CTA runs the critical chain P -> S -> U -> P (blocks kept in smem)
 };
 
 __device__ __forceinline__ int ld_acquire(const int* p) {
@@ -160,23 +161,15 @@ __device__ __forceinline__ void named_bar(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// S: X[rows x nc] <- X L^-T, L nc x nc lower.  Thread (r = tid & 63, q = tid >> 6)
-// holds X[r, 16q .. 16q+15] in registers.  Chunk q solves its 16 columns by
-// substitution (divisions by L_cc), publishes x to smem, later chunks subtract
-// x L^T; every element accumulates its terms in increasing column order.
-__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc) {
-  double* Xs = sm;                    // Xs[r][c]
-  double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
+// Substitution core.  Thread (r = tid & 63, q = tid >> 6) holds X[r, 16q .. 16q+15]
+// in b[].  Ls[c * LDB + p] = L(c, p) (lower part read only).  Chunk q solves its
+// 16 columns (correctly rounded divisions via div_by), publishes them to
+// Xpub[r * ldp + col], later chunks subtract x L^T; every element accumulates
+// its terms in increasing column order.  On return b[] holds the solution and
+// Xpub all of it.
+__device__ __forceinline__ void solve_core(double (&b)[16], const double* Ls, double* Rc, double* Xpub, int ldp,
+                                           int nc) {
   const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
-  double b[16];
-#pragma unroll
-  for (int c = 0; c < 16; ++c) {
-    const int col = 16 * q + c;
-    b[c] = (r < rows && col < nc) ? __ldcg(X + (int64_t)col * ldx + r) : 0.0;
-  }
-  load_block_rm(Ls, df::LDB, L, ldl, nc, nc, true);
-  double* Rc = Ls + df::W * df::LDB;
-  __syncthreads();
   if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / Ls[threadIdx.x * df::LDB + threadIdx.x];
   __syncthreads();
   for (int qq = 0; qq < 4 && 16 * qq < nc; ++qq) {
@@ -191,7 +184,7 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
         }
       }
 #pragma unroll
-      for (int c = 0; c < 16; ++c) Xs[r * df::LDB + 16 * qq + c] = b[c];
+      for (int c = 0; c < 16; ++c) Xpub[r * ldp + 16 * qq + c] = b[c];
     }
     __syncthreads();
     if (q > qq) {
@@ -199,33 +192,20 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
       for (int cc = 0; cc < 16; ++cc)
 #pragma unroll
         for (int c = 0; c < 16; ++c)
-          b[cc] = fma(-Xs[r * df::LDB + 16 * qq + c], Ls[(16 * q + cc) * df::LDB + 16 * qq + c], b[cc]);
-    }
-  }
-  if (r < rows) {
-#pragma unroll
-    for (int c = 0; c < 16; ++c) {
-      const int col = 16 * q + c;
-      if (col < nc) X[(int64_t)col * ldx + r] = b[c];
+          b[cc] = fma(-Xpub[r * ldp + 16 * qq + c], Ls[(16 * q + cc) * df::LDB + 16 * qq + c], b[cc]);
     }
   }
 }
 
-// P: in-place lower Cholesky of the nc x nc diagonal block.  Thread (r, q) holds
-// A[r, 16q .. 16q+15]; chunk q (two warps, named barrier 1+q) factors its 16
-// columns (pivot sqrt by the owner of row col, column scaled by division,
-// in-chunk rank-1 updates), publishes them, and later chunks apply the
+// Cholesky core of an nc x nc block.  Thread (r, q) holds A[r, 16q .. 16q+15]
+// (lower part) in a[]; chunk q (two warps, named barrier 1+q) factors its 16
+// columns (pivot sqrt by the owner of row col, division by the pivot, in-chunk
+// rank-1 updates), publishing L into S[r * LDB + col]; later chunks apply the
 // chunk's update.  Element updates run in increasing column order (Crout order).
-__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
-  double* S = sm;  // S[r][c]: published L values
-  double* Y = sm + df::W * df::LDB;  // Y[c] = 1 / L_cc
+// On return a[] holds L and S its lower part (diagonal included).
+__device__ __forceinline__ void chol_core(double (&a)[16], double* S, double* Y, int nc, int64_t col0,
+                                          unsigned long long* info) {
   const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
-  double a[16];
-#pragma unroll
-  for (int c = 0; c < 16; ++c) {
-    const int col = 16 * q + c;
-    a[c] = (r < nc && col < nc && r >= col) ? __ldcg(X + (int64_t)col * ldx + r) : 0.0;
-  }
   for (int qq = 0; qq < 4 && 16 * qq < nc; ++qq) {
     if (q == qq) {
 #pragma unroll
@@ -270,12 +250,141 @@ __device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t co
       }
     }
   }
-  if (r < nc) {
+}
+
+__device__ __forceinline__ void load_chunk(double (&v)[16], const double* G, int64_t ldg, int rows, int nc,
+                                           bool lower) {
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
+#pragma unroll
+  for (int c = 0; c < 16; ++c) {
+    const int col = 16 * q + c;
+    v[c] = (r < rows && col < nc && (!lower || r >= col)) ? __ldcg(G + (int64_t)col * ldg + r) : 0.0;
+  }
+}
+__device__ __forceinline__ void store_chunk(const double (&v)[16], double* G, int64_t ldg, int rows, int nc,
+                                            bool lower) {
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
+  if (r < rows) {
 #pragma unroll
     for (int c = 0; c < 16; ++c) {
       const int col = 16 * q + c;
-      if (col < nc && r >= col) X[(int64_t)col * ldx + r] = a[c];
+      if (col < nc && (!lower || r >= col)) G[(int64_t)col * ldg + r] = v[c];
     }
+  }
+}
+
+// S task: X[rows x nc] <- X L^-T with L = the nc x nc diagonal block at L (global).
+__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc) {
+  double* Xs = sm;                    // publication buffer [r][LDB]
+  double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
+  double* Rc = Ls + df::W * df::LDB;
+  double b[16];
+  load_chunk(b, X, ldx, rows, nc, false);
+  load_block_rm(Ls, df::LDB, L, ldl, nc, nc, true);
+  __syncthreads();
+  solve_core(b, Ls, Rc, Xs, df::LDB, nc);
+  store_chunk(b, X, ldx, rows, nc, false);
+}
+
+// P task: in-place lower Cholesky of the nc x nc diagonal block at X (global).
+__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
+  double* S = sm;
+  double* Y = sm + df::W * df::LDB;
+  double a[16];
+  load_chunk(a, X, ldx, nc, nc, true);
+  chol_core(a, S, Y, nc, col0, info);
+  store_chunk(a, X, ldx, nc, nc, true);
+}
+
+// The critical path of the tile Cholesky, run by ONE CTA with its blocks kept
+// in shared memory: P(kb) -> S(kb+1, kb) -> U(kb+1, kb+1, kb) -> P(kb+1) -> ...
+// (bulk CTAs run every other task).  Saves the global round trip, the flag
+// hand-off and the block reloads between consecutive critical tasks.
+__device__ void critical_chain(const DfParams& p, double* sm) {
+  constexpr int W = df::W;
+  const int T = p.Nb;
+  double* D = sm;                          // [r][LDB]: P publication buffer -> L_kk
+  double* XS = sm + W * df::LDB;           // [r][LDO]: X(kb+1, kb), A and B of U
+  double* Rc = XS + W * df::LDO;           // W
+  double* Y = Rc + W;                      // W
+  int* prog = p.ws + 2;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const int wm0 = (warp & 1) * 32, wn0 = (warp >> 1) * 16;
+  const int r = threadIdx.x & (W - 1), q = threadIdx.x >> 6;
+  double a[16];
+  load_chunk(a, p.X, p.ldx, min(W, p.n), min(W, p.n), true);  // P(0) input: nothing precedes it
+  for (int kb = 0; kb < T; ++kb) {
+    const int nk = min(W, p.n - kb * W);
+    double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
+    // ---- P(kb)
+    chol_core(a, D, Y, nk, p.col0 + (int64_t)kb * W, p.info);
+    store_chunk(a, Xkk, p.ldx, nk, nk, true);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      st_release(&prog[kb * p.Nb + kb], kb + 1);
+    }
+    if (kb + 1 == T) return;
+    // ---- S(ib, kb), ib = kb + 1, with L_kk from D
+    const int ib = kb + 1, rows = min(W, p.n - ib * W);
+    double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
+    if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + kb], kb);
+    __syncthreads();
+    double b[16];
+    load_chunk(b, Xik, p.ldx, rows, nk, false);
+    solve_core(b, D, Rc, XS, df::LDO, nk);
+    store_chunk(b, Xik, p.ldx, rows, nk, false);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      st_release(&prog[ib * p.Nb + kb], kb + 1);
+    }
+    // ---- U(ib, ib, kb): D <- lower(C - X X^T), C = block (ib, ib) after all earlier updates
+    if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + ib], kb);
+    __syncthreads();
+    double* Cii = p.X + (int64_t)ib * W * p.ldx + ib * W;
+    double acc[4][2][2];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int rr = wm0 + 8 * i + g, cc = wn0 + 8 * j + 2 * t + h;
+          acc[i][j][h] = (rr < rows && cc < rows && rr >= cc) ? __ldcg(Cii + (int64_t)cc * p.ldx + rr) : 0.0;
+        }
+    // operands: A(m, k) = B(m, k) = X(m, k) = XS[m * LDO + k]; columns k >= nk are zero-padded below
+    if (nk < W)
+      for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+        const int m = idx >> 6, k = idx & (W - 1);
+        if (k >= nk) XS[m * df::LDO + k] = 0.0;
+      }
+    __syncthreads();
+#pragma unroll 4
+    for (int k0 = 0; k0 < W; k0 += 4) {
+      double av[4], bv[2];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) av[i] = XS[(wm0 + 8 * i + g) * df::LDO + k0 + t];
+#pragma unroll
+      for (int j = 0; j < 2; ++j) bv[j] = negd(XS[(wn0 + 8 * j + g) * df::LDO + k0 + t]);
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) dmma_8x8x4(acc[i][j][0], acc[i][j][1], av[i], bv[j]);
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) D[(wm0 + 8 * i + g) * df::LDB + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
+    __syncthreads();
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      const int col = 16 * q + c;
+      a[c] = (r < rows && col < rows && r >= col) ? D[r * df::LDB + col] : 0.0;
+    }
+    __syncthreads();  // D is rewritten by the next chol_core
   }
 }
 
@@ -283,6 +392,17 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
   extern __shared__ __align__(16) double sm[];
   __shared__ int s_task;
   const int W = df::W;
+  int* prog = p.ws + 2;
+  if (p.crit) {
+    // the first CTA to start takes the critical chain (it is resident by construction)
+    if (threadIdx.x == 0) s_task = (atomicCAS(&p.ws[1], 0, 1) == 0);
+    __syncthreads();
+    if (s_task) {
+      critical_chain(p, sm);
+      return;
+    }
+    __syncthreads();
+  }
   for (;;) {
     if (threadIdx.x == 0) s_task = atomicAdd(&p.ws[0], 1);
     __syncthreads();
@@ -291,7 +411,6 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
     const uint32_t code = p.tasks[ticket];
     const uint32_t type = code >> 30;
     const int ib = (code >> 20) & 1023, jb = (code >> 10) & 1023, kb = code & 1023;
-    int* prog = p.ws + 1;
     const int rows = min(W, p.m - ib * W);
     if (threadIdx.x == 0) {
       if (p.potrf) {
@@ -350,9 +469,23 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
 // ------------------------------------------------------------------ host side
 namespace {
 
-std::vector<uint32_t> build_tasks(bool potrf, int Mb, int Nb) {
+bool on_chain(uint32_t code) {  // P(kb), S(kb+1, kb), U(kb+1, kb+1, kb)
+  const uint32_t type = code >> 30;
+  const int ib = (code >> 20) & 1023, jb = (code >> 10) & 1023, kb = code & 1023;
+  if (type == df::T_P) return true;
+  if (type == df::T_S) return ib == kb + 1;
+  return ib == kb + 1 && jb == kb + 1;
+}
+
+std::vector<uint32_t> build_tasks(bool potrf, int Mb, int Nb, bool crit) {
   std::vector<uint32_t> t;
   using df::enc;
+  if (potrf && crit) {
+    std::vector<uint32_t> all = build_tasks(true, Mb, Nb, false);
+    for (uint32_t c : all)
+      if (!on_chain(c)) t.push_back(c);
+    return t;
+  }
   if (potrf) {
     const int T = Nb;
     // look-ahead-1 topological order (see header comment)
@@ -383,14 +516,15 @@ std::vector<uint32_t> build_tasks(bool potrf, int Mb, int Nb) {
 }
 
 std::mutex g_mu;
-std::map<std::tuple<int, int, int, int>, std::pair<uint32_t*, int>> g_tables;  // (dev, potrf, Mb, Nb)
+std::map<std::tuple<int, int, int, int>, std::pair<uint32_t*, int>> g_tables;  // (dev, mode, Mb, Nb)
 int g_num_sms[64];
 
-cudaError_t get_table(bool potrf, int Mb, int Nb, const uint32_t** out, int* count) {
+// mode: 0 TRSM, 1 POTRF (all tasks), 2 POTRF without the critical chain
+cudaError_t get_table(int mode, int Mb, int Nb, const uint32_t** out, int* count) {
   int dev = 0;
   cudaGetDevice(&dev);
   std::lock_guard<std::mutex> g(g_mu);
-  auto key = std::make_tuple(dev, (int)potrf, Mb, Nb);
+  auto key = std::make_tuple(dev, mode, Mb, Nb);
   auto it = g_tables.find(key);
   if (it != g_tables.end()) {
     *out = it->second.first;
@@ -399,7 +533,7 @@ cudaError_t get_table(bool potrf, int Mb, int Nb, const uint32_t** out, int* cou
   }
   // Must not be called while a stream is being captured (cudaMemcpy); the runtime
   // calls dataflow_prepare() before capture.
-  std::vector<uint32_t> t = build_tasks(potrf, Mb, Nb);
+  std::vector<uint32_t> t = build_tasks(mode >= 1, Mb, Nb, mode == 2);
   uint32_t* d = nullptr;
   cudaError_t e = cudaMalloc(&d, t.size() * sizeof(uint32_t));
   if (e != cudaSuccess) return e;
@@ -433,7 +567,7 @@ cudaError_t launch_df(cudaStream_t s, int prio, DfParams& p, int max_ctas) {
   cudaError_t e = cudaMemsetAsync(p.ws, 0, dataflow_ws_bytes(p.m, p.n), s);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
-  int grid = p.ntasks < max_ctas ? p.ntasks : max_ctas;
+  int grid = max_ctas;
   if (grid < 1) grid = 1;
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(df::NT);
@@ -452,14 +586,25 @@ cudaError_t launch_df(cudaStream_t s, int prio, DfParams& p, int max_ctas) {
 
 size_t dataflow_ws_bytes(int m, int n) {
   const int Mb = (m + df::W - 1) / df::W, Nb = (n + df::W - 1) / df::W;
-  return ((size_t)(1 + Mb * Nb) * sizeof(int) + 255) / 256 * 256;
+  return ((size_t)(2 + Mb * Nb) * sizeof(int) + 255) / 256 * 256;
 }
 
 cudaError_t dataflow_prepare(int m, int n, bool potrf) {
   const int Mb = (m + df::W - 1) / df::W, Nb = (n + df::W - 1) / df::W;
   const uint32_t* t;
   int c;
-  return get_table(potrf, Mb, Nb, &t, &c);
+  if (!potrf) return get_table(0, Mb, Nb, &t, &c);
+  cudaError_t e = get_table(1, Mb, Nb, &t, &c);
+  if (e == cudaSuccess) e = get_table(2, Mb, Nb, &t, &c);
+  return e;
+}
+
+static int df_crit() {
+  static int v = [] {
+    const char* e = getenv("STF_DF_CRIT");
+    return e ? atoi(e) : 1;
+  }();
+  return v;
 }
 
 cudaError_t dataflow_init_attrs() {
@@ -476,7 +621,8 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   p.ldl = 0;
   p.m = p.n = n;
   p.Mb = p.Nb = (n + df::W - 1) / df::W;
-  cudaError_t e = get_table(true, p.Mb, p.Nb, &p.tasks, &p.ntasks);
+  p.crit = df_crit();
+  cudaError_t e = get_table(p.crit ? 2 : 1, p.Mb, p.Nb, &p.tasks, &p.ntasks);
   if (e != cudaSuccess) return e;
   p.ws = ws;
   p.col0 = col0;
@@ -484,7 +630,9 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   p.potrf = 1;
   const int T = p.Nb;
   const int par = T * (T - 1) / 2 > 0 ? T * (T - 1) / 2 : 1;  // widest update wave
-  return launch_df(stream, prio, p, std::min(par, std::min(df_max_ctas(), num_sms())));
+  int ctas = std::min(par, std::min(df_max_ctas(), num_sms()));
+  if (p.crit) ctas = std::min(p.ntasks, ctas - 1) + 1;  // + the critical-chain CTA
+  return launch_df(stream, prio, p, ctas);
 }
 
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
@@ -499,12 +647,13 @@ cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double*
   p.n = n;
   p.Mb = (M + df::W - 1) / df::W;
   p.Nb = (n + df::W - 1) / df::W;
-  cudaError_t e = get_table(false, p.Mb, p.Nb, &p.tasks, &p.ntasks);
+  cudaError_t e = get_table(0, p.Mb, p.Nb, &p.tasks, &p.ntasks);
   if (e != cudaSuccess) return e;
   p.ws = ws;
   p.col0 = 0;
   p.info = nullptr;
   p.potrf = 0;
+  p.crit = 0;
   const int par = p.Mb * (p.Nb > 1 ? p.Nb - 1 : 1);
   return launch_df(stream, prio, p, std::min(par, std::min(4 * df_max_ctas(), num_sms())));
 }

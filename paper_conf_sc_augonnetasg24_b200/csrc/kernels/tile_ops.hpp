@@ -43,10 +43,11 @@ cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double*
                       int64_t ldb, int* ws);
 size_t dataflow_ws_bytes(int m, int n);
 
-// K3 row-panel form (trsm_panel.cu): one launch, ceil(M/32) CTAs each owning 32
-// rows, left-looking over 64-wide column blocks (DMMA update + substitution).
+// K3 row-panel form (trsm_panel.cu): one launch, ceil(M/R) CTAs each owning R
+// rows (R = 32: lower latency, 64: higher efficiency; 0 = STF_TRSM_ROWS, default
+// 64), left-looking over 64-wide column blocks (DMMA update + substitution).
 cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
-                       int64_t ldb);
+                       int64_t ldb, int rows_per_cta = 0);
 cudaError_t dataflow_prepare(int m, int n, bool potrf);
 
 // K8: fill rows r0.., cols c0.. (global indices) of the seeded SPD metric matrix

@@ -244,9 +244,9 @@ static int trsm_rows() {
 }
 
 cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
-                       int64_t ldb) {
+                       int64_t ldb, int rows_per_cta) {
   if (M <= 0 || n <= 0) return cudaSuccess;
-  const int bm = trsm_rows();
+  const int bm = rows_per_cta == 32 || rows_per_cta == 64 ? rows_per_cta : trsm_rows();
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((M + bm - 1) / bm);
   cfg.blockDim = dim3(256);

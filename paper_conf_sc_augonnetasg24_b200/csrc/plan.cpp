@@ -110,6 +110,12 @@ struct Builder {
         compute(K_SYRK, i, i, k, prio && i == k + 1, key(i, k), -1, i, i);
         for (int64_t j = k + 1; j < i; ++j) compute(K_GEMM, i, j, k, prio && j == k + 1, key(i, k), key(j, k), i, j);
       }
+      if (!p.opt.lookahead && k + 1 < T) {
+        std::vector<Access> acc;
+        for (int64_t d = 0; d < p.ntiles(); ++d) acc.push_back({d, RW});
+        Task f{K_FENCE, (int32_t)k, (int32_t)k, (int32_t)k, 0, 1, 0, {-1, -1}, -1};
+        submit(f, acc.data(), (int)acc.size());
+      }
     }
     if (p.opt.with_store) {
       for (int64_t j = 0; j < T; ++j)

@@ -27,7 +27,7 @@
 
 namespace stf {
 
-enum Kind : int32_t { K_POTRF = 0, K_TRSM = 1, K_SYRK = 2, K_GEMM = 3, K_COPY = 4, K_LOAD = 5, K_STORE = 6 };
+enum Kind : int32_t { K_POTRF = 0, K_TRSM = 1, K_SYRK = 2, K_GEMM = 3, K_COPY = 4, K_LOAD = 5, K_STORE = 6, K_FENCE = 7 };
 
 struct Task {
   int32_t kind;
@@ -49,6 +49,8 @@ struct PlanOptions {
   bool priority = true;
   bool with_load = false;  // LOAD tasks first (COLMAJOR descriptors)
   bool with_store = false; // STORE tasks (write-back) at the end of program order
+  bool lookahead = true;   // false: a FENCE task (RW on every tile) closes each panel step, so
+                           // step k+1 starts only when step k is complete (ablation, NEXT-1)
 };
 
 // A "buffer" is one physical nb x nb tile instance: home tiles are buffers

@@ -81,6 +81,7 @@ struct Options {
   int64_t serial = 0;
   int64_t priority = 1;
   int64_t grid_p = 0;
+  int64_t lookahead = 1;
 };
 
 // A plan bound to physical buffers, plus its lowering artefacts.
@@ -164,6 +165,7 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.priority = o.priority != 0;
   po.with_load = load;
   po.with_store = store;
+  po.lookahead = o.lookahead != 0;
   return po;
 }
 
@@ -201,8 +203,9 @@ struct Lowerer {
                    "POTRF launch");
         return 0;
       case stf::K_TRSM:
-        if (X.opt.trsm == 2)
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb),
+        if (X.opt.trsm == 2)  // the next panel's TRSM(k+1,k) is on the critical path: low-latency variant
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb,
+                                    t.i == t.k + 1 ? 32 : 0),
                    "TRSM launch");
         else if (X.opt.trsm == 1)
           CUDA_TRY(stfk::trsm_tile(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, ws),
@@ -231,6 +234,8 @@ struct Lowerer {
                    "replica peer copy");
         return 0;
       }
+      case stf::K_FENCE:
+        return 0;  // ordering only: its waits (and event record) are the whole task
       case stf::K_LOAD:
       case stf::K_STORE: {
         const bool load = t.kind == stf::K_LOAD;
@@ -586,6 +591,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.trsm = env_int("STF_TRSM", 2);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
+  C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
   C.opt.priority = env_int("STF_PRIO", 1);
   C.opt.grid_p = 0;
   if (const char* gs = getenv("STF_GRID")) C.opt.grid_p = atoi(gs);
@@ -721,6 +727,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "trsm") *value = C.opt.trsm;
   else if (n == "streams") *value = C.opt.streams;
   else if (n == "serial") *value = C.opt.serial;
+  else if (n == "lookahead") *value = C.opt.lookahead;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;
   else return fail(-105, "unknown option '%s'", name);
@@ -789,7 +796,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
         e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
         e.key_graph == C.opt.graph &&
-        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.key_ptrs == ptrs &&
+        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.opt.lookahead == C.opt.lookahead && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
       C.cache.splice(C.cache.begin(), C.cache, it);
