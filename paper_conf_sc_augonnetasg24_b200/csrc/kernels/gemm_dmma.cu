@@ -35,9 +35,9 @@
 
 namespace stfk {
 
-template <int BK_, int STAGES_>
+template <int BK_, int STAGES_, int BN_ = 128, int MINB_ = 1>
 struct Cfg {
-  static constexpr int BM = 128, BN = 128, BK = BK_, STAGES = STAGES_;
+  static constexpr int BM = 128, BN = BN_, BK = BK_, STAGES = STAGES_, MINB = MINB_;
   static constexpr int BOX = 16;                  // doubles per 128-byte swizzle row
   static constexpr int BOX_BYTES = BOX * BK * 8;  // 2 KB at BK = 16
   static constexpr int A_BYTES = BM * BK * 8;     // 16 KB at BK = 16
@@ -47,6 +47,7 @@ struct Cfg {
 };
 using CfgK16 = Cfg<16, 4>;  // 4 x 32 KB stages
 using CfgK32 = Cfg<32, 3>;  // 3 x 64 KB stages
+using CfgN64 = Cfg<32, 2, 64, 2>;  // 128 x 64 CTA tile, 4 warps, 2 x 48 KB stages, 2 CTAs / SM (full GEMMs only)
 
 // Exact negation as a sign-bit flip on the integer pipe (keeps the FP64/DMMA pipe free).
 __device__ __forceinline__ double neg(double x) {
@@ -78,7 +79,7 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
 // arrival counter), i.e. at the earliest possible moment, with the next k-tile
 // STAGES ahead; consumers wait only on the TMA "full" mbarriers.
 template <int WM, int WN, class g>
-__global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, 1)
+__global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         double* __restrict__ C, int64_t ldc, int M, int N, int K, int lower) {
   constexpr int NCW = (g::BM / WM) * (g::BN / WN);
@@ -237,17 +238,23 @@ static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int c
 
 // Variants: warps 8 (64x32 warp tiles, 224 regs, 2 warps / SM sub-partition) or
 // 16 (32x32, <= 128 regs, 4 warps / sub-partition); BK 16 (4 stages) or 32 (3
-// stages).  STF_GEMM_WARPS / STF_GEMM_BK select; defaults 16 warps, BK 32.
+// stages).  STF_GEMM_WARPS / STF_GEMM_BK select; defaults 8 warps, BK 32 (best
+// in the concurrent factorisation, profiles/r01/ablations_*.txt).
 static int env_or(const char* name, int dflt) {
   const char* e = getenv(name);
   return e ? atoi(e) : dflt;
 }
 static int gemm_warps() {
-  static int v = env_or("STF_GEMM_WARPS", 16) == 8 ? 8 : 16;
+  static int v = env_or("STF_GEMM_WARPS", 8) == 16 ? 16 : 8;
   return v;
 }
 static int gemm_bk() {
   static int v = env_or("STF_GEMM_BK", 32) == 16 ? 16 : 32;
+  return v;
+}
+// STF_GEMM_NARROW=1: full (non-SYRK) GEMMs use the 128 x 64 tile, 2 CTAs per SM
+static int gemm_narrow() {
+  static int v = env_or("STF_GEMM_NARROW", 0);
   return v;
 }
 
@@ -268,11 +275,12 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
     return cudaErrorMisalignedAddress;
-  const int bk = gemm_bk();
+  const bool narrow = !lower && gemm_narrow();
+  const int bk = narrow ? 32 : gemm_bk();
   CUtensorMap tmA, tmB;
   if (!make_operand_map(&tmA, A, M, K, lda, bk) || !make_operand_map(&tmB, B, N, K, ldb, bk))
     return cudaErrorInvalidValue;
-  const int tM = (M + 127) / 128, tN = (N + 127) / 128;
+  const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = lower ? dim3(tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
   cfg.stream = stream;
@@ -282,6 +290,11 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   ++launch_count();
+  if (narrow) {
+    cfg.dynamicSmemBytes = CfgN64::SMEM_BYTES;
+    cfg.blockDim = dim3(128, 1, 1);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, CfgN64>, tmA, tmB, C, ldc, M, N, K, lower);
+  }
   if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
   return launch_variant<CfgK16>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
 }
@@ -299,6 +312,9 @@ static cudaError_t set_attrs() {
 cudaError_t gemm_init_attrs() {
   cudaError_t e = set_attrs<CfgK16>();
   if (e == cudaSuccess) e = set_attrs<CfgK32>();
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<64, 32, CfgN64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             CfgN64::SMEM_BYTES);
   return e;
 }
 

@@ -34,7 +34,7 @@ struct Builder {
 
   int compute_stream(const Task& t) const {
     if (p.opt.serial) return 0;
-    if (p.opt.priority && t.prio) {
+    if (p.opt.priority && t.prio >= 4) {
       if (t.kind == K_POTRF) return 0;
       return (int)(t.i % p.opt.crit_streams);
     }
@@ -102,13 +102,19 @@ struct Builder {
         }
     }
     auto key = [&](int64_t i, int64_t j) { return i * T + j; };
+    // Priority levels 0..5 (5 = most urgent), by how soon the written tile feeds a
+    // panel: POTRF, the next panel's TRSM and SYRK are on the critical path (5);
+    // the other TRSMs and the next column's GEMMs gate the next panel (4); later
+    // columns decay with their distance d = column - k.
     const bool prio = p.opt.priority;
+    auto level = [&](int64_t d) -> int { return d <= 1 ? 4 : d == 2 ? 3 : d <= 4 ? 2 : d <= 8 ? 1 : 0; };
+    auto P = [&](int lv) { return prio ? lv : 0; };
     for (int64_t k = 0; k < T; ++k) {
-      compute(K_POTRF, k, k, k, 1, -1, -1, k, k);
-      for (int64_t i = k + 1; i < T; ++i) compute(K_TRSM, i, k, k, 1, key(k, k), -1, i, k);
+      compute(K_POTRF, k, k, k, P(5), -1, -1, k, k);
+      for (int64_t i = k + 1; i < T; ++i) compute(K_TRSM, i, k, k, P(i == k + 1 ? 5 : 4), key(k, k), -1, i, k);
       for (int64_t i = k + 1; i < T; ++i) {
-        compute(K_SYRK, i, i, k, prio && i == k + 1, key(i, k), -1, i, i);
-        for (int64_t j = k + 1; j < i; ++j) compute(K_GEMM, i, j, k, prio && j == k + 1, key(i, k), key(j, k), i, j);
+        compute(K_SYRK, i, i, k, P(i == k + 1 ? 5 : level(i - k)), key(i, k), -1, i, i);
+        for (int64_t j = k + 1; j < i; ++j) compute(K_GEMM, i, j, k, P(level(j - k)), key(i, k), key(j, k), i, j);
       }
       if (!p.opt.lookahead && k + 1 < T) {
         std::vector<Access> acc;

@@ -33,7 +33,7 @@ struct Task {
   int32_t kind;
   int32_t i, j, k;   // tile indices (COPY/LOAD/STORE: tile (i,j); COPY: k = destination slot)
   int32_t slot;      // executing slot (COPY: source slot, push model)
-  int32_t prio;      // 1 = critical path (high-priority stream), 0 = bulk
+  int32_t prio;      // urgency level 0..5 (5 = critical path); >= 4 runs on the high-priority streams
   int32_t stream;    // index into the slot's stream pool (see Lowering in runtime.cpp)
   int64_t in[2];     // buffer ids read (-1 if unused)
   int64_t out;       // buffer id written

@@ -182,10 +182,13 @@ struct Lowerer {
     }
   }
   cudaStream_t stream_of(const stf::Task& t) { return C.slots[(size_t)t.slot].streams[(size_t)t.stream]; }
+  // level 5 -> the device's greatest priority, each level below one step lower (clamped)
   int prio_of(const stf::Task& t) {
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    return (X.opt.priority && t.prio) ? hi : lo;
+    if (!X.opt.priority) return lo;
+    const int v = hi + (5 - t.prio);
+    return v > lo ? lo : v;
   }
 
   int body(const stf::Task& t, size_t tidx, cudaStream_t s, int prio) {

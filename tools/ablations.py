@@ -16,7 +16,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 VARIANTS = [
-    ("default (pool 4 crit + 8 bulk streams, priorities, graph, look-ahead)", {}),
+    ("default (pool 4 crit + 8 bulk streams, graded priorities, graph, look-ahead)", {}),
     ("single stream (STF_SERIAL=1)  [paper: -5% on 1 GPU]", {"STF_SERIAL": "1"}),
     ("2 bulk streams", {"STF_STREAMS": "2"}),
     ("16 bulk streams", {"STF_STREAMS": "16"}),
@@ -26,7 +26,7 @@ VARIANTS = [
     ("TRSM dataflow kernel (STF_TRSM=1)", {"STF_TRSM": "1"}),
     ("TRSM row panel 32 rows (STF_TRSM_ROWS=32)", {"STF_TRSM_ROWS": "32"}),
     ("TRSM + POTRF recursive (STF_TRSM=0 STF_DATAFLOW=0)", {"STF_TRSM": "0", "STF_DATAFLOW": "0"}),
-    ("GEMM 8 warps 64x32 (STF_GEMM_WARPS=8)", {"STF_GEMM_WARPS": "8"}),
+    ("GEMM 16 warps 32x32 (STF_GEMM_WARPS=16)", {"STF_GEMM_WARPS": "16"}),
     ("GEMM BK=16 x 4 stages (STF_GEMM_BK=16)", {"STF_GEMM_BK": "16"}),
 ]
 
