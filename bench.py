@@ -260,7 +260,7 @@ def run_ours(args, rank, world):
     tr = load_traffic()
     dom = {"name": "gemm_nt_dmma (GEMM/SYRK tile update C -= A B^T)",
            "flop_share": round(((T - 1) * (T - 2) + (T - 1)) / T ** 2, 4),
-           "launches_per_step": (T - 1) * T // 2,
+           "launches_per_step": T * (T - 1) * (T - 2) // 6 + T * (T - 1) // 2,
            "alone_tile": kern.get("gemm_tile"), "alone_full_occupancy": kern.get("gemm_full"),
            "traffic_bytes_per_tile_launch": tr, "algorithmic_bytes_per_tile_launch": 4 * nb * nb * 8}
     roof["dominant_kernel"] = dom

@@ -104,6 +104,8 @@ const char *stf_last_error(void);
  *   "serial"   STF_SERIAL   1: every task on one stream in program order (race check)
  *   "priority" STF_PRIO     1: critical-path tasks on high-priority streams (default 1)
  *   "grid_p"   STF_GRID     rows P of the P x Q grid for COLMAJOR kinds (0 = auto)
+ *   "threads"  STF_THREADS  eager backend: host submission threads, slots split round-robin
+ *                           (default 8, capped at ngpus; the graph backend captures on one thread)
  *   "lookahead" STF_LOOKAHEAD 1: pure STF DAG (default); 0: a fence task closes every
  *                           panel step (no look-ahead; ablation of PAPER.md:399)
  * Returns 0 or -105. */

@@ -11,6 +11,7 @@
 // computed pivot and a unit-diagonal dyadic input factors bit-exactly (pin P2).
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <climits>
 #include <cmath>
 
@@ -91,8 +92,8 @@ __global__ void __launch_bounds__(64) trsm_base_kernel(const double* __restrict_
     if (c < n) B[(int64_t)c * ldb + r] = x[c];
 }
 
-int64_t& launch_count() {
-  static thread_local int64_t c = 0;
+std::atomic<int64_t>& launch_count() {
+  static std::atomic<int64_t> c{0};
   return c;
 }
 

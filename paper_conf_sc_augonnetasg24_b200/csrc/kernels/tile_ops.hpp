@@ -6,6 +6,7 @@
 // `prio` is the CUDA stream-priority value recorded on the launch (and on the
 // graph node when captured); lower numbers are higher priority.
 #pragma once
+#include <atomic>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -62,9 +63,9 @@ cudaError_t transpose_copy(cudaStream_t stream, double* dst, int64_t ldd, const 
 // Fill a device int64 sentinel used by potrf_lower's info.
 cudaError_t info_reset(cudaStream_t stream, unsigned long long* info);
 
-// Number of kernels enqueued by the launchers above on this host thread
+// Number of kernels enqueued by the launchers above, all host threads
 // (monotonic; the runtime reports per-call deltas as gpu_launches).
-int64_t& launch_count();
+std::atomic<int64_t>& launch_count();
 
 // Device attributes / one-time function attribute setup (max dynamic smem).
 cudaError_t kernels_init(int device);

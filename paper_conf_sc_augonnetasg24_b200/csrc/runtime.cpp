@@ -29,6 +29,8 @@
 #include <memory>
 #include <mutex>
 #include <string>
+#include <thread>
+#include <atomic>
 #include <vector>
 
 #include "../../include/stf_cholesky.h"
@@ -82,6 +84,7 @@ struct Options {
   int64_t priority = 1;
   int64_t grid_p = 0;
   int64_t lookahead = 1;
+  int64_t threads = 8;  // eager backend: host submission threads (one per slot group)
 };
 
 // A plan bound to physical buffers, plus its lowering artefacts.
@@ -295,20 +298,63 @@ struct Lowerer {
       CUDA_TRY(cudaEventRecord(ev, S.streams[0]), "record info event");
       for (size_t k = 1; k < S.streams.size(); ++k) CUDA_TRY(cudaStreamWaitEvent(S.streams[k], ev, 0), "wait info event");
     }
+    const int nt = (X.opt.graph || X.opt.threads <= 1) ? 1 : (int)std::min<int64_t>(X.opt.threads, X.ngpus);
+    int r = 0;
+    if (nt == 1) {
+      r = issue_range(0, 1, nullptr);
+    } else {
+      // Multi-threaded eager submission (A26): thread w issues the
+      // tasks of slots s with s % nt == w, in program order.  A cross-thread
+      // predecessor's event may be waited on only after its record was issued,
+      // so each thread spins on the producer's `recorded` flag first; a thread
+      // only ever waits on tasks earlier in program order, so this cannot deadlock.
+      std::unique_ptr<std::atomic<uint8_t>[]> recorded(new std::atomic<uint8_t>[P.tasks.size()]);
+      for (size_t t = 0; t < P.tasks.size(); ++t) recorded[t].store(0, std::memory_order_relaxed);
+      std::vector<int> rc((size_t)nt, 0);
+      std::vector<std::string> err((size_t)nt);
+      std::vector<std::thread> th;
+      for (int w = 0; w < nt; ++w)
+        th.emplace_back([&, w] {
+          Lowerer L{C, X};
+          rc[(size_t)w] = L.issue_range(w, nt, recorded.get());
+          if (rc[(size_t)w]) {
+            err[(size_t)w] = g_err;
+            for (size_t t = 0; t < P.tasks.size(); ++t) recorded[t].store(1, std::memory_order_release);  // unblock peers
+          }
+        });
+      for (auto& x : th) x.join();
+      for (int w = 0; w < nt && !r; ++w)
+        if (rc[(size_t)w]) {
+          r = rc[(size_t)w];
+          g_err = err[(size_t)w];
+        }
+    }
+    if (r) return r;
+    X.launches = stfk::launch_count() - launches0;
+    return 0;
+  }
+
+  // Issue the tasks of the slots owned by submission thread w of nt (all tasks
+  // when nt == 1) in program order.
+  int issue_range(int w, int nt, std::atomic<uint8_t>* recorded) {
+    const stf::Plan& P = X.plan;
     for (size_t t = 0; t < P.tasks.size(); ++t) {
       const stf::Task& task = P.tasks[t];
+      if (task.slot % nt != w) continue;
       set_dev(C.slots[(size_t)task.slot].device);
       cudaStream_t s = stream_of(task);
       for (const int64_t* q = P.graph.preds_begin((int64_t)t); q != P.graph.preds_end((int64_t)t); ++q) {
         const stf::Task& pt = P.tasks[(size_t)*q];
         if (pt.slot == task.slot && pt.stream == task.stream) continue;  // stream order suffices
+        if (recorded && pt.slot % nt != w)
+          while (!recorded[*q].load(std::memory_order_acquire)) std::this_thread::yield();
         CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
       }
       int r = body(task, t, s, prio_of(task));
       if (r) return r;
       if (X.events[t]) CUDA_TRY(cudaEventRecord(X.events[t], s), "event record");
+      if (recorded) recorded[t].store(1, std::memory_order_release);
     }
-    X.launches = stfk::launch_count() - launches0;
     return 0;
   }
 };
@@ -595,6 +641,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
+  C.opt.threads = env_int("STF_THREADS", 8);
   C.opt.priority = env_int("STF_PRIO", 1);
   C.opt.grid_p = 0;
   if (const char* gs = getenv("STF_GRID")) C.opt.grid_p = atoi(gs);
@@ -731,6 +778,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "streams") *value = C.opt.streams;
   else if (n == "serial") *value = C.opt.serial;
   else if (n == "lookahead") *value = C.opt.lookahead;
+  else if (n == "threads") *value = C.opt.threads;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;
   else return fail(-105, "unknown option '%s'", name);

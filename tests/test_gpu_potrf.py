@@ -54,7 +54,7 @@ def _reset_options(request):
     yield
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
-        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2)
+        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2, threads=8, lookahead=1)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
@@ -157,7 +157,7 @@ def _bits(stf, n, nb, p=1, q=1, seed=3, **opts):
     M, info = _factor_spd(stf, n, nb, p, q, seed)
     assert info == 0
     out = M.to_dense().numpy().copy()
-    _options(stf, graph=1, serial=0, priority=1, streams=8)
+    _options(stf, graph=1, serial=0, priority=1, streams=8, threads=8)
     return out
 
 
@@ -175,7 +175,18 @@ def test_bit_equal_across_virtual_grids(stf, p, q):
     n, nb = 2048, 256
     ref = _bits(stf, n, nb, 1, 1)
     assert np.array_equal(ref, _bits(stf, n, nb, p, q))
-    assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0))
+    assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0, threads=1))
+    assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0, threads=p * q))  # one submission thread per slot
+
+
+def test_no_lookahead_fence_ablation_same_bits(stf):
+    # the per-step fence only adds ordering: same kernels, same per-tile op order
+    n, nb = 2048, 256
+    ref = _bits(stf, n, nb)
+    _options(stf, lookahead=0)
+    got = _bits(stf, n, nb)
+    _options(stf, lookahead=1)
+    assert np.array_equal(ref, got)
 
 
 def test_repeated_calls_reuse_graph(stf):
