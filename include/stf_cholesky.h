@@ -127,6 +127,8 @@ typedef struct stf_plan_stats {
   double device_ms;       /* device time of the last call: CUDA events recorded on the
                              library's launch stream immediately before the graph launch
                              (eager: before the fork) and after the join */
+  int64_t graph_reuse;    /* 0 new plan, 1 exact memo hit, 2 plan of the same shape re-bound
+                             to new caller storage (graph refreshed by cudaGraphExecUpdate) */
 } stf_plan_stats;
 
 int stf_last_stats(stf_plan_stats *out);

@@ -42,6 +42,7 @@ class stf_plan_stats(ctypes.Structure):
         ("kernel_launches", ctypes.c_int64),
         ("build_ms", ctypes.c_double),
         ("device_ms", ctypes.c_double),
+        ("graph_reuse", ctypes.c_int64),
     ]
 
     def as_dict(self):

@@ -110,6 +110,8 @@ struct Exec {
   cudaGraphExec_t gexec = nullptr;
   int64_t graph_nodes = 0;
   int graph_fallback = 0;  // capture failed, eager lowering used
+  int64_t updates = 0;     // successful cudaGraphExecUpdate re-binds
+  bool rebound = false;
   int64_t launches = 0;
   double build_ms = 0;
   // caller matrix for COLMAJOR kinds
@@ -525,6 +527,54 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   return 0;
 }
 
+// Point an existing plan at new caller storage (same shape) and refresh its graph.
+int rebind(Context& C, Exec& X, const stf_matrix_desc* desc, const std::vector<uintptr_t>& ptrs) {
+  auto t0 = std::chrono::steady_clock::now();
+  const int64_t T = X.n / X.nb;
+  if (X.kind == STF_DESC_TILED_2DBC) {
+    for (size_t b = 0; b < (size_t)X.plan.ntiles(); ++b) {
+      const stf::Buffer& B = X.plan.buffers[b];
+      X.buf[b] = desc->tiles[(size_t)B.i + (size_t)B.j * (size_t)T];
+    }
+  } else {
+    X.mat = desc->ptr;
+    X.ld = desc->ld;
+    X.mat_dev = (X.kind == STF_DESC_DEVICE_COLMAJOR) ? desc->device : -1;
+  }
+  X.key_ptrs = ptrs;
+  X.key_ld = desc->ld;
+  X.key_dev = desc->device;
+  if (X.gexec) {
+    cudaSetDevice(C.origin_dev);
+    CUDA_TRY(cudaStreamBeginCapture(C.origin, cudaStreamCaptureModeThreadLocal), "begin capture");
+    int r = fork_streams(C, X.ngpus);
+    Lowerer L{C, X};
+    if (!r) r = L.issue();
+    if (!r) r = join_streams(C, X.ngpus);
+    cudaSetDevice(C.origin_dev);
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(C.origin, &g);
+    if (r || e != cudaSuccess) {
+      if (g) cudaGraphDestroy(g);
+      return r ? r : cuda_fail(e, "re-capture");
+    }
+    cudaGraphExecUpdateResultInfo ri;
+    if (cudaGraphExecUpdate(X.gexec, g, &ri) == cudaSuccess) {
+      X.updates++;
+    } else {
+      cudaGetLastError();
+      cudaGraphExecDestroy(X.gexec);
+      X.gexec = nullptr;
+      CUDA_TRY(cudaGraphInstantiateWithFlags(&X.gexec, g, cudaGraphInstantiateFlagUseNodePriority), "graph instantiate");
+    }
+    if (X.graph) cudaGraphDestroy(X.graph);
+    X.graph = g;
+  }
+  X.build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  X.rebound = true;
+  return 0;
+}
+
 int run(Context& C, Exec& X) {
   cudaSetDevice(C.origin_dev);
   CUDA_TRY(cudaEventRecord(C.t_start, C.origin), "timing start");
@@ -567,6 +617,7 @@ void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
   s->graph_nodes = X.graph_nodes;
   s->kernel_launches = X.launches;
   s->build_ms = hit ? 0.0 : X.build_ms;
+  s->graph_reuse = hit ? 1 : 0;
 }
 
 int choose_grid(int ngpus, int64_t grid_p, int* P, int* Q) {
@@ -856,6 +907,29 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
       break;
     }
   }
+  int reuse = hit ? 1 : 0;
+  if (!X) {
+    // NEXT-2: a plan of the same shape bound to other caller
+    // pointers is re-bound: same plan, workspaces and events; the graph is
+    // re-captured and applied to the existing executable graph with
+    // cudaGraphExecUpdate (falls back to a fresh instantiation if rejected).
+    for (auto it = C.cache.begin(); it != C.cache.end(); ++it) {
+      Exec& e = **it;
+      const bool pageable = A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr);
+      if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
+          e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial && e.key_graph == C.opt.graph &&
+          e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm &&
+          e.opt.lookahead == C.opt.lookahead && (e.gexec == nullptr) == (e.opt.graph == 0) &&
+          !(pageable && e.gexec)) {
+        int r = rebind(C, e, A_desc, ptrs);
+        if (r) return r;
+        C.cache.splice(C.cache.begin(), C.cache, it);
+        X = C.cache.front().get();
+        reuse = 2;
+        break;
+      }
+    }
+  }
   if (!X) {
     while (C.cache.size() >= kCacheMax) C.cache.pop_back();
     std::unique_ptr<Exec> e(new Exec());
@@ -889,6 +963,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
   int info = run(C, *X);
   fill_stats(*X, hit, &C.last);
   C.last.device_ms = C.device_ms;
+  C.last.graph_reuse = reuse;
   if (info < 0) {
     // a failed call leaves device state unknown: drop the plan
     C.cache.remove_if([&](const std::unique_ptr<Exec>& p) { return p.get() == X; });
@@ -942,6 +1017,7 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
     stats->kernel_launches = 0;
     stats->build_ms = ms;
     stats->device_ms = 0;
+    stats->graph_reuse = 0;
   }
   return 0;
 }

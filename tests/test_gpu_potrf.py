@@ -189,6 +189,28 @@ def test_no_lookahead_fence_ablation_same_bits(stf):
     assert np.array_equal(ref, got)
 
 
+def test_same_shape_new_tiles_rebinds_graph(stf):
+    """NEXT-2: a second matrix of the same shape re-uses the plan; the graph is
+    re-captured and applied with cudaGraphExecUpdate; results stay exact."""
+    A, L0 = synth.dyadic_spd(101, 1024)
+    import torch
+
+    M1 = stf.TiledMatrix(1024, 256)
+    M1.fill_spd(3)
+    assert M1.potrf() == 0
+    assert stf.last_stats()["graph_reuse"] == 0
+    M2 = stf.TiledMatrix(1024, 256)
+    M2.load_dense(torch.from_numpy(np.ascontiguousarray(A)))
+    assert M2.potrf() == 0
+    st = stf.last_stats()
+    assert st["graph_reuse"] == 2
+    assert np.array_equal(M2.to_dense().numpy(), L0)
+    M2.load_dense(torch.from_numpy(np.ascontiguousarray(A)))
+    assert M2.potrf() == 0
+    assert stf.last_stats()["graph_reuse"] == 1
+    assert np.array_equal(M2.to_dense().numpy(), L0)
+
+
 def test_repeated_calls_reuse_graph(stf):
     M = stf.TiledMatrix(1024, 256)
     M.fill_spd(2)
