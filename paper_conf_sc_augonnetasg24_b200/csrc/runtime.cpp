@@ -809,6 +809,11 @@ int stf_set_option(const char* name, int64_t value) {
     if (value > have) return fail(-105, "streams=%lld exceeds the pool created at init (%d)", (long long)value, have);
     C.opt.streams = value;
   } else if (n == "serial") C.opt.serial = value != 0;
+  else if (n == "lookahead") C.opt.lookahead = value != 0;
+  else if (n == "threads") {
+    if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
+    C.opt.threads = value;
+  }
   else if (n == "priority") C.opt.priority = value != 0;
   else if (n == "grid_p") {
     if (value < 0) return fail(-105, "grid_p must be >= 0");

@@ -83,9 +83,18 @@ def test_init_without_gpu_fails_cleanly():
     assert b"CUDA" in _abi.stf_last_error() or b"device" in _abi.stf_last_error()
 
 
+OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (2, 1), "streams": (8, 3), "serial": (0, 1),
+           "priority": (1, 0), "grid_p": (0, 2), "lookahead": (1, 0), "threads": (8, 2)}
+
+
 def test_options_roundtrip_without_gpu():
-    stf.set_option("serial", 1)
-    assert stf.get_option("serial") == 1
-    stf.set_option("serial", 0)
+    # every option the header documents can be set and read back
+    hdr = open(HEADER).read()
+    for name, (dflt, other) in OPTIONS.items():
+        assert '"%s"' % name in hdr, name
+        stf.set_option(name, other)
+        assert stf.get_option(name) == other
+        stf.set_option(name, dflt)
+        assert stf.get_option(name) == dflt
     with pytest.raises(stf.StfError):
         stf.set_option("nonsense", 1)
