@@ -78,6 +78,7 @@ struct Slot {
 struct Options {
   int64_t dataflow = 1;  // POTRF tile kernel: 1 single-launch dataflow, 0 recursive (GEMM-based)
   int64_t trsm = 2;      // TRSM tile kernel: 2 row-panel, 1 dataflow, 0 recursive
+  int64_t trsm_split = 1;  // row panel: non-critical TRSMs as panel(nb/2) + GEMM + panel(nb/2)
   int64_t graph = 1;
   int64_t streams = 8;
   int64_t serial = 0;
@@ -211,11 +212,23 @@ struct Lowerer {
                    "POTRF launch");
         return 0;
       case stf::K_TRSM:
-        if (X.opt.trsm == 2)  // the next panel's TRSM(k+1,k) is on the critical path: low-latency variant
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb,
-                                    t.i == t.k + 1 ? 32 : 0),
+        if (X.opt.trsm == 2 && t.i == t.k + 1) {
+          // the next panel's TRSM(k+1,k) is on the critical path: one low-latency launch
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 32),
                    "TRSM launch");
-        else if (X.opt.trsm == 1)
+        } else if (X.opt.trsm == 2 && X.opt.trsm_split && nb >= 512 && (nb / 2) % 64 == 0) {
+          // X = [X1 X2]: X1 = B1 L11^-T; B2 -= X1 L21^T (full-rate GEMM kernel); X2 = B2 L22^-T.
+          // Half of the TRSM flops run on the GEMM kernel (SM-time, not latency, matters here).
+          const int64_t h = nb / 2;
+          const double* L = X.buf[(size_t)t.in[0]];
+          double* B = X.buf[(size_t)t.out];
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L, nb, B, nb, 0), "TRSM launch");
+          CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)h, (int)h, B, nb, L + h, nb, B + h * nb, nb, 0), "TRSM GEMM");
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L + h * nb + h, nb, B + h * nb, nb, 0), "TRSM launch");
+        } else if (X.opt.trsm == 2) {
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 0),
+                   "TRSM launch");
+        } else if (X.opt.trsm == 1)
           CUDA_TRY(stfk::trsm_tile(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, ws),
                    "TRSM launch");
         else
@@ -689,6 +702,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.graph = env_int("STF_GRAPH", 1);
   C.opt.dataflow = env_int("STF_DATAFLOW", 1);
   C.opt.trsm = env_int("STF_TRSM", 2);
+  C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 1);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
@@ -810,6 +824,7 @@ int stf_set_option(const char* name, int64_t value) {
     C.opt.streams = value;
   } else if (n == "serial") C.opt.serial = value != 0;
   else if (n == "lookahead") C.opt.lookahead = value != 0;
+  else if (n == "trsm_split") C.opt.trsm_split = value != 0;
   else if (n == "threads") {
     if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
     C.opt.threads = value;
@@ -834,6 +849,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "streams") *value = C.opt.streams;
   else if (n == "serial") *value = C.opt.serial;
   else if (n == "lookahead") *value = C.opt.lookahead;
+  else if (n == "trsm_split") *value = C.opt.trsm_split;
   else if (n == "threads") *value = C.opt.threads;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;
@@ -903,7 +919,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
         e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
         e.key_graph == C.opt.graph &&
-        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.opt.lookahead == C.opt.lookahead && e.key_ptrs == ptrs &&
+        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.opt.trsm_split == C.opt.trsm_split && e.opt.lookahead == C.opt.lookahead && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
       C.cache.splice(C.cache.begin(), C.cache, it);
@@ -924,7 +940,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
       if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
           e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial && e.key_graph == C.opt.graph &&
           e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm &&
-          e.opt.lookahead == C.opt.lookahead && (e.gexec == nullptr) == (e.opt.graph == 0) &&
+          e.opt.trsm_split == C.opt.trsm_split && e.opt.lookahead == C.opt.lookahead && (e.gexec == nullptr) == (e.opt.graph == 0) &&
           !(pageable && e.gexec)) {
         int r = rebind(C, e, A_desc, ptrs);
         if (r) return r;
