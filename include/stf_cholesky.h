@@ -179,6 +179,15 @@ int stf_kernel_potrf(int64_t n, double *A, int64_t lda, int64_t *info);
  * Returns 0 / -4 / -101 / -103.  Not part of the factorisation. */
 int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double *avg_ms);
 
+/* Debug timeline of the dataflow POTRF tile kernel (one launch on the current
+ * device, A: n x n column-major device matrix, ctas <= 0: default grid).
+ * trace[0 .. 6T) holds %globaltimer stamps (ns) of the critical-path CTA per
+ * 64-block step kb (P start, P published, S inputs ready, S published, U inputs
+ * ready, U done), T = ceil(n/64); trace[6T + 3t ..] the claim / inputs-ready /
+ * done stamps of bulk ticket t (0 if unused).  Returns the number of entries
+ * written (<= cap) or a negative error.  Not part of the factorisation. */
+int64_t stf_debug_potrf_trace(int64_t n, double *A, int64_t lda, int ctas, int64_t *trace, int64_t cap);
+
 #ifdef __cplusplus
 }
 #endif

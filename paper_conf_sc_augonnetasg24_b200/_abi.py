@@ -54,7 +54,7 @@ EXPORTS = [
     "stf_cholesky_init", "stf_potrf", "stf_finalize", "stf_last_error",
     "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_infer_edges",
     "stf_fill_spd_tiles", "stf_fill_spd_block",
-    "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel",
+    "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace",
 ]
 
 if not os.path.exists(LIB_PATH):
@@ -91,6 +91,7 @@ stf_kernel_gemm_nt = _decl("stf_kernel_gemm_nt", _int, [_i64, _i64, _i64, _vp, _
 stf_kernel_trsm = _decl("stf_kernel_trsm", _int, [_i64, _i64, _vp, _i64, _vp, _i64])
 stf_kernel_potrf = _decl("stf_kernel_potrf", _int, [_i64, _vp, _i64, _P(_i64)])
 stf_bench_kernel = _decl("stf_bench_kernel", _int, [_int, _i64, _i64, _i64, _int, _P(_dbl)])
+stf_debug_potrf_trace = _decl("stf_debug_potrf_trace", _i64, [_i64, _vp, _i64, _int, _P(_i64), _i64])
 
 
 class StfError(RuntimeError):

@@ -67,7 +67,18 @@ struct DfParams {
   unsigned long long* info;
   int potrf;
   int crit;  // POTRF: one CTA runs the critical chain P -> S -> U -> P (blocks kept in smem)
+  unsigned long long* trace;  // debug: %globaltimer stamps (null in production)
 };
+
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define DF_STAMP(idx)                                          \
+  do {                                                         \
+    if (p.trace && threadIdx.x == 0) p.trace[(idx)] = gtime(); \
+  } while (0)
 
 __device__ __forceinline__ int ld_acquire(const int* p) {
   int v;
@@ -317,6 +328,7 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
     const int nk = min(W, p.n - kb * W);
     double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
     // ---- P(kb)
+    DF_STAMP(6 * kb + 0);
     chol_core(a, D, Y, nk, p.col0 + (int64_t)kb * W, p.info);
     store_chunk(a, Xkk, p.ldx, nk, nk, true);
     __syncthreads();
@@ -324,12 +336,14 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       __threadfence();
       st_release(&prog[kb * p.Nb + kb], kb + 1);
     }
+    DF_STAMP(6 * kb + 1);
     if (kb + 1 == T) return;
     // ---- S(ib, kb), ib = kb + 1, with L_kk from D
     const int ib = kb + 1, rows = min(W, p.n - ib * W);
     double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
     if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + kb], kb);
     __syncthreads();
+    DF_STAMP(6 * kb + 2);
     double b[16];
     load_chunk(b, Xik, p.ldx, rows, nk, false);
     solve_core(b, D, Rc, XS, df::LDO, nk);
@@ -339,9 +353,11 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       __threadfence();
       st_release(&prog[ib * p.Nb + kb], kb + 1);
     }
+    DF_STAMP(6 * kb + 3);
     // ---- U(ib, ib, kb): D <- lower(C - X X^T), C = block (ib, ib) after all earlier updates
     if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + ib], kb);
     __syncthreads();
+    DF_STAMP(6 * kb + 4);
     double* Cii = p.X + (int64_t)ib * W * p.ldx + ib * W;
     double acc[4][2][2];
 #pragma unroll
@@ -385,6 +401,7 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       a[c] = (r < rows && col < rows && r >= col) ? D[r * df::LDB + col] : 0.0;
     }
     __syncthreads();  // D is rewritten by the next chol_core
+    DF_STAMP(6 * kb + 5);
   }
 }
 
@@ -408,6 +425,7 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
     __syncthreads();
     const int ticket = s_task;
     if (ticket >= p.ntasks) return;
+    DF_STAMP(6 * p.Nb + 3 * ticket + 0);
     const uint32_t code = p.tasks[ticket];
     const uint32_t type = code >> 30;
     const int ib = (code >> 20) & 1023, jb = (code >> 10) & 1023, kb = code & 1023;
@@ -434,6 +452,7 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
       }
     }
     __syncthreads();
+    DF_STAMP(6 * p.Nb + 3 * ticket + 1);
     if (p.potrf) {
       double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
       const int nk = min(W, p.n - kb * W);
@@ -463,6 +482,7 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
       const int tgt = p.potrf ? (type == df::T_U ? ib * p.Nb + jb : ib * p.Nb + kb) : (ib * p.Nb + jb);
       st_release(&prog[tgt], kb + 1);
     }
+    DF_STAMP(6 * p.Nb + 3 * ticket + 2);
   }
 }
 
@@ -612,7 +632,7 @@ cudaError_t dataflow_init_attrs() {
 }
 
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
-                       unsigned long long* info, int* ws) {
+                       unsigned long long* info, int* ws, unsigned long long* trace, int ctas_override) {
   if (n <= 0) return cudaSuccess;
   DfParams p{};
   p.X = A;
@@ -630,8 +650,9 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   p.potrf = 1;
   const int T = p.Nb;
   const int par = T * (T - 1) / 2 > 0 ? T * (T - 1) / 2 : 1;  // widest update wave
-  int ctas = std::min(par, std::min(df_max_ctas(), num_sms()));
+  int ctas = std::min(par, std::min(ctas_override > 0 ? ctas_override : df_max_ctas(), num_sms()));
   if (p.crit) ctas = std::min(p.ntasks, ctas - 1) + 1;  // + the critical-chain CTA
+  p.trace = trace;
   return launch_df(stream, prio, p, ctas);
 }
 
@@ -654,6 +675,7 @@ cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double*
   p.info = nullptr;
   p.potrf = 0;
   p.crit = 0;
+  p.trace = nullptr;
   const int par = p.Mb * (p.Nb > 1 ? p.Nb - 1 : 1);
   return launch_df(stream, prio, p, std::min(par, std::min(4 * df_max_ctas(), num_sms())));
 }

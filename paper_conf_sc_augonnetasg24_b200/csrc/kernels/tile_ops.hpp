@@ -39,7 +39,7 @@ cudaError_t potrf_lower(cudaStream_t stream, int prio, int n, double* A, int64_t
 // dataflow_prepare() uploads the task table for the shape; it must be called
 // once before the first launch of that shape inside a stream capture.
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
-                       unsigned long long* info, int* ws);
+                       unsigned long long* info, int* ws, unsigned long long* trace = nullptr, int ctas = 0);
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                       int64_t ldb, int* ws);
 size_t dataflow_ws_bytes(int m, int n);

@@ -1234,4 +1234,31 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
   return 0;
 }
 
+int64_t stf_debug_potrf_trace(int64_t n, double* A, int64_t lda, int ctas, int64_t* trace, int64_t cap) {
+  g_err.clear();
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int r = ensure_kernel_attrs(dev);
+  if (r) return r;
+  const int Nb = (int)((n + 63) / 64);
+  const int64_t slots = 6 * Nb + 3 * (int64_t)Nb * Nb * Nb;  // >= 6 T + 3 * tasks
+  unsigned long long *d_info = nullptr, *d_tr = nullptr;
+  int* ws = nullptr;
+  cudaError_t e = cudaMalloc(&d_info, sizeof *d_info);
+  if (e == cudaSuccess) e = cudaMalloc(&d_tr, (size_t)slots * 8);
+  if (e == cudaSuccess) e = cudaMemset(d_tr, 0, (size_t)slots * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)n, (int)n));
+  if (e == cudaSuccess) e = stfk::dataflow_prepare((int)n, (int)n, true);
+  if (e == cudaSuccess) e = stfk::info_reset(0, d_info);
+  if (e == cudaSuccess) e = stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws, d_tr, ctas);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(0);
+  const int64_t cnt = std::min<int64_t>(cap, slots);
+  if (e == cudaSuccess && trace) e = cudaMemcpy(trace, d_tr, (size_t)cnt * 8, cudaMemcpyDeviceToHost);
+  cudaFree(d_info);
+  cudaFree(d_tr);
+  cudaFree(ws);
+  if (e != cudaSuccess) return cuda_fail(e, "potrf trace");
+  return cnt;
+}
+
 }  // extern "C"

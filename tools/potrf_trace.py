@@ -1,0 +1,46 @@
+"""Timeline of the dataflow POTRF tile kernel (stf_debug_potrf_trace): critical
+chain phases per 64-block step and bulk task occupancy.  usage: potrf_trace.py n ctas"""
+import ctypes
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+from paper_conf_sc_augonnetasg24_b200 import _abi  # noqa: E402
+
+n = int(sys.argv[1]) if len(sys.argv) > 1 else 1024
+ctas = int(sys.argv[2]) if len(sys.argv) > 2 else 0
+T = (n + 63) // 64
+A = torch.zeros((n, n), dtype=torch.float64, device="cuda")
+_abi.stf_fill_spd_block(A.data_ptr(), n, n, 0, 0, n, n, 1)
+cap = 6 * T + 3 * T ** 3
+tr = (ctypes.c_int64 * cap)()
+for rep in range(3):  # warm-up then the measured one
+    _abi.stf_fill_spd_block(A.data_ptr(), n, n, 0, 0, n, n, 1)
+    cnt = _abi.stf_debug_potrf_trace(n, A.data_ptr(), n, ctas, tr, cap)
+t = np.array(tr[:cnt], dtype=np.int64)
+chain = t[:6 * T].reshape(T, 6)
+bulk = t[6 * T:].reshape(-1, 3)
+bulk = bulk[bulk[:, 0] > 0]
+t0 = min(chain[0, 0], bulk[:, 0].min() if len(bulk) else chain[0, 0])
+print("n=%d ctas=%d total %.1f us, bulk tasks %d" % (n, ctas, (max(chain.max(), bulk.max() if len(bulk) else 0) - t0) / 1e3, len(bulk)))
+print("step  P_us  S_wait_us  S_us  U_wait_us  U_us  (chain, from P start)")
+for kb in range(T):
+    c = chain[kb] - t0
+    if c[1] <= 0:
+        continue
+    pu = (chain[kb, 1] - chain[kb, 0]) / 1e3
+    if kb + 1 < T:
+        print("%3d %6.1f %9.1f %6.1f %9.1f %6.1f" % (kb, pu, (chain[kb, 2] - chain[kb, 1]) / 1e3,
+              (chain[kb, 3] - chain[kb, 2]) / 1e3, (chain[kb, 4] - chain[kb, 3]) / 1e3,
+              (chain[kb, 5] - chain[kb, 4]) / 1e3))
+    else:
+        print("%3d %6.1f" % (kb, pu))
+if len(bulk):
+    w = (bulk[:, 1] - bulk[:, 0]) / 1e3
+    d = (bulk[:, 2] - bulk[:, 1]) / 1e3
+    print("bulk: wait mean %.1f us (max %.1f), run mean %.1f us (max %.1f), busy sum %.1f us" % (
+        w.mean(), w.max(), d.mean(), d.max(), d.sum()))
