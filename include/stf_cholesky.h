@@ -106,6 +106,8 @@ const char *stf_last_error(void);
  *   "serial"   STF_SERIAL   1: every task on one stream in program order (race check)
  *   "priority" STF_PRIO     1: critical-path tasks on high-priority streams (default 1)
  *   "grid_p"   STF_GRID     rows P of the P x Q grid for COLMAJOR kinds (0 = auto)
+ *   "push"     STF_PUSH     1: TRSM(i,k) writes L_ik into its consumers' replicas from its own
+ *                           epilogue (fused push over NVLink, NEXT-3); 0: COPY tasks (default)
  *   "threads"  STF_THREADS  eager backend: host submission threads, slots split round-robin
  *                           (default 8, capped at ngpus; the graph backend captures on one thread)
  *   "lookahead" STF_LOOKAHEAD 1: pure STF DAG (default); 0: a fence task closes every
@@ -119,7 +121,7 @@ int stf_get_option(const char *name, int64_t *value);
  * see stf_dag_build).  Integer host work, compared bit-exactly with the oracle. */
 typedef struct stf_plan_stats {
   int64_t tasks;          /* compute tasks (POTRF + TRSM + SYRK + GEMM) */
-  int64_t transfers;      /* inter-slot tile copies (replica updates) */
+  int64_t transfers;      /* inter-slot tile transfers (COPY tasks + fused pushes) */
   int64_t edges;          /* DAG edges between all tasks (compute + transfer) */
   int64_t transfer_bytes; /* bytes moved between slots */
   int64_t critical_path;  /* longest chain of compute tasks (3T-2 when P=Q=1) */
@@ -131,6 +133,7 @@ typedef struct stf_plan_stats {
                              (eager: before the fork) and after the join */
   int64_t graph_reuse;    /* 0 new plan, 1 exact memo hit, 2 plan of the same shape re-bound
                              to new caller storage (graph refreshed by cudaGraphExecUpdate) */
+  int64_t dag_tasks;      /* all DAG vertices: compute + COPY + LOAD/STORE + FENCE tasks */
 } stf_plan_stats;
 
 int stf_last_stats(stf_plan_stats *out);
@@ -140,7 +143,8 @@ int stf_last_stats(stf_plan_stats *out);
  * order) into edges[2*cap].  kinds[cap_tasks] receives per-task codes
  * (0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM, 4 COPY, 7 FENCE) and ijk[3*cap_tasks] the (i, j, k)
  * indices (for COPY: tile i, j and destination slot k).  Any output pointer
- * may be NULL.  Fills *stats.  Needs no GPU. */
+ * may be NULL.  Fills *stats.  Uses the current "push" and "lookahead" options.
+ * Needs no GPU. */
 int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t *edges, int64_t cap_tasks, int32_t *kinds,
                   int64_t *ijk, stf_plan_stats *stats);
 

@@ -57,7 +57,7 @@ def dag(T: int, p: int = 1, q: int = 1):
     """(edges, kinds, ijk, stats) of the plan DAG, built on the host only."""
     st = stf_plan_stats()
     check(_abi.stf_dag_build(T, p, q, 0, None, 0, None, None, ctypes.byref(st)), "stf_dag_build")
-    ntasks = st.tasks + st.transfers
+    ntasks = st.dag_tasks
     E = (ctypes.c_int64 * (2 * max(1, st.edges)))()
     K = (ctypes.c_int32 * max(1, ntasks))()
     IJK = (ctypes.c_int64 * (3 * max(1, ntasks)))()

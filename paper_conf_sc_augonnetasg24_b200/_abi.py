@@ -43,6 +43,7 @@ class stf_plan_stats(ctypes.Structure):
         ("build_ms", ctypes.c_double),
         ("device_ms", ctypes.c_double),
         ("graph_reuse", ctypes.c_int64),
+        ("dag_tasks", ctypes.c_int64),
     ]
 
     def as_dict(self):

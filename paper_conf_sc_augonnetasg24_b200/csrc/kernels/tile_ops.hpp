@@ -47,8 +47,14 @@ size_t dataflow_ws_bytes(int m, int n);
 // K3 row-panel form (trsm_panel.cu): one launch, ceil(M/R) CTAs each owning R
 // rows (R = 32: lower latency, 64: higher efficiency; 0 = STF_TRSM_ROWS, default
 // 64), left-looking over 64-wide column blocks (DMMA update + substitution).
+// Replica destinations written by a kernel's epilogue together with the home
+// tile (same offsets and leading dimension): fused push of a finished tile.
+struct Mirrors {
+  double* p[7];
+  int n;
+};
 cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
-                       int64_t ldb, int rows_per_cta = 0);
+                       int64_t ldb, int rows_per_cta = 0, const Mirrors* mirrors = nullptr);
 cudaError_t dataflow_prepare(int m, int n, bool potrf);
 
 // K8: fill rows r0.., cols c0.. (global indices) of the seeded SPD metric matrix

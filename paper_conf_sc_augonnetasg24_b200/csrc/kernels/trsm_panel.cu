@@ -71,7 +71,8 @@ __device__ __forceinline__ void stage_block(double* dst, int ld, const double* G
 
 template <int BMT>
 __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __restrict__ L, int64_t ldl, int n,
-                                                             double* __restrict__ X, int64_t ldx, int M) {
+                                                             double* __restrict__ X, int64_t ldx, int M,
+                                                             const Mirrors mir) {
   using tp = TP<BMT>;
   extern __shared__ __align__(16) double smt[];
   const int r0 = blockIdx.x * tp::BM;
@@ -218,7 +219,15 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
 #pragma unroll
       for (int c = 0; c < 16; ++c) {
         const int col = 16 * q + c;
-        if (col < nc) Xr[(int64_t)(c0 + col) * ldx + r] = b[c];
+        if (col < nc) {
+          const int64_t off = (int64_t)(c0 + col) * ldx + r0 + r;
+          X[off] = b[c];
+          // fused push (NEXT-3): the finished value also goes straight into the
+          // consumers' replicas (peer memory over NVLink / another slot's arena)
+#pragma unroll
+          for (int m = 0; m < 7; ++m)
+            if (m < mir.n) mir.p[m][off] = b[c];
+        }
       }
     }
     __threadfence();  // X[rows, jb] is re-read (cp.async.cg, L2) by the next jb iterations
@@ -244,7 +253,9 @@ static int trsm_rows() {
 }
 
 cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
-                       int64_t ldb, int rows_per_cta) {
+                       int64_t ldb, int rows_per_cta, const Mirrors* mirrors) {
+  Mirrors mir{};
+  if (mirrors) mir = *mirrors;
   if (M <= 0 || n <= 0) return cudaSuccess;
   const int bm = rows_per_cta == 32 || rows_per_cta == 64 ? rows_per_cta : trsm_rows();
   cudaLaunchConfig_t cfg = {};
@@ -258,8 +269,8 @@ cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   ++launch_count();
-  if (bm == 32) return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<32>, L, ldl, n, B, ldb, M);
-  return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<64>, L, ldl, n, B, ldb, M);
+  if (bm == 32) return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<32>, L, ldl, n, B, ldb, M, mir);
+  return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<64>, L, ldl, n, B, ldb, M, mir);
 }
 
 }  // namespace stfk

@@ -2,6 +2,7 @@
 #include "plan.hpp"
 
 #include <algorithm>
+#include <vector>
 
 namespace stf {
 
@@ -67,6 +68,31 @@ struct Builder {
     return rep_buffer[r];
   }
 
+  // slots (other than the owner) whose tasks read the final L_ik: SYRK(i,k) on
+  // owner(i,i), GEMM(i,j,k) on owner(i,j) (k<j<i), GEMM(r,i,k) on owner(r,i) (r>i)
+  std::vector<int> consumers_of_panel_tile(int64_t i, int64_t k) const {
+    std::vector<int> s;
+    auto add = [&](int g) {
+      if (g != p.owner(i, k) && std::find(s.begin(), s.end(), g) == s.end()) s.push_back(g);
+    };
+    add(p.owner(i, i));
+    for (int64_t j = k + 1; j < i; ++j) add(p.owner(i, j));
+    for (int64_t r = i + 1; r < T; ++r) add(p.owner(r, i));
+    std::sort(s.begin(), s.end());
+    return s;
+  }
+
+  int64_t replica_buffer(int64_t i, int64_t j, int slot) {
+    const int64_t d = Plan::tile_id(i, j);
+    const size_t r = (size_t)(d * G + slot);
+    if (rep_buffer[r] < 0) {
+      rep_buffer[r] = (int64_t)p.buffers.size();
+      p.buffers.push_back(Buffer{(int32_t)i, (int32_t)j, slot, true});
+      p.replicas_per_slot[(size_t)slot]++;
+    }
+    return rep_buffer[r];
+  }
+
   void compute(int32_t kind, int64_t i, int64_t j, int64_t k, int prio, int64_t ra, int64_t rb, int64_t wi,
                int64_t wj) {
     const int slot = p.owner(wi, wj);
@@ -75,13 +101,24 @@ struct Builder {
     int64_t in1 = rb >= 0 ? read_buffer(rb / T, rb % T, slot) : -1;
     Task t{kind, (int32_t)i, (int32_t)j, (int32_t)k, slot, prio, 0, {in0, in1}, w};
     t.stream = compute_stream(t);
-    Access acc[3];
+    Access acc[3 + 7];
     int n = 0;
     if (in0 >= 0) acc[n++] = {in0, READ};
     if (in1 >= 0) acc[n++] = {in1, READ};
     acc[n++] = {w, RW};
+    std::vector<int> cons;
+    if (kind == K_TRSM && p.opt.push) cons = consumers_of_panel_tile(wi, wj);
+    for (int g : cons) {
+      const int64_t rb2 = replica_buffer(wi, wj, g);
+      t.mir[t.nmir++] = rb2;
+      acc[n++] = {rb2, WRITE};
+    }
     submit(t, acc, n);
     version[(size_t)w]++;
+    for (int g : cons) {  // the pushed replicas hold the new version: no COPY at their reads
+      rep_version[(size_t)(w * G + g)] = version[(size_t)w];
+      p.npushed++;
+    }
   }
 
   void run() {
@@ -146,6 +183,7 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
   if (plan.opt.copy_streams < 1) plan.opt.copy_streams = 1;
   plan.tasks.clear();
   plan.ntransfers = 0;
+  plan.npushed = 0;
   plan.replicas_per_slot.assign((size_t)opt.nslots, 0);
   // dense datum ids: home tiles + at most one replica per (tile, slot)
   const int64_t NT = T * (T + 1) / 2;

@@ -37,6 +37,8 @@ struct Task {
   int32_t stream;    // index into the slot's stream pool (see Lowering in runtime.cpp)
   int64_t in[2];     // buffer ids read (-1 if unused)
   int64_t out;       // buffer id written
+  int32_t nmir;      // fused push (NEXT-3): replica buffers written by the same kernel
+  int64_t mir[7];
 };
 
 struct PlanOptions {
@@ -51,6 +53,8 @@ struct PlanOptions {
   bool with_store = false; // STORE tasks (write-back) at the end of program order
   bool lookahead = true;   // false: a FENCE task (RW on every tile) closes each panel step, so
                            // step k+1 starts only when step k is complete (ablation, NEXT-1)
+  bool push = false;       // TRSM(i,k) writes L_ik into its consumers' replicas itself (fused
+                           // push, NEXT-3) instead of COPY tasks at the first remote read
 };
 
 // A "buffer" is one physical nb x nb tile instance: home tiles are buffers
@@ -66,7 +70,8 @@ struct Plan {
   std::vector<Task> tasks;
   std::vector<Buffer> buffers;
   TaskGraph graph;
-  int64_t ntransfers = 0;
+  int64_t ntransfers = 0;     // COPY tasks
+  int64_t npushed = 0;        // replicas written by fused push
   int64_t critical_path = 0;  // longest chain counted in compute tasks
   std::vector<int64_t> replicas_per_slot;
 

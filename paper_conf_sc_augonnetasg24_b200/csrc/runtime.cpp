@@ -86,6 +86,7 @@ struct Options {
   int64_t grid_p = 0;
   int64_t lookahead = 1;
   int64_t threads = 8;  // eager backend: host submission threads (one per slot group)
+  int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
 };
 
 // A plan bound to physical buffers, plus its lowering artefacts.
@@ -172,6 +173,7 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.with_load = load;
   po.with_store = store;
   po.lookahead = o.lookahead != 0;
+  po.push = o.push != 0 && o.trsm == 2;
   return po;
 }
 
@@ -211,10 +213,17 @@ struct Lowerer {
           CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
                    "POTRF launch");
         return 0;
-      case stf::K_TRSM:
+      case stf::K_TRSM: {
+        stfk::Mirrors mir{}, mir2{};
+        for (int m = 0; m < t.nmir && m < 7; ++m) {
+          mir.p[m] = X.buf[(size_t)t.mir[m]];
+          mir2.p[m] = mir.p[m] + (nb / 2) * nb;  // second column half (split variant)
+        }
+        mir.n = mir2.n = t.nmir < 7 ? t.nmir : 7;
         if (X.opt.trsm == 2 && t.i == t.k + 1) {
           // the next panel's TRSM(k+1,k) is on the critical path: one low-latency launch
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 32),
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 32,
+                                    &mir),
                    "TRSM launch");
         } else if (X.opt.trsm == 2 && X.opt.trsm_split && nb >= 512 && (nb / 2) % 64 == 0) {
           // X = [X1 X2]: X1 = B1 L11^-T; B2 -= X1 L21^T (full-rate GEMM kernel); X2 = B2 L22^-T.
@@ -222,11 +231,13 @@ struct Lowerer {
           const int64_t h = nb / 2;
           const double* L = X.buf[(size_t)t.in[0]];
           double* B = X.buf[(size_t)t.out];
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L, nb, B, nb, 0), "TRSM launch");
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L, nb, B, nb, 0, &mir), "TRSM launch");
           CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)h, (int)h, B, nb, L + h, nb, B + h * nb, nb, 0), "TRSM GEMM");
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L + h * nb + h, nb, B + h * nb, nb, 0), "TRSM launch");
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L + h * nb + h, nb, B + h * nb, nb, 0, &mir2),
+                   "TRSM launch");
         } else if (X.opt.trsm == 2) {
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 0),
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 0,
+                                    &mir),
                    "TRSM launch");
         } else if (X.opt.trsm == 1)
           CUDA_TRY(stfk::trsm_tile(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, ws),
@@ -235,6 +246,7 @@ struct Lowerer {
           CUDA_TRY(stfk::trsm_rlt(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb),
                    "TRSM launch");
         return 0;
+      }
       case stf::K_SYRK:
         CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[0]],
                                nb, X.buf[(size_t)t.out], nb, 1),
@@ -623,14 +635,15 @@ void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
   int64_t compute = 0;
   for (const auto& t : P.tasks) compute += (t.kind <= stf::K_GEMM);
   s->tasks = compute;
-  s->transfers = P.ntransfers;
+  s->transfers = P.ntransfers + P.npushed;
   s->edges = P.graph.nedges();
-  s->transfer_bytes = P.ntransfers * X.nb * X.nb * 8;
+  s->transfer_bytes = (P.ntransfers + P.npushed) * X.nb * X.nb * 8;
   s->critical_path = P.critical_path;
   s->graph_nodes = X.graph_nodes;
   s->kernel_launches = X.launches;
   s->build_ms = hit ? 0.0 : X.build_ms;
   s->graph_reuse = hit ? 1 : 0;
+  s->dag_tasks = (int64_t)P.tasks.size();
 }
 
 int choose_grid(int ngpus, int64_t grid_p, int* P, int* Q) {
@@ -703,6 +716,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.dataflow = env_int("STF_DATAFLOW", 1);
   C.opt.trsm = env_int("STF_TRSM", 2);
   C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 1);
+  C.opt.push = env_int("STF_PUSH", 0);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
@@ -825,6 +839,7 @@ int stf_set_option(const char* name, int64_t value) {
   } else if (n == "serial") C.opt.serial = value != 0;
   else if (n == "lookahead") C.opt.lookahead = value != 0;
   else if (n == "trsm_split") C.opt.trsm_split = value != 0;
+  else if (n == "push") C.opt.push = value != 0;
   else if (n == "threads") {
     if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
     C.opt.threads = value;
@@ -850,6 +865,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "serial") *value = C.opt.serial;
   else if (n == "lookahead") *value = C.opt.lookahead;
   else if (n == "trsm_split") *value = C.opt.trsm_split;
+  else if (n == "push") *value = C.opt.push;
   else if (n == "threads") *value = C.opt.threads;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;
@@ -919,7 +935,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
         e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
         e.key_graph == C.opt.graph &&
-        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.opt.trsm_split == C.opt.trsm_split && e.opt.lookahead == C.opt.lookahead && e.key_ptrs == ptrs &&
+        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.opt.trsm_split == C.opt.trsm_split && e.opt.push == C.opt.push && e.opt.lookahead == C.opt.lookahead && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
       C.cache.splice(C.cache.begin(), C.cache, it);
@@ -940,7 +956,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
       if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
           e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial && e.key_graph == C.opt.graph &&
           e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm &&
-          e.opt.trsm_split == C.opt.trsm_split && e.opt.lookahead == C.opt.lookahead && (e.gexec == nullptr) == (e.opt.graph == 0) &&
+          e.opt.trsm_split == C.opt.trsm_split && e.opt.push == C.opt.push && e.opt.lookahead == C.opt.lookahead && (e.gexec == nullptr) == (e.opt.graph == 0) &&
           !(pageable && e.gexec)) {
         int r = rebind(C, e, A_desc, ptrs);
         if (r) return r;
@@ -1007,6 +1023,8 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
   if (p < 1 || q < 1) return fail(-4, "bad grid %dx%d", p, q);
   Options o;
   o.priority = 1;
+  o.push = ctx().opt.push;            // the DAG options the next stf_potrf would use
+  o.lookahead = ctx().opt.lookahead;
   stf::Plan plan;
   auto t0 = std::chrono::steady_clock::now();
   stf::build_plan(plan, T, plan_options(o, p, q, p * q, false, false));
@@ -1030,7 +1048,7 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
     int64_t compute = 0;
     for (const auto& t : plan.tasks) compute += (t.kind <= stf::K_GEMM);
     stats->tasks = compute;
-    stats->transfers = plan.ntransfers;
+    stats->transfers = plan.ntransfers + plan.npushed;
     stats->edges = plan.graph.nedges();
     stats->transfer_bytes = 0;
     stats->critical_path = plan.critical_path;
@@ -1039,6 +1057,7 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
     stats->build_ms = ms;
     stats->device_ms = 0;
     stats->graph_reuse = 0;
+    stats->dag_tasks = (int64_t)plan.tasks.size();
   }
   return 0;
 }

@@ -104,3 +104,28 @@ def test_task_counts_closed_form(T):
     _, _, _, st = stf.dag(T, 1, 1)
     assert st["tasks"] == T + T * (T - 1) + T * (T - 1) * (T - 2) // 6
     assert st["critical_path"] == 3 * T - 2
+
+
+@pytest.mark.parametrize("T,p,q,known", [(8, 2, 2, None), (32, 2, 4, 1892)])
+def test_fused_push_replaces_panel_copies(T, p, q, known):
+    """NEXT-3: with push on, TRSM(i,k) writes L_ik's replicas itself: the only
+    COPY tasks left carry L_kk; total transfers are unchanged, and reachability
+    among compute tasks still equals the single-GPU STF closure."""
+    stf.set_option("push", 1)
+    try:
+        edges, kinds, ijk, st = stf.dag(T, p, q)
+    finally:
+        stf.set_option("push", 0)
+    assert st["transfers"] == _expected_transfers(T, p, q)
+    if known:
+        assert st["transfers"] == known
+    for t, k in enumerate(kinds):
+        if k == "COPY":
+            i, j, _ = ijk[t]
+            assert i == j  # only diagonal (POTRF) tiles are still copied
+    comp = [t for t, k in enumerate(kinds) if k != "COPY"]
+    R = oracle.transitive_closure(len(kinds), set(edges))
+    ot = oracle.cholesky_tasks(T)
+    if T <= 8:
+        Ro = oracle.transitive_closure(len(ot), oracle.stf_edges([acc for _, _, acc in ot]))
+        assert np.array_equal(R[np.ix_(comp, comp)], Ro)

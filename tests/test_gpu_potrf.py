@@ -54,7 +54,7 @@ def _reset_options(request):
     yield
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
-        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2, threads=8, lookahead=1, trsm_split=1)
+        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2, threads=8, lookahead=1, trsm_split=1, push=0)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
@@ -177,6 +177,11 @@ def test_bit_equal_across_virtual_grids(stf, p, q):
     assert np.array_equal(ref, _bits(stf, n, nb, p, q))
     assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0, threads=1))
     assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0, threads=p * q))  # one submission thread per slot
+    _options(stf, push=1)  # fused push: TRSM epilogues write the consumers' replicas
+    got = _bits(stf, n, nb, p, q)
+    st = stf.last_stats()
+    _options(stf, push=0)
+    assert np.array_equal(ref, got)
 
 
 def test_no_lookahead_fence_ablation_same_bits(stf):
