@@ -77,6 +77,29 @@ def test_parity_metric_inputs(stf, n, nb):
     assert backward_ratio(A, L) <= 10
 
 
+@pytest.mark.parametrize("n,nb", [(2, 2), (4, 2), (6, 2), (64, 2), (50, 10), (90, 18), (130, 26), (300, 150)])
+def test_parity_tiny_and_ragged_tiles(stf, n, nb):
+    """Degenerate tile sizes: 2x2 tiles (T up to 32), tiles not a multiple of the
+    16-row TMA box / 64-column dataflow block / 128-row CTA tile."""
+    M, info = _factor_spd(stf, n, nb, seed=5)
+    assert info == 0
+    L = M.to_dense().numpy()
+    A = synth.spd_matrix(5, n)
+    Lo, _ = oracle.potrf(A)
+    assert relF(L, Lo) <= 1e-10
+    assert backward_ratio(A, L) <= 10
+
+
+@pytest.mark.parametrize("n,nb,p,q", [(64, 2, 2, 4), (90, 18, 2, 2)])
+def test_tiny_tiles_on_virtual_grids_bit_equal(stf, n, nb, p, q):
+    ref = _bits(stf, n, nb, 1, 1, seed=6)
+    assert np.array_equal(ref, _bits(stf, n, nb, p, q, seed=6))
+    _options(stf, push=1)
+    got = _bits(stf, n, nb, p, q, seed=6)
+    _options(stf, push=0)
+    assert np.array_equal(ref, got)
+
+
 @pytest.fixture(scope="module")
 def oracle_8192():
     A = synth.spd_matrix(1, 8192)
