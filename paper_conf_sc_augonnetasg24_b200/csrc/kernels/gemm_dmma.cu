@@ -47,7 +47,7 @@ struct Cfg {
 };
 using CfgK16 = Cfg<16, 4>;  // 4 x 32 KB stages
 using CfgK32 = Cfg<32, 3>;  // 3 x 64 KB stages
-using CfgN64 = Cfg<32, 2, 64, 2>;  // 128 x 64 CTA tile, 4 warps, 2 x 48 KB stages, 2 CTAs / SM (full GEMMs only)
+using CfgN64 = Cfg<32, 2, 64, 2>;  // 128 x 64 CTA tile, 2 x 48 KB stages, 2 CTAs / SM (full GEMMs only)
 
 // Exact negation as a sign-bit flip on the integer pipe (keeps the FP64/DMMA pipe free).
 __device__ __forceinline__ double neg(double x) {
@@ -92,13 +92,22 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
 
   int tm, tn;
   if (lower) {
-    // linear block -> (tm >= tn)
-    int b = blockIdx.x;
-    int t = (int)((sqrtf(8.0f * b + 1.0f) - 1.0f) * 0.5f);
-    while ((t + 1) * (t + 2) / 2 <= b) ++t;
-    while (t * (t + 1) / 2 > b) --t;
-    tm = t;
-    tn = b - t * (t + 1) / 2;
+    // linear block -> CTA tiles touching the lower triangle.  BN == BM: tn <= tm
+    // (row tm holds tm + 1 tiles); BN == BM / 2: tn <= 2 tm + 1 (row tm holds 2 tm + 2).
+    const int b = blockIdx.x;
+    if (g::BN == g::BM) {
+      int t = (int)((sqrtf(8.0f * b + 1.0f) - 1.0f) * 0.5f);
+      while ((t + 1) * (t + 2) / 2 <= b) ++t;
+      while (t * (t + 1) / 2 > b) --t;
+      tm = t;
+      tn = b - t * (t + 1) / 2;
+    } else {
+      int t = (int)((sqrtf(4.0f * b + 1.0f) - 1.0f) * 0.5f);
+      while ((t + 1) * (t + 2) <= b) ++t;
+      while (t * (t + 1) > b) --t;
+      tm = t;
+      tn = b - t * (t + 1);
+    }
   } else {
     tm = blockIdx.x;
     tn = blockIdx.y;
@@ -124,7 +133,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
   const int gq = lane >> 2, tq = lane & 3;
 
   // In lower mode, warps of a diagonal CTA whose warp tile is strictly upper idle.
-  const bool warp_dead = lower && (m0 == n0) && (wm0 + WM <= wn0);
+  const bool warp_dead = lower && (m0 + wm0 + WM <= n0 + wn0);  // warp tile strictly above the diagonal
 
   // acc = C, loaded straight into the accumulators (64 independent loads in
   // flight, latency hidden behind the first TMA wait); the mainloop adds
@@ -252,9 +261,11 @@ static int gemm_bk() {
   static int v = env_or("STF_GEMM_BK", 32) == 16 ? 16 : 32;
   return v;
 }
-// STF_GEMM_NARROW=1: full (non-SYRK) GEMMs use the 128 x 64 tile, 2 CTAs per SM
+// CTA tile: STF_GEMM_NARROW = 2 (default): 128 x 64, 8 warps of 32 x 32, 2 CTAs per SM
+// (one CTA's start-up and epilogue hide behind the other's mainloop: 95.6% of peak
+// on 8192^2 x 1024); 1: 128 x 64, 4 warps of 64 x 32; 0: 128 x 128, 1 CTA per SM.
 static int gemm_narrow() {
-  static int v = env_or("STF_GEMM_NARROW", 0);
+  static int v = env_or("STF_GEMM_NARROW", 2);
   return v;
 }
 
@@ -275,14 +286,14 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
     return cudaErrorMisalignedAddress;
-  const bool narrow = !lower && gemm_narrow();
+  const bool narrow = gemm_narrow() != 0;
   const int bk = narrow ? 32 : gemm_bk();
   CUtensorMap tmA, tmB;
   if (!make_operand_map(&tmA, A, M, K, lda, bk) || !make_operand_map(&tmB, B, N, K, ldb, bk))
     return cudaErrorInvalidValue;
   const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = lower ? dim3(tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
+  cfg.gridDim = lower ? dim3(narrow ? tM * (tM + 1) : tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributePriority;
@@ -292,7 +303,11 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   ++launch_count();
   if (narrow) {
     cfg.dynamicSmemBytes = CfgN64::SMEM_BYTES;
-    cfg.blockDim = dim3(128, 1, 1);
+    if (gemm_narrow() == 2) {  // 8 warps of 32 x 32, 2 CTAs (16 warps) per SM
+      cfg.blockDim = dim3(256, 1, 1);
+      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64>, tmA, tmB, C, ldc, M, N, K, lower);
+    }
+    cfg.blockDim = dim3(128, 1, 1);  // 4 warps of 64 x 32
     return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, CfgN64>, tmA, tmB, C, ldc, M, N, K, lower);
   }
   if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
@@ -314,6 +329,9 @@ cudaError_t gemm_init_attrs() {
   if (e == cudaSuccess) e = set_attrs<CfgK32>();
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<64, 32, CfgN64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             CfgN64::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, CfgN64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              CfgN64::SMEM_BYTES);
   return e;
 }
