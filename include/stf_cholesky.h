@@ -97,8 +97,9 @@ const char *stf_last_error(void);
  * Execution options (defaults from the environment at init):
  *   "dataflow" STF_DATAFLOW POTRF tile kernel: 1 single-launch dataflow (default), 0 recursive
  *   "trsm"     STF_TRSM     TRSM tile kernel: 2 row-panel (default), 1 dataflow, 0 recursive
- *   "trsm_split" STF_TRSM_SPLIT 1: non-critical row-panel TRSMs run as panel + GEMM + panel
- *                           on column halves (default); 0: one panel launch
+ *   "trsm_split" STF_TRSM_SPLIT P in [1,16]: non-critical row-panel TRSMs run right-looking
+ *                           over P column blocks (panel kernel + GEMM updates; default 4);
+ *                           1: one panel launch
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA
  *                           graph, memoised per (n, nb, grid, tiles) (default);
  *                           0: eager lowering on streams + events

@@ -144,11 +144,17 @@ struct Builder {
     // the other TRSMs and the next column's GEMMs gate the next panel (4); later
     // columns decay with their distance d = column - k.
     const bool prio = p.opt.priority;
-    auto level = [&](int64_t d) -> int { return d <= 1 ? 4 : d == 2 ? 3 : d <= 4 ? 2 : d <= 8 ? 1 : 0; };
+    const int mode = p.opt.prio_mode;
+    auto level = [&](int64_t d) -> int {
+      if (mode == 3) return d <= 1 ? 4 : 0;                                  // two levels
+      if (mode == 2) return d <= 1 ? 4 : d == 2 ? 3 : d == 3 ? 2 : d <= 5 ? 1 : 0;  // faster decay
+      return d <= 1 ? 4 : d == 2 ? 3 : d <= 4 ? 2 : d <= 8 ? 1 : 0;
+    };
     auto P = [&](int lv) { return prio ? lv : 0; };
     for (int64_t k = 0; k < T; ++k) {
       compute(K_POTRF, k, k, k, P(5), -1, -1, k, k);
-      for (int64_t i = k + 1; i < T; ++i) compute(K_TRSM, i, k, k, P(i == k + 1 ? 5 : 4), key(k, k), -1, i, k);
+      for (int64_t i = k + 1; i < T; ++i)
+        compute(K_TRSM, i, k, k, P(i == k + 1 || mode == 1 ? 5 : 4), key(k, k), -1, i, k);
       for (int64_t i = k + 1; i < T; ++i) {
         compute(K_SYRK, i, i, k, P(i == k + 1 ? 5 : level(i - k)), key(i, k), -1, i, i);
         for (int64_t j = k + 1; j < i; ++j) compute(K_GEMM, i, j, k, P(level(j - k)), key(i, k), key(j, k), i, j);

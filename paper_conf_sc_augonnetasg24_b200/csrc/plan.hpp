@@ -49,6 +49,7 @@ struct PlanOptions {
   int copy_streams = 2;
   bool serial = false;     // all tasks of all slots on stream 0 (program order)
   bool priority = true;
+  int prio_mode = 0;       // level assignment variant (0 default; see plan.cpp)
   bool with_load = false;  // LOAD tasks first (COLMAJOR descriptors)
   bool with_store = false; // STORE tasks (write-back) at the end of program order
   bool lookahead = true;   // false: a FENCE task (RW on every tile) closes each panel step, so

@@ -78,7 +78,7 @@ struct Slot {
 struct Options {
   int64_t dataflow = 1;  // POTRF tile kernel: 1 single-launch dataflow, 0 recursive (GEMM-based)
   int64_t trsm = 2;      // TRSM tile kernel: 2 row-panel, 1 dataflow, 0 recursive
-  int64_t trsm_split = 1;  // row panel: non-critical TRSMs as panel(nb/2) + GEMM + panel(nb/2)
+  int64_t trsm_split = 4;  // row panel: non-critical TRSMs as `trsm_split` column blocks (panel + GEMM updates)
   int64_t graph = 1;
   int64_t streams = 8;
   int64_t serial = 0;
@@ -112,6 +112,7 @@ struct Exec {
   cudaGraphExec_t gexec = nullptr;
   int64_t graph_nodes = 0;
   int graph_fallback = 0;  // capture failed, eager lowering used
+  unsigned skip_mask = 0;  // STF_DEBUG_SKIP: task kinds whose kernels are not launched (timing what-ifs)
   int64_t updates = 0;     // successful cudaGraphExecUpdate re-binds
   bool rebound = false;
   int64_t launches = 0;
@@ -170,6 +171,7 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.copy_streams = kCopyStreams;
   po.serial = o.serial != 0;
   po.priority = o.priority != 0;
+  po.prio_mode = (int)env_int("STF_PRIO_MODE", 0);
   po.with_load = load;
   po.with_store = store;
   po.lookahead = o.lookahead != 0;
@@ -201,6 +203,7 @@ struct Lowerer {
 
   int body(const stf::Task& t, size_t tidx, cudaStream_t s, int prio) {
     const int64_t nb = X.nb;
+    if (X.skip_mask & (1u << t.kind)) return 0;  // debug what-if timing only (results invalid)
     int* ws = X.task_ws.empty() ? nullptr : X.task_ws[tidx];
     const size_t tile_bytes = (size_t)(nb * nb) * sizeof(double);
     Slot& S = C.slots[(size_t)t.slot];
@@ -214,27 +217,40 @@ struct Lowerer {
                    "POTRF launch");
         return 0;
       case stf::K_TRSM: {
-        stfk::Mirrors mir{}, mir2{};
-        for (int m = 0; m < t.nmir && m < 7; ++m) {
-          mir.p[m] = X.buf[(size_t)t.mir[m]];
-          mir2.p[m] = mir.p[m] + (nb / 2) * nb;  // second column half (split variant)
+        stfk::Mirrors mir{};
+        for (int m = 0; m < t.nmir && m < 7; ++m) mir.p[m] = X.buf[(size_t)t.mir[m]];
+        mir.n = t.nmir < 7 ? t.nmir : 7;
+        if ((X.skip_mask & (3u << 16)) && t.i != t.k + 1) {  // debug what-if: non-critical TRSM costed as a GEMM
+          const int kk = (X.skip_mask & (1u << 17)) ? (int)(nb / 2) : (int)nb;   // (half: triangular-GEMM flops)
+          CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, kk, X.buf[(size_t)t.out], nb, X.buf[(size_t)t.in[0]],
+                                 nb, X.buf[(size_t)t.out], nb, 0),
+                   "TRSM what-if");
+          return 0;
         }
-        mir.n = mir2.n = t.nmir < 7 ? t.nmir : 7;
         if (X.opt.trsm == 2 && t.i == t.k + 1) {
           // the next panel's TRSM(k+1,k) is on the critical path: one low-latency launch
           CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 32,
                                     &mir),
                    "TRSM launch");
-        } else if (X.opt.trsm == 2 && X.opt.trsm_split && nb >= 512 && (nb / 2) % 64 == 0) {
-          // X = [X1 X2]: X1 = B1 L11^-T; B2 -= X1 L21^T (full-rate GEMM kernel); X2 = B2 L22^-T.
-          // Half of the TRSM flops run on the GEMM kernel (SM-time, not latency, matters here).
-          const int64_t h = nb / 2;
+        } else if (X.opt.trsm == 2 && X.opt.trsm_split > 1 && nb % (64 * X.opt.trsm_split) == 0) {
+          // Right-looking over `parts` column blocks of width w:
+          //   X_p = B_p L_pp^-T (row-panel kernel);  B_{>p} -= X_p L_{>p,p}^T (full-rate GEMM kernel).
+          // Only 1/parts of the TRSM flops stay in the substitution kernel (SM-time matters here,
+          // not latency; the critical TRSM(k+1,k) takes the single-launch branch above).
+          const int64_t parts = X.opt.trsm_split, w = nb / parts;
           const double* L = X.buf[(size_t)t.in[0]];
           double* B = X.buf[(size_t)t.out];
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L, nb, B, nb, 0, &mir), "TRSM launch");
-          CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)h, (int)h, B, nb, L + h, nb, B + h * nb, nb, 0), "TRSM GEMM");
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)h, L + h * nb + h, nb, B + h * nb, nb, 0, &mir2),
-                   "TRSM launch");
+          for (int64_t pp = 0; pp < parts; ++pp) {
+            stfk::Mirrors mp = mir;
+            for (int m = 0; m < mp.n; ++m) mp.p[m] = mir.p[m] + pp * w * nb;
+            CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)w, L + pp * w * nb + pp * w, nb, B + pp * w * nb, nb, 0,
+                                      &mp),
+                     "TRSM launch");
+            if (pp + 1 < parts)
+              CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)(nb - (pp + 1) * w), (int)w, B + pp * w * nb, nb,
+                                     L + pp * w * nb + (pp + 1) * w, nb, B + (pp + 1) * w * nb, nb, 0),
+                       "TRSM GEMM");
+          }
         } else if (X.opt.trsm == 2) {
           CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 0,
                                     &mir),
@@ -715,7 +731,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.graph = env_int("STF_GRAPH", 1);
   C.opt.dataflow = env_int("STF_DATAFLOW", 1);
   C.opt.trsm = env_int("STF_TRSM", 2);
-  C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 1);
+  C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 4);
   C.opt.push = env_int("STF_PUSH", 0);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
@@ -838,7 +854,10 @@ int stf_set_option(const char* name, int64_t value) {
     C.opt.streams = value;
   } else if (n == "serial") C.opt.serial = value != 0;
   else if (n == "lookahead") C.opt.lookahead = value != 0;
-  else if (n == "trsm_split") C.opt.trsm_split = value != 0;
+  else if (n == "trsm_split") {
+    if (value < 1 || value > 16) return fail(-105, "trsm_split must be in [1, 16]");
+    C.opt.trsm_split = value;
+  }
   else if (n == "push") C.opt.push = value != 0;
   else if (n == "threads") {
     if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
@@ -983,6 +1002,20 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     e->key_ld = A_desc->ld;
     e->key_dev = A_desc->device;
     if (A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr)) e->opt.graph = 0;  // pageable: no capture
+    if (const char* sk = getenv("STF_DEBUG_SKIP")) {
+      std::string v(sk);
+      const char* names[] = {"potrf", "trsm", "syrk", "gemm", "copy", "trsm_as_gemm", "trsm_as_half_gemm"};
+      const unsigned bits[] = {1u << 0, 1u << 1, 1u << 2, 1u << 3, 1u << 4, 1u << 16, 1u << 17};
+      size_t pos = 0;
+      while (pos <= v.size()) {  // comma-separated list of exact names
+        size_t end = v.find(',', pos);
+        if (end == std::string::npos) end = v.size();
+        const std::string item = v.substr(pos, end - pos);
+        for (unsigned k = 0; k < 7; ++k)
+          if (item == names[k]) e->skip_mask |= bits[k];
+        pos = end + 1;
+      }
+    }
     int r = prepare(C, *e, A_desc);
     if (r == -103 && !C.cache.empty()) {  // out of memory: drop memoised plans and retry once
       C.cache.clear();

@@ -24,11 +24,11 @@ def stf():
     s.finalize()
 
 
-@pytest.mark.parametrize("trsm,split", [(1, 0), (2, 0), (2, 1)])
+@pytest.mark.parametrize("trsm,split", [(1, 1), (2, 1), (2, 2), (2, 4), (2, 8)])
 def test_parity_trsm_variants(stf, trsm, split):
     _options(stf, trsm=trsm, trsm_split=split)
     M, info = _factor_spd(stf, 1536, 512, seed=2)
-    _options(stf, trsm=2, trsm_split=1)
+    _options(stf, trsm=2, trsm_split=4)
     assert info == 0
     Lo, _ = oracle.potrf(synth.spd_matrix(2, 1536))
     assert relF(M.to_dense().numpy(), Lo) <= 1e-10
@@ -54,7 +54,7 @@ def _reset_options(request):
     yield
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
-        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2, threads=8, lookahead=1, trsm_split=1, push=0)
+        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2, threads=8, lookahead=1, trsm_split=4, push=0)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):

@@ -24,7 +24,9 @@ VARIANTS = [
     ("no look-ahead: fence per panel step (STF_LOOKAHEAD=0)", {"STF_LOOKAHEAD": "0"}),
     ("eager streams+events, no graph (STF_GRAPH=0)", {"STF_GRAPH": "0"}),
     ("TRSM dataflow kernel (STF_TRSM=1)", {"STF_TRSM": "1"}),
-    ("TRSM one panel launch, no GEMM split (STF_TRSM_SPLIT=0)", {"STF_TRSM_SPLIT": "0"}),
+    ("TRSM one panel launch, no GEMM split (STF_TRSM_SPLIT=1)", {"STF_TRSM_SPLIT": "1"}),
+    ("TRSM split in 2 column blocks (STF_TRSM_SPLIT=2)", {"STF_TRSM_SPLIT": "2"}),
+    ("TRSM split in 8 column blocks (STF_TRSM_SPLIT=8)", {"STF_TRSM_SPLIT": "8"}),
     ("TRSM row panel 32 rows (STF_TRSM_ROWS=32)", {"STF_TRSM_ROWS": "32"}),
     ("TRSM + POTRF recursive (STF_TRSM=0 STF_DATAFLOW=0)", {"STF_TRSM": "0", "STF_DATAFLOW": "0"}),
     ("GEMM 16 warps 32x32 (STF_GEMM_WARPS=16)", {"STF_GEMM_WARPS": "16"}),
