@@ -193,6 +193,31 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
  * written (<= cap) or a negative error.  Not part of the factorisation. */
 int64_t stf_debug_potrf_trace(int64_t n, double *A, int64_t lda, int ctas, int64_t *trace, int64_t cap);
 
+/* ---------------------------------------------------------------- multi-process mode
+ * One process per GPU (e.g. torch.distributed / torchrun): process `rank` owns
+ * slot `rank` of a p x q grid (p*q == world) on CUDA device `device`.  Every
+ * process builds the same plan (the STF DAG is deterministic) and runs only its
+ * own slot's tasks.  A finished tile is pushed into the consumer process's
+ * replica over NVLink (copy-engine copy into CUDA-IPC-mapped memory, or the
+ * TRSM epilogue's peer stores with "push"), followed by a 32-bit flag write
+ * into the consumer's flag array (cuStreamWriteValue32); the consumer's stream
+ * waits on that flag (cuStreamWaitValue32) -- device-side hand-off, no host
+ * round trip, no SMs.
+ *   1. stf_mp_init(rank, world, device)
+ *   2. stf_mp_prepare(n, nb, desc, blob): desc = TILED_2DBC whose tiles table
+ *      holds this process's own tiles (others ignored); writes this process's
+ *      stf_mp_blob_size() bytes of IPC handles into blob
+ *   3. exchange the blobs (all-gather, rank order) and call stf_mp_import(blobs)
+ *   4. per factorisation: barrier across processes, stf_mp_potrf() (returns the
+ *      LAPACK info of this process's columns; the caller takes the minimum > 0
+ *      over processes), barrier.
+ * stf_finalize releases everything.  Errors as above. */
+int stf_mp_init(int rank, int world, int device);
+int64_t stf_mp_blob_size(void);
+int stf_mp_prepare(int64_t n, int64_t nb, const stf_matrix_desc *A_desc, void *blob);
+int stf_mp_import(const void *blobs);
+int stf_mp_potrf(void);
+
 #ifdef __cplusplus
 }
 #endif

@@ -162,6 +162,63 @@ class TiledMatrix:
         return check(_abi.stf_potrf(self.n, self.nb, b"L", ctypes.byref(self.desc), self.ngpus), "stf_potrf")
 
 
+class MpTiledMatrix:
+    """Multi-process mode (one process per GPU): this process's share of a
+    p x q block-cyclic TILED_2DBC matrix -- only the tiles it owns, in one
+    allocation on `device`.  Usage (see include/stf_cholesky.h):
+
+        mp_init(rank, world, device)
+        A = MpTiledMatrix(n, nb, p, q, rank, device); A.fill_spd(seed)
+        blob = A.prepare(); A.import_blobs(all_gather(blob)); barrier()
+        info = A.potrf(); barrier()
+
+    The blob exchange and barriers are the caller's (torch.distributed).
+    """
+
+    def __init__(self, n: int, nb: int, p: int, q: int, rank: int, device: int):
+        import torch
+
+        assert n % nb == 0 and 0 <= rank < p * q
+        self.n, self.nb, self.p, self.q, self.rank, self.device = n, nb, p, q, rank, device
+        self.T = T = n // nb
+        own = [(i, j) for j in range(T) for i in range(j, T) if self.owner(i, j) == rank]
+        self.slab = torch.empty((max(1, len(own)), nb, nb), dtype=torch.float64, device="cuda:%d" % device)
+        self.tiles = {ij: self.slab[k] for k, ij in enumerate(own)}
+        self._table = (ctypes.c_void_p * (T * T))()
+        for (i, j), t in self.tiles.items():
+            self._table[i + j * T] = t.data_ptr()
+        self.desc = stf_matrix_desc(STF_DESC_TILED_2DBC, device, 0, None, p, q,
+                                    ctypes.cast(self._table, ctypes.POINTER(ctypes.c_void_p)))
+
+    def owner(self, i: int, j: int) -> int:
+        return (i % self.p) * self.q + (j % self.q)
+
+    def fill_spd(self, seed: int) -> None:
+        check(_abi.stf_fill_spd_tiles(self.n, self.nb, ctypes.byref(self.desc), self.p * self.q, seed),
+              "stf_fill_spd_tiles")
+
+    def prepare(self) -> bytes:
+        """Build this process's plan and return its IPC blob (stf_mp_prepare)."""
+        buf = ctypes.create_string_buffer(int(_abi.stf_mp_blob_size()))
+        check(_abi.stf_mp_prepare(self.n, self.nb, ctypes.byref(self.desc), buf), "stf_mp_prepare")
+        return buf.raw
+
+    def import_blobs(self, blobs: Sequence[bytes]) -> None:
+        """stf_mp_import with every process's blob, in rank order."""
+        joined = b"".join(blobs)
+        assert len(joined) == len(blobs) * int(_abi.stf_mp_blob_size())
+        buf = ctypes.create_string_buffer(joined, len(joined))
+        check(_abi.stf_mp_import(buf), "stf_mp_import")
+
+    def potrf(self) -> int:
+        """stf_mp_potrf: runs this process's tasks; LAPACK info of its columns."""
+        return check(_abi.stf_mp_potrf(), "stf_mp_potrf")
+
+
+def mp_init(rank: int, world: int, device: int) -> None:
+    check(_abi.stf_mp_init(rank, world, device), "stf_mp_init")
+
+
 def potrf_colmajor(ptr: int, n: int, ld: int, nb: int, uplo: str = "L", device: Optional[int] = None,
                    ngpus: int = 1) -> int:
     """stf_potrf on a caller column-major matrix (device ordinal -> DEVICE_COLMAJOR,

@@ -16,6 +16,7 @@
 //   A12 abstract events: a task's completion is an event only when a successor
 //       runs on another stream; in a graph these become plain edges.
 //   A13 finalize: synchronous completion + write-back.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -121,8 +122,22 @@ struct Exec {
   double* mat = nullptr;
   int64_t ld = 0;
   int mat_dev = -1;  // -1: host
+  // multi-process mode (one process per slot): replicas of slot s live in slot s's
+  // arena at rep_off[b]; their readiness is a 32-bit flag (index flag_idx[b]) in
+  // slot s's flag array, written by the remote producer after the transfer.
+  bool mp = false;
+  std::vector<size_t> rep_off;        // per buffer id (replicas), element offset in its slot's arena
+  std::vector<int> flag_idx;          // per buffer id (replicas), index in its slot's flag array
+  double* local_arena = nullptr;      // this slot's replica arena (exported)
+  uint32_t* local_flags = nullptr;    // this slot's flags (exported)
+  size_t local_flag_count = 0;
+  std::vector<double*> peer_arena;    // per slot, IPC-mapped (null for self / no replicas)
+  std::vector<uint32_t*> peer_flags;  // per slot, IPC-mapped
+  std::vector<void*> ipc_opened;      // to cudaIpcCloseMemHandle
+  uint32_t epoch = 0;
 
   ~Exec() {
+    for (void* p : ipc_opened) cudaIpcCloseMemHandle(p);
     if (gexec) cudaGraphExecDestroy(gexec);
     if (graph) cudaGraphDestroy(graph);
     for (size_t t = 0; t < events.size(); ++t)
@@ -150,7 +165,25 @@ struct Context {
   std::vector<cudaEvent_t> fork_join;  // per slot-stream, for fork/join around a call
   cudaEvent_t t_start = nullptr, t_end = nullptr;  // timing events on `origin`
   double device_ms = 0;
+  int mp_me = -1;  // multi-process mode: the slot this process owns (-1: single-process mode)
+  std::unique_ptr<Exec> mp_exec;  // multi-process mode: the current plan
 };
+
+// CUDA driver stream memory operations (flag hand-off between processes, no SMs)
+typedef CUresult (*PFN_wv32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+PFN_wv32 g_write_value32 = nullptr, g_wait_value32 = nullptr;
+bool load_memops() {
+  if (g_write_value32 && g_wait_value32) return true;
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &p, cudaEnableDefault, &q) == cudaSuccess &&
+      q == cudaDriverEntryPointSuccess)
+    g_write_value32 = reinterpret_cast<PFN_wv32>(p);
+  if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &p, cudaEnableDefault, &q) == cudaSuccess &&
+      q == cudaDriverEntryPointSuccess)
+    g_wait_value32 = reinterpret_cast<PFN_wv32>(p);
+  return g_write_value32 && g_wait_value32;
+}
 
 Context& ctx() {
   static Context c;
@@ -383,18 +416,43 @@ struct Lowerer {
     const stf::Plan& P = X.plan;
     for (size_t t = 0; t < P.tasks.size(); ++t) {
       const stf::Task& task = P.tasks[t];
+      if (X.mp && task.slot != C.mp_me) continue;  // another process runs it
       if (task.slot % nt != w) continue;
       set_dev(C.slots[(size_t)task.slot].device);
       cudaStream_t s = stream_of(task);
+      if (X.mp) {
+        // inputs that are replicas here were written by another process: wait
+        // (on the device, no host round trip) for the producer's flag
+        for (int a = 0; a < 2; ++a) {
+          const int64_t b = task.in[a];
+          if (b >= 0 && P.buffers[(size_t)b].replica && task.kind != stf::K_COPY) {
+            const CUresult cr = g_wait_value32((CUstream)s, (CUdeviceptr)(X.local_flags + X.flag_idx[(size_t)b]),
+                                               X.epoch, CU_STREAM_WAIT_VALUE_GEQ);
+            if (cr != CUDA_SUCCESS) return fail(-101, "cuStreamWaitValue32 failed (%d)", (int)cr);
+          }
+        }
+      }
       for (const int64_t* q = P.graph.preds_begin((int64_t)t); q != P.graph.preds_end((int64_t)t); ++q) {
         const stf::Task& pt = P.tasks[(size_t)*q];
         if (pt.slot == task.slot && pt.stream == task.stream) continue;  // stream order suffices
+        if (X.mp && pt.slot != C.mp_me) continue;  // cross-process: replica flags above
         if (recorded && pt.slot % nt != w)
           while (!recorded[*q].load(std::memory_order_acquire)) std::this_thread::yield();
         CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
       }
       int r = body(task, t, s, prio_of(task));
       if (r) return r;
+      if (X.mp) {  // publish remote replicas written by this task (COPY target, fused-push mirrors)
+        auto signal = [&](int64_t b) -> int {
+          const int dst = P.buffers[(size_t)b].slot;
+          const CUresult cr = g_write_value32((CUstream)s, (CUdeviceptr)(X.peer_flags[(size_t)dst] + X.flag_idx[(size_t)b]),
+                                              X.epoch, CU_STREAM_WRITE_VALUE_DEFAULT);
+          return cr == CUDA_SUCCESS ? 0 : fail(-101, "cuStreamWriteValue32 failed (%d)", (int)cr);
+        };
+        if (task.kind == stf::K_COPY && (r = signal(task.out))) return r;
+        for (int m = 0; m < task.nmir; ++m)
+          if ((r = signal(task.mir[m]))) return r;
+      }
       if (X.events[t]) CUDA_TRY(cudaEventRecord(X.events[t], s), "event record");
       if (recorded) recorded[t].store(1, std::memory_order_release);
     }
@@ -461,8 +519,38 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
     X.ld = desc->ld;
     X.mat_dev = (X.kind == STF_DESC_DEVICE_COLMAJOR) ? desc->device : -1;
   }
+  if (X.mp) {
+    // offsets and flag slots of every replica, identical in every process (same plan)
+    X.rep_off.assign(P.buffers.size(), 0);
+    X.flag_idx.assign(P.buffers.size(), -1);
+    std::vector<size_t> used((size_t)X.ngpus, 0);
+    for (size_t b = 0; b < P.buffers.size(); ++b) {
+      const stf::Buffer& B = P.buffers[b];
+      if (!B.replica) continue;
+      X.flag_idx[b] = (int)used[(size_t)B.slot];
+      X.rep_off[b] = (used[(size_t)B.slot]++) * (size_t)(X.nb * X.nb);
+    }
+    const int me = C.mp_me;
+    const size_t cnt = used[(size_t)me];
+    X.local_flag_count = cnt;
+    if (cnt) {
+      double* arena = nullptr;
+      int r = alloc_on(X, C.slots[(size_t)me].device, cnt * tile_bytes, &arena);
+      if (r) return r;
+      X.local_arena = arena;
+      double* fl = nullptr;
+      r = alloc_on(X, C.slots[(size_t)me].device, (cnt * sizeof(uint32_t) + 7) / 8 * 8, &fl);
+      if (r) return r;
+      X.local_flags = reinterpret_cast<uint32_t*>(fl);
+      CUDA_TRY(cudaMemset(X.local_flags, 0, cnt * sizeof(uint32_t)), "flag init");
+      for (size_t b = 0; b < P.buffers.size(); ++b)
+        if (P.buffers[b].replica && P.buffers[b].slot == me) X.buf[b] = arena + X.rep_off[b];
+    }
+    X.peer_arena.assign((size_t)X.ngpus, nullptr);
+    X.peer_flags.assign((size_t)X.ngpus, nullptr);
+  }
   // library-owned storage: per slot one arena for (COLMAJOR) home tiles + replicas
-  for (int s = 0; s < X.ngpus; ++s) {
+  for (int s = 0; s < X.ngpus && !X.mp; ++s) {
     size_t count = 0;
     for (size_t b = 0; b < P.buffers.size(); ++b) {
       const stf::Buffer& B = P.buffers[b];
@@ -488,6 +576,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   if (X.opt.dataflow || X.opt.trsm == 1) {
     const size_t wsb = stfk::dataflow_ws_bytes((int)X.nb, (int)X.nb);
     for (int s = 0; s < X.ngpus; ++s) {
+      if (X.mp && s != C.mp_me) continue;
       size_t cnt = 0;
       for (const auto& t : P.tasks) cnt += (t.slot == s && (t.kind == stf::K_POTRF || t.kind == stf::K_TRSM));
       if (!cnt) continue;
@@ -513,6 +602,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   X.events_dev.assign(P.tasks.size(), 0);
   for (size_t t = 0; t < P.tasks.size(); ++t) {
     const stf::Task& a = P.tasks[t];
+    if (X.mp && a.slot != C.mp_me) continue;  // never issued here
     bool need = false;
     for (int64_t e = soff[t]; e < soff[t + 1] && !need; ++e) {
       const stf::Task& b = P.tasks[(size_t)succ[(size_t)e]];
@@ -617,6 +707,7 @@ int rebind(Context& C, Exec& X, const stf_matrix_desc* desc, const std::vector<u
 }
 
 int run(Context& C, Exec& X) {
+  if (X.mp) X.epoch++;  // flags are monotonic: run e waits for value >= e
   cudaSetDevice(C.origin_dev);
   CUDA_TRY(cudaEventRecord(C.t_start, C.origin), "timing start");
   if (X.opt.graph) {
@@ -802,6 +893,8 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
 
 static void release_all(Context& C) {
   C.cache.clear();
+  C.mp_exec.reset();
+  C.mp_me = -1;
   for (size_t k = 0; k < C.fork_join.size(); ++k)
     if (C.fork_join[k]) cudaEventDestroy(C.fork_join[k]);
   C.fork_join.clear();
@@ -1133,6 +1226,7 @@ int stf_fill_spd_tiles(int64_t n, int64_t nb, const stf_matrix_desc* A_desc, int
   for (int64_t j = 0; j < T; ++j)
     for (int64_t i = j; i < T; ++i) {
       double* tp = A_desc->tiles[(size_t)(i + j * T)];
+      if (!tp) continue;  // not held by this process (multi-process mode)
       int d = 0;
       if (!device_of(tp, &d)) return fail(-4, "tile (%lld,%lld) is not device memory", (long long)i, (long long)j);
       cudaSetDevice(d);
@@ -1216,6 +1310,114 @@ int stf_kernel_potrf(int64_t n, double* A, int64_t lda, int64_t* info) {
   if (e != cudaSuccess) return cuda_fail(e, "potrf");
   if (info) *info = (v == ULLONG_MAX) ? 0 : (int64_t)v;
   return 0;
+}
+
+// ---------------------------------------------------------------- multi-process mode
+namespace {
+struct MpBlob {
+  int32_t magic;
+  int32_t slot;
+  int64_t count;  // replicas (and flags) of this slot
+  cudaIpcMemHandle_t arena;
+  cudaIpcMemHandle_t flags;
+};
+constexpr int32_t kMpMagic = 0x53544650;  // "STFP"
+}  // namespace
+
+int stf_mp_init(int rank, int world, int device) {
+  if (world < 1 || rank < 0 || rank >= world) return fail(-5, "bad rank %d / world %d", rank, world);
+  if (!load_memops()) return fail(-101, "CUDA stream memory operations unavailable");
+  std::vector<int> devs((size_t)world, device);
+  int r = stf_cholesky_init(world, devs.data());
+  if (r) return r;
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  C.mp_me = rank;
+  return 0;
+}
+
+int64_t stf_mp_blob_size(void) { return (int64_t)sizeof(MpBlob); }
+
+int stf_mp_prepare(int64_t n, int64_t nb, const stf_matrix_desc* A_desc, void* blob) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (C.mp_me < 0) return fail(-100, "stf_mp_prepare: call stf_mp_init first");
+  if (n < 1 || nb < 2 || (nb & 1) || n % nb || nb > 16384) return fail(-2, "bad n / nb");
+  if (!A_desc || A_desc->kind != STF_DESC_TILED_2DBC || !A_desc->tiles) return fail(-4, "TILED_2DBC descriptor required");
+  const int world = (int)C.slots.size();
+  if ((int64_t)A_desc->p * A_desc->q != world) return fail(-4, "grid %dx%d != world %d", A_desc->p, A_desc->q, world);
+  if (C.opt.lookahead == 0) return fail(-105, "lookahead=0 (fence tasks) is not supported in multi-process mode");
+  const int64_t T = n / nb;
+  const int P = A_desc->p, Q = A_desc->q, me = C.mp_me;
+  for (int64_t j = 0; j < T; ++j)
+    for (int64_t i = j; i < T; ++i) {
+      if ((int)((i % P) * Q + (j % Q)) != me) continue;
+      const double* tp = A_desc->tiles[(size_t)(i + j * T)];
+      int d = -1;
+      if (!tp || !device_of(tp, &d) || d != C.slots[(size_t)me].device)
+        return fail(-4, "own tile (%lld,%lld) is not device memory on this process's device", (long long)i,
+                    (long long)j);
+    }
+  std::unique_ptr<Exec> e(new Exec());
+  e->n = n;
+  e->nb = nb;
+  e->kind = STF_DESC_TILED_2DBC;
+  e->ngpus = world;
+  e->P = P;
+  e->Q = Q;
+  e->opt = C.opt;
+  e->opt.graph = 0;  // eager, multi-threaded submission is not needed: one slot per process
+  e->mp = true;
+  int r = prepare(C, *e, A_desc);
+  if (r) return r;
+  MpBlob b{};
+  b.magic = kMpMagic;
+  b.slot = me;
+  b.count = (int64_t)e->local_flag_count;
+  if (e->local_flag_count) {
+    CUDA_TRY(cudaIpcGetMemHandle(&b.arena, e->local_arena), "cudaIpcGetMemHandle(arena)");
+    CUDA_TRY(cudaIpcGetMemHandle(&b.flags, e->local_flags), "cudaIpcGetMemHandle(flags)");
+  }
+  if (blob) memcpy(blob, &b, sizeof b);
+  C.mp_exec = std::move(e);
+  return 0;
+}
+
+int stf_mp_import(const void* blobs) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (!C.mp_exec) return fail(-100, "stf_mp_import: call stf_mp_prepare first");
+  Exec& X = *C.mp_exec;
+  const MpBlob* B = static_cast<const MpBlob*>(blobs);
+  for (int s = 0; s < X.ngpus; ++s) {
+    if (B[s].magic != kMpMagic || B[s].slot != s) return fail(-4, "blob %d is not slot %d's", s, s);
+    if (s == C.mp_me || B[s].count == 0) continue;
+    void *pa = nullptr, *pf = nullptr;
+    CUDA_TRY(cudaIpcOpenMemHandle(&pa, B[s].arena, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle(arena)");
+    X.ipc_opened.push_back(pa);
+    CUDA_TRY(cudaIpcOpenMemHandle(&pf, B[s].flags, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle(flags)");
+    X.ipc_opened.push_back(pf);
+    X.peer_arena[(size_t)s] = static_cast<double*>(pa);
+    X.peer_flags[(size_t)s] = static_cast<uint32_t*>(pf);
+  }
+  for (size_t b = 0; b < X.plan.buffers.size(); ++b) {
+    const stf::Buffer& Bf = X.plan.buffers[b];
+    if (Bf.replica && Bf.slot != C.mp_me) X.buf[b] = X.peer_arena[(size_t)Bf.slot] + X.rep_off[b];
+  }
+  return 0;
+}
+
+int stf_mp_potrf(void) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  g_err.clear();
+  if (!C.mp_exec) return fail(-100, "stf_mp_potrf: call stf_mp_prepare / stf_mp_import first");
+  int info = run(C, *C.mp_exec);
+  fill_stats(*C.mp_exec, false, &C.last);
+  C.last.device_ms = C.device_ms;
+  return info;
 }
 
 int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double* avg_ms) {

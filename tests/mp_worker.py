@@ -1,0 +1,73 @@
+"""Multi-process worker (one process per GPU slot), launched by torchrun from
+tests/test_gpu_mp.py.  Each rank owns slot `rank` of a p x q grid, holds only
+its own tiles and runs only its own tasks (stf_mp_*); tiles cross processes
+through CUDA IPC replicas + device-side flags.  Rank 0 then re-factors the same
+matrix in single-process mode with virtual slots and checks bit equality.
+
+argv: n nb p q [push] [reps]
+"""
+import os
+import sys
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_sc_augonnetasg24_b200 as stf  # noqa: E402
+
+
+def main():
+    n, nb, p, q = (int(a) for a in sys.argv[1:5])
+    push = int(sys.argv[5]) if len(sys.argv) > 5 else 0
+    reps = int(sys.argv[6]) if len(sys.argv) > 6 else 2
+    dist.init_process_group("gloo")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    assert world == p * q
+    dev = int(os.environ.get("STF_MP_DEVICE", "0"))
+    torch.cuda.set_device(dev)
+    seed = 20240917
+    stf.mp_init(rank, world, dev)
+    stf.set_option("push", push)
+    A = stf.MpTiledMatrix(n, nb, p, q, rank, dev)
+    blob = A.prepare()
+    blobs = [None] * world
+    dist.all_gather_object(blobs, blob)
+    A.import_blobs(blobs)
+    infos, times = [], []
+    for _ in range(reps):  # re-run the same plan: epochs advance, flags stay valid
+        A.fill_spd(seed)
+        torch.cuda.synchronize()
+        dist.barrier()
+        infos.append(A.potrf())
+        times.append(stf.last_stats()["device_ms"])
+        dist.barrier()
+    mine = {ij: t.T.cpu().numpy().copy() for ij, t in A.tiles.items()}
+    allt = [None] * world
+    dist.all_gather_object(allt, (mine, infos, times))
+    dist.barrier()
+    stf.finalize()
+    if rank == 0:
+        stf.init(world, [dev] * world)
+        stf.set_option("push", push)
+        R = stf.TiledMatrix(n, nb, p, q, devices=[dev] * world)
+        R.fill_spd(seed)
+        info_ref = R.potrf()
+        stf.finalize()
+        bad = 0
+        for (m, inf, _tm) in allt:
+            assert all(i == info_ref for i in inf), (inf, info_ref)
+            for (i, j), blk in m.items():
+                ref = R.tiles[(i, j)].T.cpu().numpy()
+                if not np.array_equal(blk, ref):
+                    bad += 1
+        ntiles = sum(len(m) for m, _, _ in allt)
+        assert ntiles == (n // nb) * (n // nb + 1) // 2
+        print("MP_RESULT world=%d tiles=%d mismatched=%d info=%d ms=%s" %
+              (world, ntiles, bad, info_ref, [round(x, 3) for _, _, t in allt for x in t]))
+        assert bad == 0
+    dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,36 @@
+"""Multi-process mode (one process per GPU, include/stf_cholesky.h stf_mp_*):
+p*q processes each own one slot of the block-cyclic grid, hold only their own
+tiles and run only their own tasks; finished tiles reach consumer processes as
+CUDA-IPC replicas with device-side flag hand-off.  The box
+has one GPU, so all ranks share cuda:0 -- the IPC/flag protocol is the same as
+across NVLink peers.  Checked: bit equality with the single-process run of the
+same plan (virtual slots), info, and two back-to-back runs of one plan."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _run(n, nb, p, q, push=0, reps=2, port=29611):
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % (p * q),
+           "--master-addr", "127.0.0.1", "--master-port", str(port),
+           os.path.join(ROOT, "tests", "mp_worker.py"), str(n), str(nb), str(p), str(q), str(push), str(reps)]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-3000:]
+    line = [l for l in out.stdout.splitlines() if l.startswith("MP_RESULT")]
+    assert line and "mismatched=0" in line[0], out.stdout[-2000:]
+    return line[0]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("p,q,push,port", [(1, 2, 0, 29611), (2, 2, 0, 29621), (2, 2, 1, 29631), (2, 1, 1, 29641)])
+def test_multiprocess_bit_equal_to_single_process(p, q, push, port):
+    print(_run(1536, 128, p, q, push=push, port=port))
+
+
+@pytest.mark.gpu
+def test_multiprocess_large_tile():
+    print(_run(2048, 512, 2, 2, push=1, reps=2, port=29651))
