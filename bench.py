@@ -2,10 +2,15 @@
 """Benchmark: FP64 Cholesky GFLOP/s (n^3/3) of the STF tiled factorisation.
 
 Contract (driver): `python bench.py --gpus N --steps K --warmup W` prints ONE
-JSON line on rank 0.  Under torchrun (N > 1) every rank joins the barriers; the
-library is single-process multi-GPU by design (north_star's
-`stf_potrf(..., ngpus)`), so rank 0 drives all N GPUs and the other ranks
-contribute 0 device time to the max-over-ranks.
+JSON line on rank 0.  Under torchrun (N > 1) the default is the library's
+multi-process mode (--mode mp, include/stf_cholesky.h stf_mp_*): one process per
+GPU, rank r owns slot r of the block-cyclic grid, holds only its own tiles and
+runs only its own tasks (one CUDA graph per process); tiles reach consumer
+processes through CUDA-IPC replicas with device-side flag hand-off.  Each rank
+times its own graph with CUDA events; the step time is the max over ranks.
+--mode single keeps the paper's single-process multi-GPU call (PAPER.md:447,
+north_star's `stf_potrf(..., ngpus)`): rank 0 drives all N GPUs and the other
+ranks contribute 0 device time to the max-over-ranks.
 
 One step = one synchronous stf_potrf of the whole matrix (every §8(a) row: DAG,
 placement, replica pushes, POTRF/TRSM/SYRK/GEMM kernels, completion) on
@@ -174,11 +179,18 @@ def run_ours(args, rank, world):
 
     dist_on = world > 1
     if dist_on:
-        dist.init_process_group("nccl" if torch.cuda.is_available() else "gloo")
-        torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+        # NCCL needs one GPU per rank; virtual slots (all ranks on cuda:0) use gloo
+        nccl = torch.cuda.is_available() and not args.virtual
+        dist.init_process_group("nccl" if nccl else "gloo")
+        if torch.cuda.is_available():
+            torch.cuda.set_device(0 if args.virtual else int(os.environ.get("LOCAL_RANK", "0")))
     N = args.gpus
     n, nb = args.n, args.nb
     P, Q = grid_for(N)
+    mode = args.mode or ("mp" if dist_on else "single")
+    if mode == "mp":
+        assert dist_on and world == N, "--mode mp needs torchrun with one rank per GPU"
+        return run_mp(args, rank, world, P, Q)
     result = None
     total_ms = 0.0
     if rank == 0:
@@ -223,6 +235,75 @@ def run_ours(args, rank, world):
             dist.destroy_process_group()
         return 0
 
+    report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "single", args.steps * stats["kernel_launches"])
+    stf.finalize()
+    if dist_on:
+        dist.destroy_process_group()
+    return 0
+
+
+def run_mp(args, rank, world, P, Q):
+    """--mode mp: one process per GPU (stf_mp_*), max over ranks of each rank's device time."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_augonnetasg24_b200 as stf
+
+    N, n, nb = world, args.n, args.nb
+    dev = 0 if args.virtual else int(os.environ.get("LOCAL_RANK", rank))
+    torch.cuda.set_device(dev)
+    stf.mp_init(rank, world, dev)
+    A = stf.MpTiledMatrix(n, nb, P, Q, rank, dev)
+    blob = A.prepare()
+    blobs = [None] * world
+    dist.all_gather_object(blobs, blob)
+    A.import_blobs(blobs)
+
+    def step():
+        A.fill_spd(1)  # untimed regeneration of this rank's tiles
+        torch.cuda.synchronize(dev)
+        dist.barrier()
+        info = A.potrf()
+        assert info == 0 or os.environ.get("STF_DEBUG_SKIP"), info
+        ms = stf.last_stats()["device_ms"]
+        dist.barrier()
+        return ms
+
+    t0 = time.perf_counter()
+    step()
+    first_ms = 1000 * (time.perf_counter() - t0)
+    for _ in range(args.warmup - 1):
+        step()
+    clocks = ClockSampler()
+    if rank == 0:
+        clocks.start()
+    mine = [step() for _ in range(args.steps)]
+    clk = clocks.stop() if rank == 0 else None
+    stats = stf.last_stats()
+    steps_ms = [max_over_ranks(x, True) for x in mine]  # per step: the slowest rank
+    total_ms = sum(steps_ms)
+    launches = torch.tensor([float(stats["kernel_launches"])], dtype=torch.float64,
+                            device="cuda" if dist.get_backend() == "nccl" else "cpu")
+    dist.all_reduce(launches)
+    nodes = [None] * world
+    dist.all_gather_object(nodes, stats["graph_nodes"])
+    stf.finalize()
+    dist.barrier()
+    if rank == 0:
+        # e2e and kernels-alone numbers through the single-process API on all N GPUs
+        devices = list(range(N)) if args.virtual == 0 else [0] * N
+        stf.init(N, devices)
+        stats = dict(stats, graph_nodes=sum(nodes), kernel_launches=int(launches.item()))
+        report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "mp", args.steps * int(launches.item()))
+        stf.finalize()
+    dist.barrier()
+    dist.destroy_process_group()
+    return 0
+
+
+def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, gpu_launches):
+    import torch
+
+    n, nb = args.n, args.nb
     flops = n ** 3 / 3.0
     value = flops * args.steps / (total_ms * 1e-3) / 1e9
     ms_per_step = total_ms / args.steps
@@ -234,8 +315,9 @@ def run_ours(args, rank, world):
 
     # ---- roofline: the factorisation is one graph launch on the library's launch stream
     achieved_tf = value / 1e3
-    roof = {"bound": "tensor", "achieved": round(achieved_tf, 3), "peak": FP64_PEAK_TFLOPS * N, "unit": "TFLOP/s",
-            "frac": round(achieved_tf / (FP64_PEAK_TFLOPS * N), 4), "traffic": None,
+    ndev = 1 if args.virtual else N  # virtual slots share one GPU's tensor cores
+    roof = {"bound": "tensor", "achieved": round(achieved_tf, 3), "peak": FP64_PEAK_TFLOPS * ndev, "unit": "TFLOP/s",
+            "frac": round(achieved_tf / (FP64_PEAK_TFLOPS * ndev), 4), "traffic": None,
             "kernel": "whole-DAG CUDA graph launch (n^3/3 flop per launch, %d kernels inside)" % stats["kernel_launches"],
             "peak_src": FP64_PEAK_SRC}
     # dominant kernel (GEMM tile update) timed alone on its own stream at this nb and at full occupancy
@@ -283,8 +365,10 @@ def run_ours(args, rank, world):
                    "l2": "inputs larger than L2 (%.1f GB of tiles) and regenerated before every step" %
                          (n // nb * (n // nb + 1) / 2 * nb * nb * 8 / 1e9),
                    "graph": stf.get_option("graph"), "streams": stf.get_option("streams"),
-                   "virtual_slots": bool(args.virtual)},
-        "gpu_launches": int(stats["kernel_launches"]) * args.steps,
+                   "virtual_slots": bool(args.virtual),
+                   "processes": ("one per GPU (stf_mp_*, CUDA-IPC replicas, device-side flags)" if mode == "mp"
+                                 else "one process drives all %d GPU(s) (stf_potrf)" % N)},
+        "gpu_launches": int(gpu_launches),
         "clocks": clk,
         "roofline": roof,
         "cpu_baseline": cpu,
@@ -294,10 +378,6 @@ def run_ours(args, rank, world):
         "step_ms": [round(x, 3) for x in steps_ms],
     }
     print(json.dumps(line), flush=True)
-    stf.finalize()
-    if dist_on:
-        dist.destroy_process_group()
-    return 0
 
 
 def e2e_run(stf, n, nb, N, args):
@@ -351,9 +431,11 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=32768)
-    ap.add_argument("--nb", type=int, default=1024)
-    ap.add_argument("--virtual", type=int, default=0, help="map all slots onto cuda:0")
+    ap.add_argument("--n", "--order", dest="n", type=int, default=32768)
+    ap.add_argument("--nb", "--tile", dest="nb", type=int, default=1024)
+    ap.add_argument("--virtual-slots", dest="virtual", type=int, default=0, help="map all slots onto cuda:0")
+    ap.add_argument("--mode", default=None, choices=["single", "mp"],
+                    help="N>1: mp = one process per GPU (default under torchrun), single = rank 0 drives all GPUs")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")

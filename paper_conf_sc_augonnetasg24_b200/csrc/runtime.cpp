@@ -134,7 +134,7 @@ struct Exec {
   std::vector<double*> peer_arena;    // per slot, IPC-mapped (null for self / no replicas)
   std::vector<uint32_t*> peer_flags;  // per slot, IPC-mapped
   std::vector<void*> ipc_opened;      // to cudaIpcCloseMemHandle
-  uint32_t epoch = 0;
+  uint32_t epoch = 1;  // multi-process: value a published replica flag carries (reset to 0 at run end)
 
   ~Exec() {
     for (void* p : ipc_opened) cudaIpcCloseMemHandle(p);
@@ -473,6 +473,18 @@ int fork_streams(Context& C, int ngpus) {
   return 0;
 }
 
+// Multi-process mode: once every local task is done (after the join), all of
+// this process's replica flags have been consumed; clear them for the next
+// run.  Producers cannot publish the next run's tiles before the caller's
+// barrier that follows stf_mp_potrf, so one constant flag value serves every
+// run and the whole run (waits, writes, reset) can live in one CUDA graph.
+int mp_reset_flags(Context& C, Exec& X) {
+  if (!X.mp || !X.local_flag_count) return 0;
+  cudaSetDevice(C.origin_dev);
+  CUDA_TRY(cudaMemsetAsync(X.local_flags, 0, X.local_flag_count * sizeof(uint32_t), C.origin), "flag reset");
+  return 0;
+}
+
 int join_streams(Context& C, int ngpus) {
   for (int s = 0; s < ngpus; ++s) {
     Slot& S = C.slots[(size_t)s];
@@ -500,6 +512,48 @@ int alloc_on(Exec& X, int dev, size_t bytes, double** out) {
 }
 
 // Build plan + buffers + events (+ graph) for X (key fields already set).
+// Capture the whole DAG.  A capture the driver rejects (e.g. a multi-device
+// topology it cannot express) falls back to the eager stream backend for this
+// plan: same tasks, same edges, same results.
+int capture_graph(Context& C, Exec& X) {
+  cudaSetDevice(C.origin_dev);
+  int r = 0;
+  cudaGraph_t g = nullptr;
+  cudaError_t e = cudaStreamBeginCapture(C.origin, cudaStreamCaptureModeThreadLocal);
+  if (e == cudaSuccess) {
+    r = fork_streams(C, X.ngpus);
+    Lowerer L{C, X};
+    if (!r) r = L.issue();
+    if (!r) r = join_streams(C, X.ngpus);
+    if (!r) r = mp_reset_flags(C, X);
+    cudaSetDevice(C.origin_dev);
+    e = cudaStreamEndCapture(C.origin, &g);
+  }
+  if (r == 0 && e == cudaSuccess && g) {
+    e = cudaGraphInstantiateWithFlags(&X.gexec, g, cudaGraphInstantiateFlagUseNodePriority);
+    if (e == cudaSuccess) {
+      X.graph = g;
+      size_t nn = 0;
+      cudaGraphGetNodes(g, nullptr, &nn);
+      X.graph_nodes = (int64_t)nn;
+    }
+  }
+  if (!X.gexec) {
+    if (g) cudaGraphDestroy(g);
+    if (r == -103) return r;  // out of memory is not a capture problem
+    cudaGetLastError();
+    for (int d : C.devices) {  // drain anything a partial capture may have left behind
+      cudaSetDevice(d);
+      cudaDeviceSynchronize();
+    }
+    cudaGetLastError();
+    g_err.clear();
+    X.opt.graph = 0;
+    X.graph_fallback = 1;
+  }
+  return 0;
+}
+
 int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   auto t0 = std::chrono::steady_clock::now();
   const int64_t T = X.n / X.nb;
@@ -615,44 +669,9 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
       X.events_dev[t] = dev;
     }
   }
-  if (X.opt.graph) {
-    // Capture the whole DAG.  A capture the driver rejects (e.g. a multi-device
-    // topology it cannot express) falls back to the eager stream backend for
-    // this plan: same tasks, same edges, same results.
-    cudaSetDevice(C.origin_dev);
-    int r = 0;
-    cudaGraph_t g = nullptr;
-    cudaError_t e = cudaStreamBeginCapture(C.origin, cudaStreamCaptureModeThreadLocal);
-    if (e == cudaSuccess) {
-      r = fork_streams(C, X.ngpus);
-      Lowerer L{C, X};
-      if (!r) r = L.issue();
-      if (!r) r = join_streams(C, X.ngpus);
-      cudaSetDevice(C.origin_dev);
-      e = cudaStreamEndCapture(C.origin, &g);
-    }
-    if (r == 0 && e == cudaSuccess && g) {
-      e = cudaGraphInstantiateWithFlags(&X.gexec, g, cudaGraphInstantiateFlagUseNodePriority);
-      if (e == cudaSuccess) {
-        X.graph = g;
-        size_t nn = 0;
-        cudaGraphGetNodes(g, nullptr, &nn);
-        X.graph_nodes = (int64_t)nn;
-      }
-    }
-    if (!X.gexec) {
-      if (g) cudaGraphDestroy(g);
-      if (r == -103) return r;  // out of memory is not a capture problem
-      cudaGetLastError();
-      for (int d : C.devices) {  // drain anything a partial capture may have left behind
-        cudaSetDevice(d);
-        cudaDeviceSynchronize();
-      }
-      cudaGetLastError();
-      g_err.clear();
-      X.opt.graph = 0;
-      X.graph_fallback = 1;
-    }
+  if (X.opt.graph && !X.mp) {  // multi-process: captured by stf_mp_import, once peer replicas are mapped
+    int r = capture_graph(C, X);
+    if (r) return r;
   }
   X.build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return 0;
@@ -682,6 +701,7 @@ int rebind(Context& C, Exec& X, const stf_matrix_desc* desc, const std::vector<u
     Lowerer L{C, X};
     if (!r) r = L.issue();
     if (!r) r = join_streams(C, X.ngpus);
+    if (!r) r = mp_reset_flags(C, X);
     cudaSetDevice(C.origin_dev);
     cudaGraph_t g = nullptr;
     cudaError_t e = cudaStreamEndCapture(C.origin, &g);
@@ -707,7 +727,6 @@ int rebind(Context& C, Exec& X, const stf_matrix_desc* desc, const std::vector<u
 }
 
 int run(Context& C, Exec& X) {
-  if (X.mp) X.epoch++;  // flags are monotonic: run e waits for value >= e
   cudaSetDevice(C.origin_dev);
   CUDA_TRY(cudaEventRecord(C.t_start, C.origin), "timing start");
   if (X.opt.graph) {
@@ -717,6 +736,7 @@ int run(Context& C, Exec& X) {
     Lowerer L{C, X};
     if (!r) r = L.issue();
     if (!r) r = join_streams(C, X.ngpus);
+    if (!r) r = mp_reset_flags(C, X);
     if (r) return r;
   }
   cudaSetDevice(C.origin_dev);
@@ -1367,7 +1387,7 @@ int stf_mp_prepare(int64_t n, int64_t nb, const stf_matrix_desc* A_desc, void* b
   e->P = P;
   e->Q = Q;
   e->opt = C.opt;
-  e->opt.graph = 0;  // eager, multi-threaded submission is not needed: one slot per process
+  e->opt.threads = 1;  // one slot per process: one submission thread
   e->mp = true;
   int r = prepare(C, *e, A_desc);
   if (r) return r;
@@ -1406,6 +1426,7 @@ int stf_mp_import(const void* blobs) {
     const stf::Buffer& Bf = X.plan.buffers[b];
     if (Bf.replica && Bf.slot != C.mp_me) X.buf[b] = X.peer_arena[(size_t)Bf.slot] + X.rep_off[b];
   }
+  if (X.opt.graph) return capture_graph(C, X);
   return 0;
 }
 

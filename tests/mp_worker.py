@@ -4,7 +4,7 @@ its own tiles and runs only its own tasks (stf_mp_*); tiles cross processes
 through CUDA IPC replicas + device-side flags.  Rank 0 then re-factors the same
 matrix in single-process mode with virtual slots and checks bit equality.
 
-argv: n nb p q [push] [reps]
+argv: n nb p q [push] [reps] [graph]
 """
 import os
 import sys
@@ -21,6 +21,7 @@ def main():
     n, nb, p, q = (int(a) for a in sys.argv[1:5])
     push = int(sys.argv[5]) if len(sys.argv) > 5 else 0
     reps = int(sys.argv[6]) if len(sys.argv) > 6 else 2
+    graph = int(sys.argv[7]) if len(sys.argv) > 7 else 1
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
     assert world == p * q
@@ -29,22 +30,24 @@ def main():
     seed = 20240917
     stf.mp_init(rank, world, dev)
     stf.set_option("push", push)
+    stf.set_option("graph", graph)
     A = stf.MpTiledMatrix(n, nb, p, q, rank, dev)
     blob = A.prepare()
     blobs = [None] * world
     dist.all_gather_object(blobs, blob)
     A.import_blobs(blobs)
     infos, times = [], []
-    for _ in range(reps):  # re-run the same plan: epochs advance, flags stay valid
+    for _ in range(reps):  # re-run the same plan: each run clears its flags at the end
         A.fill_spd(seed)
         torch.cuda.synchronize()
         dist.barrier()
         infos.append(A.potrf())
-        times.append(stf.last_stats()["device_ms"])
+        st = stf.last_stats()
+        times.append(st["device_ms"])
         dist.barrier()
     mine = {ij: t.T.cpu().numpy().copy() for ij, t in A.tiles.items()}
     allt = [None] * world
-    dist.all_gather_object(allt, (mine, infos, times))
+    dist.all_gather_object(allt, (mine, infos, times, st["graph_nodes"]))
     dist.barrier()
     stf.finalize()
     if rank == 0:
@@ -55,16 +58,16 @@ def main():
         info_ref = R.potrf()
         stf.finalize()
         bad = 0
-        for (m, inf, _tm) in allt:
+        for (m, inf, _tm, _g) in allt:
             assert all(i == info_ref for i in inf), (inf, info_ref)
             for (i, j), blk in m.items():
                 ref = R.tiles[(i, j)].T.cpu().numpy()
                 if not np.array_equal(blk, ref):
                     bad += 1
-        ntiles = sum(len(m) for m, _, _ in allt)
+        ntiles = sum(len(m) for m, _, _, _ in allt)
         assert ntiles == (n // nb) * (n // nb + 1) // 2
-        print("MP_RESULT world=%d tiles=%d mismatched=%d info=%d ms=%s" %
-              (world, ntiles, bad, info_ref, [round(x, 3) for _, _, t in allt for x in t]))
+        print("MP_RESULT world=%d tiles=%d mismatched=%d info=%d graph_nodes=%s ms=%s" %
+              (world, ntiles, bad, info_ref, [g for _, _, _, g in allt], [round(x, 3) for _, _, t, _ in allt for x in t]))
         assert bad == 0
     dist.destroy_process_group()
 
