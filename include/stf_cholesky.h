@@ -113,6 +113,13 @@ const char *stf_last_error(void);
  *                           (default 8, capped at ngpus; the graph backend captures on one thread)
  *   "lookahead" STF_LOOKAHEAD 1: pure STF DAG (default); 0: a fence task closes every
  *                           panel step (no look-ahead; ablation of PAPER.md:399)
+ *   "mem_cap_tiles" STF_MEM_CAP_TILES  0 (default) or >= 3: a HOST_COLMAJOR call on one GPU
+ *                           keeps at most this many nb x nb tiles on the device (out-of-core,
+ *                           NEXT-4): tiles are loaded on demand and dirty
+ *                           tiles written back on eviction (Belady order, left-looking
+ *                           super-columns).  A cap >= T(T+1)/2 tiles means no cap.  Rejected
+ *                           (-105) for HOST_COLMAJOR calls on more than one GPU; ignored for
+ *                           device-resident kinds, whose matrix is on the device already.
  * Returns 0 or -105. */
 int stf_set_option(const char *name, int64_t value);
 int stf_get_option(const char *name, int64_t *value);
@@ -135,6 +142,9 @@ typedef struct stf_plan_stats {
   int64_t graph_reuse;    /* 0 new plan, 1 exact memo hit, 2 plan of the same shape re-bound
                              to new caller storage (graph refreshed by cudaGraphExecUpdate) */
   int64_t dag_tasks;      /* all DAG vertices: compute + COPY + LOAD/STORE + FENCE tasks */
+  int64_t host_loads;     /* LOAD tasks: tiles copied from the caller's matrix (COLMAJOR kinds) */
+  int64_t host_stores;    /* STORE tasks: tiles written back to the caller's matrix */
+  int64_t frames;         /* device tile frames of an out-of-core plan ("mem_cap_tiles"), else 0 */
 } stf_plan_stats;
 
 int stf_last_stats(stf_plan_stats *out);
@@ -142,12 +152,21 @@ int stf_last_stats(stf_plan_stats *out);
 /* Build (without running) the STF DAG of a T x T tile Cholesky on a p x q grid
  * and copy up to `cap` edges (src, dst pairs of task indices in submission
  * order) into edges[2*cap].  kinds[cap_tasks] receives per-task codes
- * (0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM, 4 COPY, 7 FENCE) and ijk[3*cap_tasks] the (i, j, k)
- * indices (for COPY: tile i, j and destination slot k).  Any output pointer
- * may be NULL.  Fills *stats.  Uses the current "push" and "lookahead" options.
+ * (0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM, 4 COPY, 5 LOAD, 6 STORE, 7 FENCE) and ijk[3*cap_tasks]
+ * the (i, j, k) indices (for COPY: tile i, j and destination slot k).  Any output pointer
+ * may be NULL.  Fills *stats.  Uses the current "push", "lookahead" and "mem_cap_tiles"
+ * options (the latter, for p = q = 1: the out-of-core plan of a HOST_COLMAJOR call).
  * Needs no GPU. */
 int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t *edges, int64_t cap_tasks, int32_t *kinds,
                   int64_t *ijk, stf_plan_stats *stats);
+
+/* Buffers of the tasks of the last stf_dag_build on this thread: io[3*t] and
+ * io[3*t+1] = buffer ids read (-1 unused), io[3*t+2] = buffer written (-1 for
+ * STORE/FENCE).  Buffers: home tiles 0..T(T+1)/2-1 (tile (i,j) -> i(i+1)/2 + j)
+ * then replicas; in an out-of-core plan the device frames 0..frames-1 (LOAD
+ * writes a frame from the caller's tile (i, j), STORE reads one).  Returns the
+ * number of buffers.  Needs no GPU. */
+int stf_dag_tasks_io(int64_t cap_tasks, int64_t *io);
 
 /* Generic STF rule on an arbitrary access list (the Algorithm 1 example):
  * ntasks tasks, task t has nacc[t] accesses listed consecutively in data[] and

@@ -68,6 +68,14 @@ def dag(T: int, p: int = 1, q: int = 1):
     return edges, kinds, ijk, st.as_dict()
 
 
+def dag_io(ntasks: int):
+    """(buffers read, buffer written) of every task of the last dag() call, and
+    the number of buffers (home tiles + replicas, or device frames out of core)."""
+    IO = (ctypes.c_int64 * (3 * max(1, ntasks)))()
+    nbuf = check(_abi.stf_dag_tasks_io(ntasks, IO), "stf_dag_tasks_io")
+    return [((IO[3 * t], IO[3 * t + 1]), IO[3 * t + 2]) for t in range(ntasks)], nbuf
+
+
 def infer_edges(tasks: Sequence[Sequence[tuple]]) -> set:
     """Generic STF rule (C++ core) on [[(datum:int, mode:'r'|'w'|'rw'), ...], ...]."""
     mode_code = {"r": 1, "w": 2, "rw": 3}

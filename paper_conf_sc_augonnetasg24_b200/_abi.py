@@ -44,6 +44,9 @@ class stf_plan_stats(ctypes.Structure):
         ("device_ms", ctypes.c_double),
         ("graph_reuse", ctypes.c_int64),
         ("dag_tasks", ctypes.c_int64),
+        ("host_loads", ctypes.c_int64),
+        ("host_stores", ctypes.c_int64),
+        ("frames", ctypes.c_int64),
     ]
 
     def as_dict(self):
@@ -56,7 +59,7 @@ EXPORTS = [
     "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_infer_edges",
     "stf_fill_spd_tiles", "stf_fill_spd_block",
     "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace",
-    "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
+    "stf_dag_tasks_io", "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
 ]
 
 if not os.path.exists(LIB_PATH):
@@ -93,6 +96,7 @@ stf_kernel_gemm_nt = _decl("stf_kernel_gemm_nt", _int, [_i64, _i64, _i64, _vp, _
 stf_kernel_trsm = _decl("stf_kernel_trsm", _int, [_i64, _i64, _vp, _i64, _vp, _i64])
 stf_kernel_potrf = _decl("stf_kernel_potrf", _int, [_i64, _vp, _i64, _P(_i64)])
 stf_bench_kernel = _decl("stf_bench_kernel", _int, [_int, _i64, _i64, _i64, _int, _P(_dbl)])
+stf_dag_tasks_io = _decl("stf_dag_tasks_io", _int, [_i64, _P(_i64)])
 stf_mp_init = _decl("stf_mp_init", _int, [_int, _int, _int])
 stf_mp_blob_size = _decl("stf_mp_blob_size", _i64, [])
 stf_mp_prepare = _decl("stf_mp_prepare", _int, [_i64, _i64, _P(stf_matrix_desc), _vp])

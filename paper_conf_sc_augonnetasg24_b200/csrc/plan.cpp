@@ -2,6 +2,9 @@
 #include "plan.hpp"
 
 #include <algorithm>
+#include <climits>
+#include <set>
+#include <utility>
 #include <vector>
 
 namespace stf {
@@ -135,6 +138,7 @@ struct Builder {
           Task t{K_LOAD, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own), {-1, -1}, w};
           Access acc[1] = {{w, WRITE}};
           submit(t, acc, 1);
+          p.nloads++;
           version[(size_t)w]++;
         }
     }
@@ -174,11 +178,181 @@ struct Builder {
           Task t{K_STORE, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own), {d, -1}, -1};
           Access acc[1] = {{d, READ}};
           submit(t, acc, 1);
+          p.nstores++;
         }
     }
   }
 };
 
+}  // namespace
+
+// ------------------------------------------------------------------ NEXT-4
+// Memory-capped (out-of-core) plan: the matrix stays in the
+// caller's host memory and only `F` device tile frames exist.  The STF rule
+// does all the synchronisation: each frame is a logical datum (a compute task
+// accesses the frame holding its tile with the tile's mode), each host tile is
+// another one; LOAD(tile -> frame f) reads the host tile and writes frame f,
+// STORE(frame f -> tile) reads frame f and writes the host tile.  Reusing a
+// frame therefore waits for the previous occupant's readers (WAR) and writer
+// (WAW), and a reload waits for the eviction's write-back (RAW).
+//
+// Program order.  Any order in which every task follows the tasks whose
+// outputs it reads gives the same DAG up to frame edges and bit-identical
+// results (each tile still receives its updates k = 0, 1, ... in order).  For
+// traffic the plan uses a left-looking super-column order: columns are taken
+// in blocks [j0, j1] whose tiles fit in about half of the frames; the block
+// first receives all updates from columns k < j0 (k outer, so each panel tile
+// L_ik is loaded once per block), then is factored right-looking inside.
+// Each tile is written back once; reads of earlier panels cost about
+// 8 nb^2 bytes per w*2 nb^3 flops for a block of width w.
+// Eviction is Belady's (furthest next use in program order), never a frame the
+// current task uses.
+namespace {
+struct OocBuilder {
+  Plan& p;
+  const int64_t T;
+  const int64_t F;
+  struct CT {
+    int32_t kind, i, j, k, prio;
+    int64_t r0, r1, w;  // tile ids read (or -1) and written
+  };
+  std::vector<CT> seq;
+
+  OocBuilder(Plan& plan, int64_t T_, int64_t F_) : p(plan), T(T_), F(F_) {}
+
+  int64_t id(int64_t i, int64_t j) const { return Plan::tile_id(i, j); }
+
+  void emit_updates_from(int64_t k, int64_t j0, int64_t j1) {
+    for (int64_t j = j0; j <= j1; ++j) {
+      seq.push_back({K_SYRK, (int32_t)j, (int32_t)j, (int32_t)k, 2, id(j, k), -1, id(j, j)});
+      for (int64_t i = j + 1; i < T; ++i)
+        seq.push_back({K_GEMM, (int32_t)i, (int32_t)j, (int32_t)k, 1, id(i, k), id(j, k), id(i, j)});
+    }
+  }
+
+  void make_sequence() {
+    int64_t j0 = 0;
+    while (j0 < T) {
+      // widest block whose tiles use at most half the frames (at least one column)
+      int64_t j1 = j0, used = T - j0;
+      while (j1 + 1 < T && used + (T - j1 - 1) <= F / 2) used += T - (++j1);
+      for (int64_t k = 0; k < j0; ++k) emit_updates_from(k, j0, j1);
+      for (int64_t j = j0; j <= j1; ++j) {
+        seq.push_back({K_POTRF, (int32_t)j, (int32_t)j, (int32_t)j, 5, -1, -1, id(j, j)});
+        for (int64_t i = j + 1; i < T; ++i)
+          seq.push_back({K_TRSM, (int32_t)i, (int32_t)j, (int32_t)j, i == j + 1 ? 5 : 4, id(j, j), -1, id(i, j)});
+        if (j < j1) emit_updates_from(j, j + 1, j1);
+      }
+      j0 = j1 + 1;
+    }
+  }
+
+  void run(int crit_streams, int bulk_streams, int load_stream, int store_stream, bool serial, bool priority) {
+    make_sequence();
+    const int64_t NT = p.ntiles();
+    p.buffers.clear();
+    for (int64_t f = 0; f < F; ++f) p.buffers.push_back(Buffer{-1, -1, 0, false});
+    auto host = [&](int64_t t) { return F + t; };  // datum id of the caller's copy of tile t
+    // next-use bookkeeping for Belady
+    std::vector<std::vector<int64_t>> uses((size_t)NT);
+    for (size_t q = 0; q < seq.size(); ++q)
+      for (int64_t t : {seq[q].r0, seq[q].r1, seq[q].w})
+        if (t >= 0) uses[(size_t)t].push_back((int64_t)q);
+    std::vector<size_t> ptr((size_t)NT, 0);
+    const int64_t kNever = INT64_MAX;
+    auto next_use = [&](int64_t t, int64_t after) -> int64_t {
+      auto& u = uses[(size_t)t];
+      size_t& k = ptr[(size_t)t];
+      while (k < u.size() && u[k] <= after) ++k;
+      return k < u.size() ? u[k] : kNever;
+    };
+    std::vector<int64_t> frame_of((size_t)NT, -1), tile_in((size_t)F, -1);
+    std::vector<char> dirty((size_t)F, 0);
+    std::set<std::pair<int64_t, int64_t>> resident;  // (next use, tile)
+    std::vector<int64_t> key((size_t)NT, 0);
+    std::vector<int64_t> free_frames;
+    for (int64_t f = F - 1; f >= 0; --f) free_frames.push_back(f);
+    int32_t ij[2];
+    auto tile_ij = [&](int64_t t) {
+      int64_t i = 0;
+      while ((i + 1) * (i + 2) / 2 <= t) ++i;
+      ij[0] = (int32_t)i;
+      ij[1] = (int32_t)(t - i * (i + 1) / 2);
+    };
+    auto store = [&](int64_t f) {
+      tile_ij(tile_in[(size_t)f]);
+      Task s{K_STORE, ij[0], ij[1], 0, 0, 0, store_stream, {f, -1}, -1};
+      Access acc[2] = {{f, READ}, {host(tile_in[(size_t)f]), WRITE}};
+      p.graph.submit(acc, 2);
+      p.tasks.push_back(s);
+      p.nstores++;
+      dirty[(size_t)f] = 0;
+    };
+    auto compute_stream = [&](const CT& c) -> int {
+      if (serial) return 0;
+      if (priority && c.prio >= 4) return c.kind == K_POTRF ? 0 : (int)(c.i % crit_streams);
+      return crit_streams + (int)((c.i * T + c.j) % bulk_streams);
+    };
+    for (size_t q = 0; q < seq.size(); ++q) {
+      const CT& c = seq[q];
+      const int64_t need[3] = {c.r0, c.r1, c.w};
+      for (int a = 0; a < 3; ++a) {
+        const int64_t t = need[a];
+        if (t < 0 || frame_of[(size_t)t] >= 0) continue;
+        int64_t f;
+        if (!free_frames.empty()) {
+          f = free_frames.back();
+          free_frames.pop_back();
+        } else {
+          // furthest next use among residents the current task does not touch
+          auto it = resident.end();
+          do {
+            --it;
+          } while (it->second == need[0] || it->second == need[1] || it->second == need[2]);
+          const int64_t v = it->second;
+          resident.erase(it);
+          f = frame_of[(size_t)v];
+          if (dirty[(size_t)f]) store(f);
+          frame_of[(size_t)v] = -1;
+          tile_in[(size_t)f] = -1;
+        }
+        tile_ij(t);
+        Task l{K_LOAD, ij[0], ij[1], 0, 0, priority ? c.prio : 0, load_stream, {-1, -1}, f};
+        Access acc[2] = {{host(t), READ}, {f, WRITE}};
+        p.graph.submit(acc, 2);
+        p.tasks.push_back(l);
+        p.nloads++;
+        frame_of[(size_t)t] = f;
+        tile_in[(size_t)f] = t;
+        key[(size_t)t] = -1;  // inserted below with its next use
+      }
+      // the task itself
+      Task t{c.kind, c.i, c.j, c.k, 0, priority ? c.prio : 0, 0,
+             {c.r0 >= 0 ? frame_of[(size_t)c.r0] : -1, c.r1 >= 0 ? frame_of[(size_t)c.r1] : -1},
+             frame_of[(size_t)c.w]};
+      t.stream = compute_stream(c);
+      Access acc[3];
+      int n = 0;
+      if (t.in[0] >= 0) acc[n++] = {t.in[0], READ};
+      if (t.in[1] >= 0) acc[n++] = {t.in[1], READ};
+      acc[n++] = {t.out, RW};
+      p.graph.submit(acc, n);
+      p.tasks.push_back(t);
+      dirty[(size_t)t.out] = 1;
+      // refresh the next-use keys of the tiles just used
+      for (int a = 0; a < 3; ++a) {
+        const int64_t x = need[a];
+        if (x < 0) continue;
+        if (key[(size_t)x] >= 0) resident.erase({key[(size_t)x], x});
+        key[(size_t)x] = next_use(x, (int64_t)q);
+        resident.insert({key[(size_t)x], x});
+      }
+    }
+    // write back what is still dirty
+    for (int64_t f = 0; f < F; ++f)
+      if (tile_in[(size_t)f] >= 0 && dirty[(size_t)f]) store(f);
+  }
+};
 }  // namespace
 
 void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
@@ -190,12 +364,24 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
   plan.tasks.clear();
   plan.ntransfers = 0;
   plan.npushed = 0;
+  plan.nloads = 0;
+  plan.nstores = 0;
   plan.replicas_per_slot.assign((size_t)opt.nslots, 0);
-  // dense datum ids: home tiles + at most one replica per (tile, slot)
   const int64_t NT = T * (T + 1) / 2;
-  plan.graph = TaskGraph(NT + NT * opt.nslots + 1);
-  Builder b(plan, T);
-  b.run();
+  if (opt.frames > 0 && opt.nslots == 1 && opt.with_load && opt.with_store) {
+    // out-of-core: datum ids = frames, then the caller's host tiles
+    plan.graph = TaskGraph(opt.frames + NT + 1);
+    const int base = plan.opt.serial ? 1 : plan.opt.crit_streams + plan.opt.bulk_streams;
+    OocBuilder b(plan, T, opt.frames);
+    b.run(plan.opt.crit_streams, plan.opt.bulk_streams, base, base + (plan.opt.copy_streams > 1 ? 1 : 0),
+          plan.opt.serial, plan.opt.priority);
+  } else {
+    plan.opt.frames = 0;
+    // dense datum ids: home tiles + at most one replica per (tile, slot)
+    plan.graph = TaskGraph(NT + NT * opt.nslots + 1);
+    Builder b(plan, T);
+    b.run();
+  }
   // longest chain of compute tasks (COPY/LOAD/STORE weigh 0)
   std::vector<int64_t> depth(plan.tasks.size(), 0);
   int64_t best = 0;

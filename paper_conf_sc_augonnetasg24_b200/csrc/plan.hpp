@@ -56,10 +56,14 @@ struct PlanOptions {
                            // step k+1 starts only when step k is complete (ablation, NEXT-1)
   bool push = false;       // TRSM(i,k) writes L_ik into its consumers' replicas itself (fused
                            // push, NEXT-3) instead of COPY tasks at the first remote read
+  int64_t frames = 0;      // > 0 (one slot, with_load/with_store): memory-capped out-of-core
+                           // plan (NEXT-4) over this many device tile frames; see plan.cpp
 };
 
 // A "buffer" is one physical nb x nb tile instance: home tiles are buffers
-// 0..NT-1 (lower tile (i,j) -> i*(i+1)/2 + j), replicas follow.
+// 0..NT-1 (lower tile (i,j) -> i*(i+1)/2 + j), replicas follow.  In an
+// out-of-core plan the buffers are the device frames instead (i = j = -1):
+// tiles move between the caller's host matrix and frames by LOAD/STORE tasks.
 struct Buffer {
   int32_t i, j, slot;
   bool replica;
@@ -73,6 +77,8 @@ struct Plan {
   TaskGraph graph;
   int64_t ntransfers = 0;     // COPY tasks
   int64_t npushed = 0;        // replicas written by fused push
+  int64_t nloads = 0;         // LOAD tasks (caller matrix -> device tile)
+  int64_t nstores = 0;        // STORE tasks (device tile -> caller matrix)
   int64_t critical_path = 0;  // longest chain counted in compute tasks
   std::vector<int64_t> replicas_per_slot;
 

@@ -41,6 +41,7 @@
 namespace {
 
 thread_local std::string g_err;
+thread_local stf::Plan g_dag_plan;  // the plan of the last stf_dag_build (stf_dag_tasks_io)
 
 int fail(int code, const char* fmt, ...) {
   char buf[512];
@@ -88,7 +89,15 @@ struct Options {
   int64_t lookahead = 1;
   int64_t threads = 8;  // eager backend: host submission threads (one per slot group)
   int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
+  int64_t mem_cap_tiles = 0;  // HOST_COLMAJOR on one GPU: device tile frames (0 = whole matrix resident)
 };
+
+// options that change the plan or its lowering (part of the memo key)
+bool same_plan_options(const Options& a, int64_t a_graph, const Options& b) {
+  return a.streams == b.streams && a.serial == b.serial && a_graph == b.graph && a.priority == b.priority &&
+         a.dataflow == b.dataflow && a.trsm == b.trsm && a.trsm_split == b.trsm_split && a.push == b.push &&
+         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles;
+}
 
 // A plan bound to physical buffers, plus its lowering artefacts.
 struct Exec {
@@ -558,7 +567,11 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   auto t0 = std::chrono::steady_clock::now();
   const int64_t T = X.n / X.nb;
   const bool colmajor = X.kind != STF_DESC_TILED_2DBC;
-  stf::build_plan(X.plan, T, plan_options(X.opt, X.P, X.Q, X.ngpus, colmajor, colmajor));
+  stf::PlanOptions po = plan_options(X.opt, X.P, X.Q, X.ngpus, colmajor, colmajor);
+  if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
+      X.opt.mem_cap_tiles < T * (T + 1) / 2)
+    po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames
+  stf::build_plan(X.plan, T, po);
   const stf::Plan& P = X.plan;
   const size_t tile_bytes = (size_t)(X.nb * X.nb) * sizeof(double);
   X.buf.assign(P.buffers.size(), nullptr);
@@ -771,6 +784,9 @@ void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
   s->build_ms = hit ? 0.0 : X.build_ms;
   s->graph_reuse = hit ? 1 : 0;
   s->dag_tasks = (int64_t)P.tasks.size();
+  s->host_loads = P.nloads;
+  s->host_stores = P.nstores;
+  s->frames = P.opt.frames;
 }
 
 int choose_grid(int ngpus, int64_t grid_p, int* P, int* Q) {
@@ -844,6 +860,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.trsm = env_int("STF_TRSM", 2);
   C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 4);
   C.opt.push = env_int("STF_PUSH", 0);
+  C.opt.mem_cap_tiles = env_int("STF_MEM_CAP_TILES", 0);
   C.opt.streams = env_int("STF_STREAMS", 8);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
@@ -972,6 +989,10 @@ int stf_set_option(const char* name, int64_t value) {
     C.opt.trsm_split = value;
   }
   else if (n == "push") C.opt.push = value != 0;
+  else if (n == "mem_cap_tiles") {
+    if (value != 0 && value < 3) return fail(-105, "mem_cap_tiles must be 0 (no cap) or >= 3 (a GEMM holds 3 tiles)");
+    C.opt.mem_cap_tiles = value;
+  }
   else if (n == "threads") {
     if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
     C.opt.threads = value;
@@ -998,6 +1019,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "lookahead") *value = C.opt.lookahead;
   else if (n == "trsm_split") *value = C.opt.trsm_split;
   else if (n == "push") *value = C.opt.push;
+  else if (n == "mem_cap_tiles") *value = C.opt.mem_cap_tiles;
   else if (n == "threads") *value = C.opt.threads;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;
@@ -1043,6 +1065,8 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     }
   }
   const int64_t T = n / nb;
+  if (A_desc->kind == STF_DESC_HOST_COLMAJOR && ngpus > 1 && C.opt.mem_cap_tiles > 0)
+    return fail(-105, "mem_cap_tiles (out-of-core) supports HOST_COLMAJOR calls on one GPU");
   // tile residency check (TILED_2DBC): every lower tile on its owner's device
   std::vector<uintptr_t> ptrs;
   if (A_desc->kind == STF_DESC_TILED_2DBC) {
@@ -1065,9 +1089,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
   for (auto it = C.cache.begin(); it != C.cache.end(); ++it) {
     Exec& e = **it;
     if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
-        e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial &&
-        e.key_graph == C.opt.graph &&
-        e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm && e.opt.trsm_split == C.opt.trsm_split && e.opt.push == C.opt.push && e.opt.lookahead == C.opt.lookahead && e.key_ptrs == ptrs &&
+        e.Q == Q && same_plan_options(e.opt, e.key_graph, C.opt) && e.key_ptrs == ptrs &&
         (A_desc->kind == STF_DESC_TILED_2DBC ||
          (e.mat == A_desc->ptr && e.key_ld == A_desc->ld && e.key_dev == A_desc->device))) {
       C.cache.splice(C.cache.begin(), C.cache, it);
@@ -1086,9 +1108,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
       Exec& e = **it;
       const bool pageable = A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr);
       if (e.n == n && e.nb == nb && e.uplo == up && e.kind == A_desc->kind && e.ngpus == ngpus && e.P == P &&
-          e.Q == Q && e.opt.streams == C.opt.streams && e.opt.serial == C.opt.serial && e.key_graph == C.opt.graph &&
-          e.opt.priority == C.opt.priority && e.opt.dataflow == C.opt.dataflow && e.opt.trsm == C.opt.trsm &&
-          e.opt.trsm_split == C.opt.trsm_split && e.opt.push == C.opt.push && e.opt.lookahead == C.opt.lookahead && (e.gexec == nullptr) == (e.opt.graph == 0) &&
+          e.Q == Q && same_plan_options(e.opt, e.key_graph, C.opt) && (e.gexec == nullptr) == (e.opt.graph == 0) &&
           !(pageable && e.gexec)) {
         int r = rebind(C, e, A_desc, ptrs);
         if (r) return r;
@@ -1162,6 +1182,17 @@ int stf_last_stats(stf_plan_stats* out) {
   return 0;
 }
 
+int stf_dag_tasks_io(int64_t cap_tasks, int64_t* io) {
+  g_err.clear();
+  const stf::Plan& plan = g_dag_plan;
+  for (size_t t = 0; t < plan.tasks.size() && (int64_t)t < cap_tasks; ++t) {
+    io[3 * t] = plan.tasks[t].in[0];
+    io[3 * t + 1] = plan.tasks[t].in[1];
+    io[3 * t + 2] = plan.tasks[t].out;
+  }
+  return (int)std::min<size_t>(plan.buffers.size(), INT_MAX);
+}
+
 int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t cap_tasks, int32_t* kinds,
                   int64_t* ijk, stf_plan_stats* stats) {
   g_err.clear();
@@ -1171,9 +1202,13 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
   o.priority = 1;
   o.push = ctx().opt.push;            // the DAG options the next stf_potrf would use
   o.lookahead = ctx().opt.lookahead;
-  stf::Plan plan;
+  stf::Plan& plan = g_dag_plan;
   auto t0 = std::chrono::steady_clock::now();
-  stf::build_plan(plan, T, plan_options(o, p, q, p * q, false, false));
+  // with "mem_cap_tiles" set and one slot: the out-of-core plan of a HOST_COLMAJOR call
+  const bool ooc = ctx().opt.mem_cap_tiles > 0 && p * q == 1 && ctx().opt.mem_cap_tiles < T * (T + 1) / 2;
+  stf::PlanOptions po = plan_options(o, p, q, p * q, ooc, ooc);
+  if (ooc) po.frames = ctx().opt.mem_cap_tiles;
+  stf::build_plan(plan, T, po);
   double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   int64_t e = 0;
   for (int64_t t = 0; t < plan.graph.ntasks(); ++t)
@@ -1204,6 +1239,9 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
     stats->device_ms = 0;
     stats->graph_reuse = 0;
     stats->dag_tasks = (int64_t)plan.tasks.size();
+    stats->host_loads = plan.nloads;
+    stats->host_stores = plan.nstores;
+    stats->frames = plan.opt.frames;
   }
   return 0;
 }

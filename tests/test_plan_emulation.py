@@ -1,0 +1,164 @@
+"""Execute the library's plans (the exact task list, buffers and DAG edges that
+stf_potrf lowers) on the CPU with the oracle's tile operations, in RANDOM
+topological orders of the DAG.  An edge the plan is missing -- a replica read
+before its COPY, a frame reloaded while a reader still needs the old tile, a
+reload before the write-back -- lets some order read a wrong tile, and the
+result leaves oracle.tiled_potrf's bits.  Since every tile still receives its
+updates k = 0, 1, ... in order, the result must equal oracle.tiled_potrf
+bit for bit.  Integer/ordering work: exact comparison.  No GPU needed.
+
+Covers the 2D block-cyclic plans with replicas (§8 rows a3/a5/a7), the
+fence ablation (NEXT-1) and the out-of-core plans over F device frames with
+LOAD/STORE tasks (NEXT-4)."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_augonnetasg24_b200 as stf
+import synth
+
+NB = 4  # tile order for the emulation (values are irrelevant to the schedule)
+
+
+def _plan(T, p, q, frames=0, lookahead=1):
+    stf.set_option("mem_cap_tiles", frames)
+    stf.set_option("lookahead", lookahead)
+    try:
+        edges, kinds, ijk, st = stf.dag(T, p, q)
+        io, nbuf = stf.dag_io(len(kinds))
+    finally:
+        stf.set_option("mem_cap_tiles", 0)
+        stf.set_option("lookahead", 1)
+    return edges, kinds, ijk, io, nbuf, st
+
+
+def _emulate(T, A, kinds, ijk, io, nbuf, edges, order_seed, host_resident):
+    """Run the tasks in a random topological order (Kahn, random ready pick)."""
+    nb = NB
+    # column-major tiles written in place, as oracle.tiled_potrf does (numpy's
+    # matmul rounding depends on operand layout)
+    H = {(i, j): np.asfortranarray(A[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb]) for i in range(T) for j in range(i + 1)}
+    buf = [np.zeros((nb, nb), order="F") for _ in range(nbuf)]
+    if not host_resident:  # TILED_2DBC: home buffers hold the caller's tiles
+        for (i, j), t in H.items():
+            buf[i * (i + 1) // 2 + j][:, :] = t
+    n = len(kinds)
+    succ = [[] for _ in range(n)]
+    indeg = [0] * n
+    for s, d in edges:
+        succ[s].append(d)
+        indeg[d] += 1
+    rng = np.random.default_rng(max(order_seed, 0))
+    ready = [t for t in range(n) if indeg[t] == 0]
+    done = 0
+    while ready:
+        t = ready.pop(int(rng.integers(len(ready))) if order_seed >= 0 else 0)
+        (r0, r1), w = io[t]
+        kd = kinds[t]
+        i, j, k = ijk[t]
+        if kd == "POTRF":
+            L, info = oracle.potrf(buf[w])
+            assert info == 0
+            buf[w][:, :] = L
+        elif kd == "TRSM":
+            buf[w][:, :] = oracle.tile_trsm(buf[w], buf[r0])
+        elif kd == "SYRK":
+            buf[w][:, :] = oracle.tile_syrk(buf[w], buf[r0])
+        elif kd == "GEMM":
+            buf[w][:, :] = oracle.tile_gemm(buf[w], buf[r0], buf[r1])
+        elif kd == "COPY":
+            buf[w][:, :] = buf[r0]
+        elif kd == "LOAD":
+            buf[w][:, :] = H[(i, j)]
+        elif kd == "STORE":
+            H[(i, j)][:, :] = buf[r0]
+        else:
+            assert kd == "FENCE"
+        done += 1
+        for d in succ[t]:
+            indeg[d] -= 1
+            if indeg[d] == 0:
+                ready.append(d)
+        if order_seed < 0:
+            ready.sort()
+    assert done == n, "the plan's DAG has a cycle"
+    out = np.zeros((T * nb, T * nb))
+    for (i, j) in H:
+        tile = H[(i, j)] if host_resident else buf[i * (i + 1) // 2 + j]
+        out[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb] = tile
+    return np.tril(out)
+
+
+def _reference(T, A):
+    L, info = oracle.tiled_potrf(A, NB)
+    assert info == 0
+    return np.tril(L)
+
+
+@pytest.mark.parametrize("T,p,q,lookahead", [(5, 1, 1, 1), (6, 1, 2, 1), (6, 2, 2, 1), (7, 2, 4, 1), (6, 2, 2, 0)])
+def test_distributed_plan_any_topological_order(T, p, q, lookahead):
+    A = synth.spd_matrix(7, T * NB)
+    edges, kinds, ijk, io, nbuf, st = _plan(T, p, q, lookahead=lookahead)
+    ref = _reference(T, A)
+    for seed in (-1, 1, 2, 3):
+        got = _emulate(T, A, kinds, ijk, io, nbuf, edges, seed, host_resident=False)
+        assert np.array_equal(got, ref), (seed, np.abs(got - ref).max())
+
+
+@pytest.mark.parametrize("T,frames", [(4, 3), (4, 5), (6, 3), (6, 4), (6, 7), (6, 12), (8, 6), (8, 20), (9, 10)])
+def test_out_of_core_plan_any_topological_order(T, frames):
+    A = synth.spd_matrix(11, T * NB)
+    edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames)
+    NT = T * (T + 1) // 2
+    assert st["frames"] == frames and nbuf == frames
+    assert "COPY" not in kinds
+    # every buffer a task touches is a frame; each tile is loaded and written back at least once
+    for (r0, r1), w in io:
+        assert all(-1 <= b < frames for b in (r0, r1, w))
+    assert st["host_loads"] >= NT and st["host_stores"] >= NT
+    assert kinds.count("LOAD") == st["host_loads"] and kinds.count("STORE") == st["host_stores"]
+    ref = _reference(T, A)
+    for seed in (-1, 1, 2, 3, 4):
+        got = _emulate(T, A, kinds, ijk, io, nbuf, edges, seed, host_resident=True)
+        assert np.array_equal(got, ref), (seed, np.abs(got - ref).max())
+
+
+def test_out_of_core_compute_order_matches_stf_closure():
+    """Frames add orderings (WAR on reuse), never drop one: every pair the
+    single-GPU STF closure orders is still ordered among the compute tasks."""
+    T, frames = 6, 5
+    edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames)
+    comp = [t for t, k in enumerate(kinds) if k in ("POTRF", "TRSM", "SYRK", "GEMM")]
+    R = oracle.transitive_closure(len(kinds), set(edges))
+    ot = oracle.cholesky_tasks(T)
+    Ro = oracle.transitive_closure(len(ot), oracle.stf_edges([acc for _, _, acc in ot]))
+    # map our compute tasks (left-looking order) onto the oracle's task list by (kind, i, j, k)
+    name = {}
+    for idx, (kd, (i, j, k), _) in enumerate(ot):
+        name[(kd, i, j, k)] = idx
+    ours = []
+    for t in comp:
+        kd = kinds[t]
+        i, j, k = ijk[t]
+        # library names: TRSM(i,k) = (i,k,k), SYRK(i,k) = (i,i,k) -- same as the oracle's
+        ours.append(name[(kd, i, j, k)])
+    assert sorted(ours) == list(range(len(ot)))
+    sub = R[np.ix_(comp, comp)]
+    for a, ta in enumerate(ours):
+        for b, tb in enumerate(ours):
+            if Ro[ta, tb]:
+                assert sub[a, b], (kinds[comp[a]], ijk[comp[a]], kinds[comp[b]], ijk[comp[b]])
+
+
+def test_out_of_core_traffic_left_looking():
+    """With room for wide super-columns the plan re-reads far fewer tiles than a
+    right-looking sweep: loads stay within a small multiple of the tile count."""
+    T = 16
+    NT = T * (T + 1) // 2
+    _, _, _, _, _, st_small = _plan(T, 1, 1, frames=24)
+    _, _, _, _, _, st_big = _plan(T, 1, 1, frames=NT // 2)
+    assert st_big["host_loads"] < st_small["host_loads"]
+    assert st_big["host_stores"] == NT  # every tile written back exactly once
+    assert st_big["host_loads"] <= 3 * NT
+    _, _, _, _, _, st_none = _plan(T, 1, 1, frames=NT)  # cap >= matrix: no out-of-core plan
+    assert st_none["frames"] == 0 and st_none["host_loads"] == 0
