@@ -10,7 +10,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libstf_cholesky.so")
+LIB_PATH = os.environ.get("STF_LIB_PATH") or os.path.join(_HERE, "libstf_cholesky.so")  # override: A/B experiments only
 
 STF_DESC_TILED_2DBC = 0
 STF_DESC_DEVICE_COLMAJOR = 1

@@ -222,11 +222,16 @@ struct OocBuilder {
 
   int64_t id(int64_t i, int64_t j) const { return Plan::tile_id(i, j); }
 
+  // updates from column k to columns j0..j1.  Column j0 is the next to be
+  // factored: its updates are critical (high-priority streams), so they are not
+  // queued behind the wider block's updates in the bulk streams' FIFO order.
   void emit_updates_from(int64_t k, int64_t j0, int64_t j1) {
     for (int64_t j = j0; j <= j1; ++j) {
-      seq.push_back({K_SYRK, (int32_t)j, (int32_t)j, (int32_t)k, 2, id(j, k), -1, id(j, j)});
+      const int d = (int)(j - j0);
+      seq.push_back({K_SYRK, (int32_t)j, (int32_t)j, (int32_t)k, d == 0 ? 5 : d == 1 ? 3 : 2, id(j, k), -1, id(j, j)});
       for (int64_t i = j + 1; i < T; ++i)
-        seq.push_back({K_GEMM, (int32_t)i, (int32_t)j, (int32_t)k, 1, id(i, k), id(j, k), id(i, j)});
+        seq.push_back({K_GEMM, (int32_t)i, (int32_t)j, (int32_t)k, d == 0 ? 4 : d == 1 ? 2 : 1, id(i, k), id(j, k),
+                       id(i, j)});
     }
   }
 

@@ -27,6 +27,22 @@ def main():
     A = torch.empty((n, n), dtype=torch.float64, pin_memory=True)
     dev = torch.empty((n, n), dtype=torch.float64, device="cuda:0")
     tile_b = nb * nb * 8
+    # PCIe roofline: pinned host <-> device copy bandwidth of this box (1 GiB, best of 3)
+    h = torch.empty(1 << 27, dtype=torch.float64, pin_memory=True)
+    d = torch.empty(1 << 27, dtype=torch.float64, device="cuda:0")
+    bw = {}
+    for name, (dst, src) in (("h2d", (d, h)), ("d2h", (h, d))):
+        best = 1e9
+        for _ in range(3):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            dst.copy_(src, non_blocking=True)
+            e1.record()
+            e1.synchronize()
+            best = min(best, e0.elapsed_time(e1))
+        bw[name] = (1 << 30) / (best * 1e-3) / 1e9
+    del h, d
+    print(json.dumps({"pcie_h2d_GBps": round(bw["h2d"], 1), "pcie_d2h_GBps": round(bw["d2h"], 1)}), flush=True)
     out = []
     for cap in caps:
         stf.set_option("mem_cap_tiles", cap)
@@ -50,6 +66,7 @@ def main():
                 "host_loads": st["host_loads"], "host_stores": st["host_stores"],
                 "h2d_GB": round(st["host_loads"] * tile_b / 1e9, 2), "d2h_GB": round(st["host_stores"] * tile_b / 1e9, 2),
                 "h2d_GBps_avg": round(st["host_loads"] * tile_b / (ms * 1e-3) / 1e9, 1),
+                "pcie_bound_ms": round(max(st["host_loads"] * tile_b / bw["h2d"], st["host_stores"] * tile_b / bw["d2h"]) / 1e6, 1),
                 "graph_nodes": st["graph_nodes"], "build_ms": round(res[0][2]["build_ms"], 1)}
         print(json.dumps(line), flush=True)
         out.append(line)
