@@ -208,57 +208,113 @@ __device__ __forceinline__ void solve_core(double (&b)[16], const double* Ls, do
   }
 }
 
-// Cholesky core of an nc x nc block.  Thread (r, q) holds A[r, 16q .. 16q+15]
-// (lower part) in a[]; chunk q (two warps, named barrier 1+q) factors its 16
-// columns (pivot sqrt by the owner of row col, division by the pivot, in-chunk
-// rank-1 updates), publishing L into S[r * LDB + col]; later chunks apply the
-// chunk's update.  Element updates run in increasing column order (Crout order).
-// On return a[] holds L and S its lower part (diagonal included).
-__device__ __forceinline__ void chol_core(double (&a)[16], double* S, double* Y, int nc, int64_t col0,
+// Cholesky core of an nc x nc block (nc <= 64), latency-optimised for the
+// critical chain (tools/chol_lab.cu, bit-identical to the quarter-serial form).  Thread (r = tid & 63,
+// q = tid >> 6) holds A[r, 4m + q] in a[m] (interleaved columns, so all 256
+// threads share every column's update).  Column j+1 needs ONE barrier:
+//   * every owner thread of column j+1 (q == (j+1) & 3, two warps) recomputes
+//     the pivot itself: d = a_{j+1,j+1} - L_{j+1,j}^2 from the published
+//     diagonal Dp[j+1] and L_{j+1,j}, s = sqrt(d), y = 1/s (IEEE), then divides
+//     its own element, L_{r,j+1} = div_by(a_{r,j+1} - L_rj L_{j+1,j}, s, y),
+//     and publishes it in Lc[(j+1) % 3];
+//   * the other threads apply column j's update to their elements; the owners'
+//     own updates from column j are deferred to the next iteration (their
+//     columns are >= j+5, not needed before then), so the owner warps run the
+//     pivot chain alone.
+// Every element still receives its updates in increasing column order with the
+// same fma(-L_rk, L_ck, a) as the unblocked algorithm; sqrt and division are
+// correctly rounded.  Rows above the diagonal and rows >= nc carry garbage that
+// is never read or stored (no divergent branches in the loop).  Non-positive
+// pivot (or NaN): info = min(info, col0 + col + 1), s = NaN.
+// Scratch: Lc[3 * W], Dp[W + 2].  On return S[r * LDB + c] = L(r, c) for r >= c
+// (after a __syncthreads); a[] is consumed.
+__device__ __forceinline__ void chol_core(double (&a)[16], double* S, double* Lc, double* Dp, int nc, int64_t col0,
                                           unsigned long long* info) {
-  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
-  for (int qq = 0; qq < 4 && 16 * qq < nc; ++qq) {
-    if (q == qq) {
+  constexpr int W = df::W;
+  const int r = threadIdx.x & (W - 1), q = threadIdx.x >> 6;
+  const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
+  if (q == 0 && r == 0) Dp[0] = a[0];
+  if (q == 1 && r == 1) Dp[1] = a[0];
+  __syncthreads();
+  int bad = 0;  // 1-based column of this thread's failed pivot (row r is column r's pivot row)
+  if (q == 0) {
+    const double d = Dp[0];
+    const bool ok = d > 0.0;
+    bad = (!ok && r == 0) ? 1 : bad;
+    const double s = ok ? sqrt(d) : kNaN, y = 1.0 / s;
+    a[0] = (r == 0) ? s : div_by(a[0], s, y);
+    Lc[r] = a[0];
+  }
+  __syncthreads();
+  // Groups of 4 columns at run time; a[m] holds column 4(g + m) + q during group g
+  // (the window shifts by one element per group, so register indices stay static).
+  const int ng = (nc + 3) >> 2;
+  for (int g = 0; g < ng; ++g) {
 #pragma unroll
-      for (int c = 0; c < 16; ++c) {
-        const int col = 16 * qq + c;
-        if (col < nc) {
-          if (r == col) {
-            double s = a[c];
-            if (!(s > 0.0)) {
-              atomicMin(info, (unsigned long long)(col0 + col + 1));
-              s = __longlong_as_double(0x7ff8000000000000LL);
-            } else {
-              s = sqrt(s);
+    for (int u = 0; u < 4; ++u) {
+      const int j = 4 * g + u, j1 = j + 1;
+      if (j1 < nc) {  // uniform
+        const int b = j % 3, bn = j1 % 3, bp = (j + 2) % 3;
+        const int w1 = (u == 3) ? 1 : 0;  // window slot of column j+1 in quarter (u+1)&3
+        const double lr = Lc[b * W + r];
+        if (q == ((u + 1) & 3)) {  // warp-uniform: the owners of column j+1 run the pivot chain
+          const double l1 = Lc[b * W + j1];
+          const double d = fma(-l1, l1, Dp[j1]);
+          const bool ok = d > 0.0;
+          bad = (!ok && r == j1) ? j1 + 1 : bad;
+          const double s = ok ? sqrt(d) : kNaN, y = 1.0 / s;
+          const double v = div_by(fma(-lr, l1, a[w1]), s, y);
+          a[w1] = (r == j1) ? s : v;
+          Lc[bn * W + r] = a[w1];
+        } else {
+          if (j >= 1 && q == u) {  // deferred: this quarter's updates from column j-1 (columns > j)
+            const double lp = Lc[bp * W + r];
+            const double* Lp = Lc + bp * W + 4 * g + q;
+#pragma unroll
+            for (int m = 0; m < 16; ++m)
+              if (4 * m + q > u) a[m] = fma(-lp, Lp[(4 * m) & 63], a[m]);
+          }
+          const double* Lb = Lc + b * W + 4 * g + q;
+#pragma unroll
+          for (int m = 0; m < 16; ++m) {
+            if (4 * m + q > u + 1) {  // column 4(g+m)+q > j+1
+              a[m] = fma(-lr, Lb[(4 * m) & 63], a[m]);
+              if (4 * m + q == u + 2 && r == j + 2) Dp[j + 2] = a[m];
             }
-            a[c] = s;
-            S[col * df::LDB + col] = s;
-            Y[col] = 1.0 / s;
-          }
-          named_bar(1 + qq, 64);
-          if (r > col && r < nc) {
-            a[c] = div_by(a[c], S[col * df::LDB + col], Y[col]);
-            S[r * df::LDB + col] = a[c];
-          }
-          named_bar(1 + qq, 64);
-          if (r > col && r < nc) {
-#pragma unroll
-            for (int c2 = c + 1; c2 < 16; ++c2)
-              if (16 * qq + c2 <= r) a[c2] = fma(-a[c], S[(16 * qq + c2) * df::LDB + col], a[c2]);
           }
         }
       }
+      __syncthreads();
     }
-    __syncthreads();
-    if (q > qq && r < nc) {
+    // column 4g+q is final: publish it, shift the window
+    {
+      const int c = 4 * g + q;
+      if (r >= c && r < nc && c < nc) S[r * df::LDB + c] = a[0];
+    }
 #pragma unroll
-      for (int cc = 0; cc < 16; ++cc) {
-        if (16 * q + cc <= r) {
+    for (int m = 0; m < 15; ++m) a[m] = a[m + 1];
+    a[15] = 0.0;
+  }
+  if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
+  __syncthreads();
+}
+
+// interleaved-column register blocks (chol_core layout): v[m] = G(r, 4m + q)
+__device__ __forceinline__ void load_il(double (&v)[16], const double* G, int64_t ldg, int rows, int nc, bool lower) {
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
 #pragma unroll
-          for (int c = 0; c < 16; ++c)
-            a[cc] = fma(-S[r * df::LDB + 16 * qq + c], S[(16 * q + cc) * df::LDB + 16 * qq + c], a[cc]);
-        }
-      }
+  for (int m = 0; m < 16; ++m) {
+    const int col = 4 * m + q;
+    v[m] = (r < rows && col < nc && (!lower || r >= col)) ? __ldcg(G + (int64_t)col * ldg + r) : 0.0;
+  }
+}
+__device__ __forceinline__ void store_il(const double (&v)[16], double* G, int64_t ldg, int rows, int nc, bool lower) {
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
+  if (r < rows) {
+#pragma unroll
+    for (int m = 0; m < 16; ++m) {
+      const int col = 4 * m + q;
+      if (col < nc && (!lower || r >= col)) G[(int64_t)col * ldg + r] = v[m];
     }
   }
 }
@@ -300,11 +356,12 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
 // P task: in-place lower Cholesky of the nc x nc diagonal block at X (global).
 __device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
   double* S = sm;
-  double* Y = sm + df::W * df::LDB;
+  double* Lc = sm + df::W * df::LDB;
+  double* Dp = Lc + 3 * df::W;
   double a[16];
-  load_chunk(a, X, ldx, nc, nc, true);
-  chol_core(a, S, Y, nc, col0, info);
-  store_chunk(a, X, ldx, nc, nc, true);
+  load_il(a, X, ldx, nc, nc, true);
+  chol_core(a, S, Lc, Dp, nc, col0, info);
+  store_block_rm(S, df::LDB, X, ldx, nc, nc, true);
 }
 
 // The critical path of the tile Cholesky, run by ONE CTA with its blocks kept
@@ -317,20 +374,21 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
   double* D = sm;                          // [r][LDB]: P publication buffer -> L_kk
   double* XS = sm + W * df::LDB;           // [r][LDO]: X(kb+1, kb), A and B of U
   double* Rc = XS + W * df::LDO;           // W
-  double* Y = Rc + W;                      // W
+  double* Lc = XS;                         // 3 W: chol_core scratch (XS is dead during P)
+  double* Dp = XS + 3 * W;                 // W + 2
   int* prog = p.ws + 2;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   const int wm0 = (warp & 1) * 32, wn0 = (warp >> 1) * 16;
   const int r = threadIdx.x & (W - 1), q = threadIdx.x >> 6;
   double a[16];
-  load_chunk(a, p.X, p.ldx, min(W, p.n), min(W, p.n), true);  // P(0) input: nothing precedes it
+  load_il(a, p.X, p.ldx, min(W, p.n), min(W, p.n), true);  // P(0) input: nothing precedes it
   for (int kb = 0; kb < T; ++kb) {
     const int nk = min(W, p.n - kb * W);
     double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
     // ---- P(kb)
     DF_STAMP(6 * kb + 0);
-    chol_core(a, D, Y, nk, p.col0 + (int64_t)kb * W, p.info);
-    store_chunk(a, Xkk, p.ldx, nk, nk, true);
+    chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
+    store_block_rm(D, df::LDB, Xkk, p.ldx, nk, nk, true);
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
@@ -396,9 +454,9 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
         for (int h = 0; h < 2; ++h) D[(wm0 + 8 * i + g) * df::LDB + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
     __syncthreads();
 #pragma unroll
-    for (int c = 0; c < 16; ++c) {
-      const int col = 16 * q + c;
-      a[c] = (r < rows && col < rows && r >= col) ? D[r * df::LDB + col] : 0.0;
+    for (int m = 0; m < 16; ++m) {
+      const int col = 4 * m + q;
+      a[m] = (r < rows && col < rows && r >= col) ? D[r * df::LDB + col] : 0.0;
     }
     __syncthreads();  // D is rewritten by the next chol_core
     DF_STAMP(6 * kb + 5);
