@@ -96,10 +96,14 @@ const char *stf_last_error(void);
 /* ---------------------------------------------------------------- options
  * Execution options (defaults from the environment at init):
  *   "dataflow" STF_DATAFLOW POTRF tile kernel: 1 single-launch dataflow (default), 0 recursive
- *   "trsm"     STF_TRSM     TRSM tile kernel: 2 row-panel (default), 1 dataflow, 0 recursive
+ *   "trsm"     STF_TRSM     TRSM tile kernel: 3 (default) = resident panel for the critical
+ *                           TRSM(k+1,k) when nb <= 1024 and nb % 64 == 0, row panel otherwise;
+ *                           2 row panel, 1 dataflow, 0 recursive
  *   "trsm_split" STF_TRSM_SPLIT P in [1,16]: non-critical row-panel TRSMs run right-looking
  *                           over P column blocks (panel kernel + GEMM updates; default 4);
  *                           1: one panel launch
+ *   "trsm_res_tail" STF_TRSM_RES_TAIL R >= 0: with trsm 3, TRSM(i,k) of the last R panel
+ *                           steps (T - k <= R) also use the resident panel (default 16)
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA
  *                           graph, memoised per (n, nb, grid, tiles) (default);
  *                           0: eager lowering on streams + events
@@ -211,6 +215,16 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
  * done stamps of bulk ticket t (0 if unused).  Returns the number of entries
  * written (<= cap) or a negative error.  Not part of the factorisation. */
 int64_t stf_debug_potrf_trace(int64_t n, double *A, int64_t lda, int ctas, int64_t *trace, int64_t cap);
+
+/* Debug timeline of the resident-panel TRSM kernel (B[M x n] <- B L^-T, device
+ * pointers, current device; requires 64 <= n <= 1024, n % 64 == 0).  With
+ * T = n/64, trace[5 kb + e] holds the %globaltimer stamps (ns) of CTA 0 for
+ * column block kb: e = 0 MMA step start, 1 MMA waits for the previous block's
+ * solution, 2 it is available, 3 updated block handed to the solver, 4 solver
+ * starts; trace[5T + kb] the solver's end.  Returns the number of entries
+ * written (<= cap) or a negative error.  Not part of the factorisation. */
+int64_t stf_debug_trsm_trace(int64_t M, int64_t n, const double *L, int64_t ldl, double *B, int64_t ldb,
+                             int64_t *trace, int64_t cap);
 
 /* ---------------------------------------------------------------- multi-process mode
  * One process per GPU (e.g. torch.distributed / torchrun): process `rank` owns

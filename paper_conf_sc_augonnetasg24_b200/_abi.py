@@ -59,6 +59,7 @@ EXPORTS = [
     "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_infer_edges",
     "stf_fill_spd_tiles", "stf_fill_spd_block",
     "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace",
+    "stf_debug_trsm_trace",
     "stf_dag_tasks_io", "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
 ]
 
@@ -103,6 +104,7 @@ stf_mp_prepare = _decl("stf_mp_prepare", _int, [_i64, _i64, _P(stf_matrix_desc),
 stf_mp_import = _decl("stf_mp_import", _int, [_vp])
 stf_mp_potrf = _decl("stf_mp_potrf", _int, [])
 stf_debug_potrf_trace = _decl("stf_debug_potrf_trace", _i64, [_i64, _vp, _i64, _int, _P(_i64), _i64])
+stf_debug_trsm_trace = _decl("stf_debug_trsm_trace", _i64, [_i64, _i64, _vp, _i64, _vp, _i64, _P(_i64), _i64])
 
 
 class StfError(RuntimeError):

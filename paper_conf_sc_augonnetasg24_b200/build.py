@@ -27,6 +27,7 @@ SOURCES = [
     "kernels/panel.cu",
     "kernels/dataflow.cu",
     "kernels/trsm_panel.cu",
+    "kernels/trsm_res.cu",
     "plan.cpp",
     "runtime.cpp",
 ]

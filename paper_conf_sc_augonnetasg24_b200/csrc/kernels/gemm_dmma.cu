@@ -232,7 +232,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 }
 
 // rows x cols column-major FP64 operand, box {16 rows, bk cols}, 128B swizzle, OOB -> 0.
-static bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld, int bk) {
+bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld, int bk) {
   auto fn = encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {(cuuint64_t)rows, (cuuint64_t)cols};

@@ -228,6 +228,7 @@ cudaError_t info_reset(cudaStream_t stream, unsigned long long* info) {
 cudaError_t gemm_init_attrs();
 cudaError_t dataflow_init_attrs();
 cudaError_t trsm_panel_init_attrs();
+cudaError_t trsm_res_init_attrs();
 
 cudaError_t kernels_init(int device) {
   int cur = 0;
@@ -236,6 +237,7 @@ cudaError_t kernels_init(int device) {
   cudaError_t e = gemm_init_attrs();
   if (e == cudaSuccess) e = dataflow_init_attrs();
   if (e == cudaSuccess) e = trsm_panel_init_attrs();
+  if (e == cudaSuccess) e = trsm_res_init_attrs();
   cudaSetDevice(cur);
   return e;
 }

@@ -57,6 +57,14 @@ cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double
                        int64_t ldb, int rows_per_cta = 0, const Mirrors* mirrors = nullptr);
 cudaError_t dataflow_prepare(int m, int n, bool potrf);
 
+// K3 resident-panel form (trsm_res.cu): one launch, ceil(M/16) CTAs each keeping
+// its 16 x n row panel in shared memory; MMA warps (left-looking DMMA updates)
+// and solver warps (substitution) overlap.  Requires trsm_res_supported(n, L, ldl):
+// 64 <= n <= 1024, n % 64 == 0, ldl even, L 16-byte aligned.
+bool trsm_res_supported(int n, const double* L, int64_t ldl);
+cudaError_t trsm_res(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                     int64_t ldb, const Mirrors* mirrors = nullptr, unsigned long long* trace = nullptr);
+
 // K8: fill rows r0.., cols c0.. (global indices) of the seeded SPD metric matrix
 // of order n into dst[rows x cols] (ld).  Same SplitMix64 spec as synth/spd.py.
 cudaError_t fill_spd(cudaStream_t stream, double* dst, int64_t ld, int64_t n, int64_t r0, int64_t c0, int rows,

@@ -79,7 +79,7 @@ struct Slot {
 
 struct Options {
   int64_t dataflow = 1;  // POTRF tile kernel: 1 single-launch dataflow, 0 recursive (GEMM-based)
-  int64_t trsm = 2;      // TRSM tile kernel: 2 row-panel, 1 dataflow, 0 recursive
+  int64_t trsm = 3;      // TRSM tile kernel: 3 resident panel, 2 row-panel, 1 dataflow, 0 recursive
   int64_t trsm_split = 4;  // row panel: non-critical TRSMs as `trsm_split` column blocks (panel + GEMM updates)
   int64_t graph = 1;
   int64_t streams = 8;
@@ -90,13 +90,14 @@ struct Options {
   int64_t threads = 8;  // eager backend: host submission threads (one per slot group)
   int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
   int64_t mem_cap_tiles = 0;  // HOST_COLMAJOR on one GPU: device tile frames (0 = whole matrix resident)
+  int64_t trsm_res_tail = 16;  // trsm 3: non-critical TRSM(i,k) also resident-panel when T - k <= this
 };
 
 // options that change the plan or its lowering (part of the memo key)
 bool same_plan_options(const Options& a, int64_t a_graph, const Options& b) {
   return a.streams == b.streams && a.serial == b.serial && a_graph == b.graph && a.priority == b.priority &&
          a.dataflow == b.dataflow && a.trsm == b.trsm && a.trsm_split == b.trsm_split && a.push == b.push &&
-         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles;
+         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.trsm_res_tail == b.trsm_res_tail;
 }
 
 // A plan bound to physical buffers, plus its lowering artefacts.
@@ -217,7 +218,7 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.with_load = load;
   po.with_store = store;
   po.lookahead = o.lookahead != 0;
-  po.push = o.push != 0 && o.trsm == 2;
+  po.push = o.push != 0 && o.trsm >= 2;
   return po;
 }
 
@@ -269,12 +270,19 @@ struct Lowerer {
                    "TRSM what-if");
           return 0;
         }
-        if (X.opt.trsm == 2 && t.i == t.k + 1) {
+        if (X.opt.trsm == 3 && (t.i == t.k + 1 || X.n / nb - t.k <= X.opt.trsm_res_tail) &&
+            stfk::trsm_res_supported((int)nb, X.buf[(size_t)t.in[0]], nb)) {
+          // the next panel's TRSM(k+1,k) is on the critical path, and near the end of the
+          // factorisation every TRSM is latency-bound: the resident-panel kernel (16 rows per
+          // CTA, 4x the CTAs of the row panel, solve overlapped with the updates)
+          CUDA_TRY(stfk::trsm_res(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, &mir),
+                   "TRSM launch");
+        } else if (X.opt.trsm >= 2 && t.i == t.k + 1) {
           // the next panel's TRSM(k+1,k) is on the critical path: one low-latency launch
           CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 32,
                                     &mir),
                    "TRSM launch");
-        } else if (X.opt.trsm == 2 && X.opt.trsm_split > 1 && nb % (64 * X.opt.trsm_split) == 0) {
+        } else if (X.opt.trsm >= 2 && X.opt.trsm_split > 1 && nb % (64 * X.opt.trsm_split) == 0) {
           // Right-looking over `parts` column blocks of width w:
           //   X_p = B_p L_pp^-T (row-panel kernel);  B_{>p} -= X_p L_{>p,p}^T (full-rate GEMM kernel).
           // Only 1/parts of the TRSM flops stay in the substitution kernel (SM-time matters here,
@@ -293,7 +301,7 @@ struct Lowerer {
                                      L + pp * w * nb + (pp + 1) * w, nb, B + (pp + 1) * w * nb, nb, 0),
                        "TRSM GEMM");
           }
-        } else if (X.opt.trsm == 2) {
+        } else if (X.opt.trsm >= 2) {
           CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 0,
                                     &mir),
                    "TRSM launch");
@@ -857,8 +865,9 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   if (ngpus < 1 || ngpus > 64) return fail(-5, "ngpus=%d out of range", ngpus);
   C.opt.graph = env_int("STF_GRAPH", 1);
   C.opt.dataflow = env_int("STF_DATAFLOW", 1);
-  C.opt.trsm = env_int("STF_TRSM", 2);
+  C.opt.trsm = env_int("STF_TRSM", 3);
   C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 4);
+  C.opt.trsm_res_tail = env_int("STF_TRSM_RES_TAIL", 16);
   C.opt.push = env_int("STF_PUSH", 0);
   C.opt.mem_cap_tiles = env_int("STF_MEM_CAP_TILES", 0);
   C.opt.streams = env_int("STF_STREAMS", 8);
@@ -974,7 +983,8 @@ int stf_set_option(const char* name, int64_t value) {
   if (n == "graph") C.opt.graph = value != 0;
   else if (n == "dataflow") C.opt.dataflow = value != 0;
   else if (n == "trsm") {
-    if (value < 0 || value > 2) return fail(-105, "trsm must be 0 (recursive), 1 (dataflow) or 2 (row panel)");
+    if (value < 0 || value > 3)
+      return fail(-105, "trsm must be 0 (recursive), 1 (dataflow), 2 (row panel) or 3 (resident panel)");
     C.opt.trsm = value;
   }
   else if (n == "streams") {
@@ -987,6 +997,10 @@ int stf_set_option(const char* name, int64_t value) {
   else if (n == "trsm_split") {
     if (value < 1 || value > 16) return fail(-105, "trsm_split must be in [1, 16]");
     C.opt.trsm_split = value;
+  }
+  else if (n == "trsm_res_tail") {
+    if (value < 0) return fail(-105, "trsm_res_tail must be >= 0");
+    C.opt.trsm_res_tail = value;
   }
   else if (n == "push") C.opt.push = value != 0;
   else if (n == "mem_cap_tiles") {
@@ -1018,6 +1032,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "serial") *value = C.opt.serial;
   else if (n == "lookahead") *value = C.opt.lookahead;
   else if (n == "trsm_split") *value = C.opt.trsm_split;
+  else if (n == "trsm_res_tail") *value = C.opt.trsm_res_tail;
   else if (n == "push") *value = C.opt.push;
   else if (n == "mem_cap_tiles") *value = C.opt.mem_cap_tiles;
   else if (n == "threads") *value = C.opt.threads;
@@ -1328,7 +1343,12 @@ int stf_kernel_trsm(int64_t M, int64_t n, const double* L, int64_t ldl, double* 
   cudaGetDevice(&dev);
   int r = ensure_kernel_attrs(dev);
   if (r) return r;
-  if (ctx().opt.trsm == 2) {
+  if (ctx().opt.trsm == 3 && stfk::trsm_res_supported((int)n, L, ldl)) {
+    CUDA_TRY(stfk::trsm_res(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm (resident panel)");
+    CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
+    return 0;
+  }
+  if (ctx().opt.trsm >= 2) {
     CUDA_TRY(stfk::trsm_panel(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm (row panel)");
     CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
     return 0;
@@ -1522,7 +1542,9 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
         case 0: step(stfk::gemm_nt(s, 0, (int)M, (int)N, (int)K, A, ldm, B, ldn, Cm, ldm, 0)); break;
         case 1: step(stfk::gemm_nt(s, 0, (int)M, (int)M, (int)K, A, ldm, A, ldm, Cm, ldm, 1)); break;
         case 2:
-          step(ctx().opt.trsm == 2   ? stfk::trsm_panel(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)
+          step(ctx().opt.trsm == 3 && stfk::trsm_res_supported((int)N, Src, ldm)
+                   ? stfk::trsm_res(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)
+               : ctx().opt.trsm >= 2 ? stfk::trsm_panel(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)
                : ctx().opt.trsm == 1 ? stfk::trsm_tile(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm, ws)
                                      : stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm));
           break;
@@ -1571,6 +1593,27 @@ int64_t stf_debug_potrf_trace(int64_t n, double* A, int64_t lda, int ctas, int64
   cudaFree(d_tr);
   cudaFree(ws);
   if (e != cudaSuccess) return cuda_fail(e, "potrf trace");
+  return cnt;
+}
+
+int64_t stf_debug_trsm_trace(int64_t M, int64_t n, const double* L, int64_t ldl, double* B, int64_t ldb,
+                             int64_t* trace, int64_t cap) {
+  g_err.clear();
+  if (M < 1 || !stfk::trsm_res_supported((int)n, L, ldl)) return fail(-4, "unsupported TRSM trace shape");
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int r = ensure_kernel_attrs(dev);
+  if (r) return r;
+  const int64_t slots = 6 * (n / 64);
+  unsigned long long* d_tr = nullptr;
+  cudaError_t e = cudaMalloc(&d_tr, (size_t)slots * 8);
+  if (e == cudaSuccess) e = cudaMemset(d_tr, 0, (size_t)slots * 8);
+  if (e == cudaSuccess) e = stfk::trsm_res(0, 0, (int)M, (int)n, L, ldl, B, ldb, nullptr, d_tr);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(0);
+  const int64_t cnt = std::min<int64_t>(cap, slots);
+  if (e == cudaSuccess && trace) e = cudaMemcpy(trace, d_tr, (size_t)cnt * 8, cudaMemcpyDeviceToHost);
+  cudaFree(d_tr);
+  if (e != cudaSuccess) return cuda_fail(e, "trsm trace");
   return cnt;
 }
 

@@ -21,15 +21,17 @@ def abi():
     return _abi
 
 
-@pytest.fixture(params=[(1, 2), (1, 1), (0, 0)], ids=["dataflow+rowpanel", "dataflow", "recursive"])
+@pytest.fixture(params=[(1, 3), (1, 2), (1, 1), (0, 0)], ids=["dataflow+resident", "dataflow+rowpanel", "dataflow",
+                                                              "recursive"])
 def variant(request, abi):
     """(POTRF, TRSM) implementations: POTRF dataflow (1) / recursive (0);
-    TRSM row panel (2, product default) / dataflow (1) / recursive (0)."""
+    TRSM resident panel (3, product default; row panel where unsupported) /
+    row panel (2) / dataflow (1) / recursive (0)."""
     abi.stf_set_option(b"dataflow", request.param[0])
     abi.stf_set_option(b"trsm", request.param[1])
     yield request.param
     abi.stf_set_option(b"dataflow", 1)
-    abi.stf_set_option(b"trsm", 2)
+    abi.stf_set_option(b"trsm", 3)
 
 
 def _even(x):
@@ -89,7 +91,7 @@ def test_syrk_lower(abi, N, K):
 
 
 @pytest.mark.parametrize("M,n", [(64, 64), (100, 70), (1024, 1024), (300, 200), (1, 1), (512, 129), (2048, 2048),
-                                 (130, 1000)])
+                                 (130, 1000), (1000, 1024), (17, 64), (1, 128), (33, 192), (250, 512), (1024, 960)])
 def test_trsm(abi, variant, M, n):
     rng = np.random.default_rng(M + n)
     Lfull = np.tril(rng.standard_normal((n, n))) * 0.1 + np.diag(1.0 + rng.random(n))

@@ -24,11 +24,11 @@ def stf():
     s.finalize()
 
 
-@pytest.mark.parametrize("trsm,split", [(1, 1), (2, 1), (2, 2), (2, 4), (2, 8)])
+@pytest.mark.parametrize("trsm,split", [(1, 1), (2, 1), (2, 2), (2, 4), (2, 8), (3, 4)])
 def test_parity_trsm_variants(stf, trsm, split):
     _options(stf, trsm=trsm, trsm_split=split)
     M, info = _factor_spd(stf, 1536, 512, seed=2)
-    _options(stf, trsm=2, trsm_split=4)
+    _options(stf, trsm=3, trsm_split=4)
     assert info == 0
     Lo, _ = oracle.potrf(synth.spd_matrix(2, 1536))
     assert relF(M.to_dense().numpy(), Lo) <= 1e-10
@@ -38,7 +38,7 @@ def test_parity_recursive_panel_kernels(stf):
     """The recursive (GEMM-based) POTRF/TRSM variant through the whole path."""
     _options(stf, dataflow=0, trsm=0)
     M, info = _factor_spd(stf, 2048, 512, seed=1)
-    _options(stf, dataflow=1, trsm=2)
+    _options(stf, dataflow=1, trsm=3)
     assert info == 0
     Lo, _ = oracle.potrf(synth.spd_matrix(1, 2048))
     assert relF(M.to_dense().numpy(), Lo) <= 1e-10
@@ -54,7 +54,7 @@ def _reset_options(request):
     yield
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
-        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=2, threads=8, lookahead=1, trsm_split=4, push=0)
+        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=3, threads=8, lookahead=1, trsm_split=4, push=0)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
