@@ -346,8 +346,13 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
            "alone_tile": kern.get("gemm_tile"), "alone_full_occupancy": kern.get("gemm_full"),
            "traffic_bytes_per_tile_launch": tr, "algorithmic_bytes_per_tile_launch": 4 * nb * nb * 8}
     roof["dominant_kernel"] = dom
-    roof["traffic_note"] = ("the launch unit is the whole-DAG graph; per-kernel DRAM traffic is in "
-                            "dominant_kernel (ncu --set full, profiles/gemm_traffic.json)")
+    gt = load_graph_traffic(n, nb) if ndev == 1 else None
+    if gt:
+        roof["traffic"] = gt["traffic_bytes"]
+        roof["traffic_src"] = gt["src"]
+    roof["traffic_note"] = ("traffic = DRAM bytes of one whole-DAG graph launch (ncu --graph-profiling graph, "
+                            "committed under profiles/); algorithmic minimum 8.86 GB at n=32768 (lower tiles read "
+                            "and written once); per-kernel DRAM traffic of the GEMM tile in dominant_kernel")
 
     cpu = None
     if N == 1 and not args.no_cpu:
@@ -414,6 +419,20 @@ def e2e_run(stf, n, nb, N, args):
             "ms_per_step": round(dev_ms, 3), "host_wall_ms_per_step": round(wall_ms, 3),
             "api": "stf_potrf(STF_DESC_HOST_COLMAJOR, pinned), lower tiles copied in and written back as tasks",
             "steps": len(times)}
+
+
+def load_graph_traffic(n, nb):
+    """DRAM bytes of one whole-DAG graph launch at (n, nb), from the newest committed ncu summary."""
+    import glob
+
+    best = None
+    for p in sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", "graph_traffic_n%d_nb%d*.json" % (n, nb)))):
+        try:
+            d = json.load(open(p))
+            best = {"traffic_bytes": d["traffic_bytes"], "src": os.path.relpath(p, ROOT)}
+        except (OSError, ValueError, KeyError):
+            pass
+    return best
 
 
 def load_traffic():

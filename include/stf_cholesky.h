@@ -102,8 +102,9 @@ const char *stf_last_error(void);
  *   "trsm_split" STF_TRSM_SPLIT P in [1,16]: non-critical row-panel TRSMs run right-looking
  *                           over P column blocks (panel kernel + GEMM updates; default 4);
  *                           1: one panel launch
- *   "trsm_res_tail" STF_TRSM_RES_TAIL R >= 0: with trsm 3, TRSM(i,k) of the last R panel
- *                           steps (T - k <= R) also use the resident panel (default 16)
+ *   "trsm_res_tail" STF_TRSM_RES_TAIL C >= 0: with trsm 3, every TRSM(i,k) of a panel step
+ *                           whose trailing order n - k nb <= C uses the resident panel (there
+ *                           the factorisation is latency-bound; default 8192)
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA
  *                           graph, memoised per (n, nb, grid, tiles) (default);
  *                           0: eager lowering on streams + events

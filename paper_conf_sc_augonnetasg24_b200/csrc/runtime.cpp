@@ -90,7 +90,7 @@ struct Options {
   int64_t threads = 8;  // eager backend: host submission threads (one per slot group)
   int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
   int64_t mem_cap_tiles = 0;  // HOST_COLMAJOR on one GPU: device tile frames (0 = whole matrix resident)
-  int64_t trsm_res_tail = 16;  // trsm 3: non-critical TRSM(i,k) also resident-panel when T - k <= this
+  int64_t trsm_res_tail = 8192;  // trsm 3: every TRSM(i,k) resident-panel once the trailing order n - k nb <= this
 };
 
 // options that change the plan or its lowering (part of the memo key)
@@ -270,7 +270,7 @@ struct Lowerer {
                    "TRSM what-if");
           return 0;
         }
-        if (X.opt.trsm == 3 && (t.i == t.k + 1 || X.n / nb - t.k <= X.opt.trsm_res_tail) &&
+        if (X.opt.trsm == 3 && (t.i == t.k + 1 || X.n - t.k * nb <= X.opt.trsm_res_tail) &&
             stfk::trsm_res_supported((int)nb, X.buf[(size_t)t.in[0]], nb)) {
           // the next panel's TRSM(k+1,k) is on the critical path, and near the end of the
           // factorisation every TRSM is latency-bound: the resident-panel kernel (16 rows per
@@ -867,7 +867,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.dataflow = env_int("STF_DATAFLOW", 1);
   C.opt.trsm = env_int("STF_TRSM", 3);
   C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 4);
-  C.opt.trsm_res_tail = env_int("STF_TRSM_RES_TAIL", 16);
+  C.opt.trsm_res_tail = env_int("STF_TRSM_RES_TAIL", 8192);
   C.opt.push = env_int("STF_PUSH", 0);
   C.opt.mem_cap_tiles = env_int("STF_MEM_CAP_TILES", 0);
   C.opt.streams = env_int("STF_STREAMS", 8);
