@@ -36,6 +36,7 @@
 #include <vector>
 
 #include "ptx.cuh"
+#include "solve_block.cuh"
 #include "tile_ops.hpp"
 
 namespace stfk {
@@ -45,7 +46,8 @@ constexpr int W = 64;       // block order
 constexpr int LDO = 68;     // smem stride of DMMA operand blocks [k][row] (68 = 4 mod 16: conflict-free)
 constexpr int LDB = 65;     // smem stride of substitution / Cholesky blocks [row][col]
 constexpr int NT = 256;
-constexpr int SMEM_BYTES = 2 * W * LDO * 8;  // 69,632 B
+// critical CTA: D [W][LDB] + XS [W][LDO] + Rc [W] + 4 swizzled 16-row panels + Y [W]
+constexpr int SMEM_BYTES = (W * LDB + W * LDO + W + 4 * 16 * W + W) * 8;  // 103,168 B
 enum : uint32_t { T_P = 0, T_S = 1, T_U = 2 };
 
 __host__ __device__ inline uint32_t enc(uint32_t t, uint32_t i, uint32_t j, uint32_t k) {
@@ -299,6 +301,98 @@ __device__ __forceinline__ void chol_core(double (&a)[16], double* S, double* Lc
   __syncthreads();
 }
 
+// P of a full 64 x 64 diagonal block held row-major in D (lower part, LDB stride),
+// in place, latency-optimised for the critical chain.  8 panels of 8 columns:
+//   (a) warp 0 factors the panel: every lane factors the 8 x 8 diagonal block
+//       redundantly in registers (no shuffles on the sqrt -> reciprocal -> divide
+//       chain) and the two rows it owns below it (lane, lane + 32);
+//   (b) six warps on the other SM sub-partitions apply the panel to the trailing
+//       lower block on DMMA (K = 8), so the chain warp's FP64 pipe stays free.
+// Correctly rounded sqrt and division (div_by with y = RN(1/s)); every element
+// receives its updates in increasing column order, each a single fma or a DMMA
+// k-step pair, deterministic.  Non-positive pivot (or NaN): info = min(info,
+// col0 + col + 1), s = NaN.
+__device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
+  constexpr int LD = df::LDB;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
+  int bad = 0;
+#pragma unroll 1
+  for (int p = 0; p < 8; ++p) {
+    const int c0 = 8 * p;
+    if (warp == 0) {
+      double dg[8][8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j <= i; ++j) dg[i][j] = D[(c0 + i) * LD + c0 + j];
+      const int r1 = lane, r2 = lane + 32;
+      const bool b1 = r1 >= c0 + 8, b2 = r2 >= c0 + 8;
+      double v1[8], v2[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
+        v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const double d = dg[i][i];
+        const bool ok = d > 0.0;
+        if (!ok && bad == 0) bad = c0 + i + 1;
+        const double sq = ok ? sqrt(d) : kNaN, y = 1.0 / sq;
+        dg[i][i] = sq;
+#pragma unroll
+        for (int r = i + 1; r < 8; ++r) dg[r][i] = div_by(dg[r][i], sq, y);
+#pragma unroll
+        for (int r = i + 1; r < 8; ++r)
+#pragma unroll
+          for (int c = i + 1; c <= r; ++c) dg[r][c] = fma(-dg[r][i], dg[c][i], dg[r][c]);
+        v1[i] = div_by(v1[i], sq, y);
+        v2[i] = div_by(v2[i], sq, y);
+#pragma unroll
+        for (int c = i + 1; c < 8; ++c) {
+          v1[c] = fma(-v1[i], dg[c][i], v1[c]);
+          v2[c] = fma(-v2[i], dg[c][i], v2[c]);
+        }
+      }
+      if (lane == 0) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j <= i; ++j) D[(c0 + i) * LD + c0 + j] = dg[i][j];
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        if (b1) D[r1 * LD + c0 + j] = v1[j];
+        if (b2) D[r2 * LD + c0 + j] = v2[j];
+      }
+    }
+    __syncthreads();
+    if (p < 7 && warp != 0 && warp != 4) {  // trailing lower block, rows and columns >= c0 + 8
+      const int mw = warp < 4 ? warp - 1 : warp - 2;  // 0..5
+      const int nf = 7 - p, npairs = nf * (nf + 1) / 2;
+      for (int idx = mw; idx < npairs; idx += 6) {
+        int fi = 0;
+        while ((fi + 1) * (fi + 2) / 2 <= idx) ++fi;
+        const int fj = idx - fi * (fi + 1) / 2;
+        const int R0 = c0 + 8 + 8 * fi, C0 = c0 + 8 + 8 * fj;
+        double* cp = D + (R0 + g) * LD + C0 + 2 * t;
+        double acc0 = cp[0], acc1 = cp[1];
+#pragma unroll
+        for (int ks = 0; ks < 2; ++ks) {
+          const double a = D[(R0 + g) * LD + c0 + 4 * ks + t];
+          const double b = negd(D[(C0 + g) * LD + c0 + 4 * ks + t]);
+          dmma_8x8x4(acc0, acc1, a, b);
+        }
+        cp[0] = acc0;
+        cp[1] = acc1;
+      }
+    }
+    __syncthreads();
+  }
+  if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
+}
+
 // interleaved-column register blocks (chol_core layout): v[m] = G(r, 4m + q)
 __device__ __forceinline__ void load_il(double (&v)[16], const double* G, int64_t ldg, int rows, int nc, bool lower) {
   const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
@@ -387,7 +481,18 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
     double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
     // ---- P(kb)
     DF_STAMP(6 * kb + 0);
-    chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
+    if (nk == W) {
+      if (kb == 0) {  // P(0) input: nothing precedes it
+        for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+          const int rr = idx & (W - 1), cc = idx >> 6;
+          if (rr >= cc) D[rr * df::LDB + cc] = __ldcg(Xkk + (int64_t)cc * p.ldx + rr);
+        }
+        __syncthreads();
+      }
+      chol_block(D, p.col0 + (int64_t)kb * W, p.info);
+    } else {
+      chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
+    }
     store_block_rm(D, df::LDB, Xkk, p.ldx, nk, nk, true);
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -402,11 +507,36 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
     if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + kb], kb);
     __syncthreads();
     DF_STAMP(6 * kb + 2);
-    double b[16];
-    load_chunk(b, Xik, p.ldx, rows, nk, false);
-    solve_core(b, D, Rc, XS, df::LDO, nk);
-    store_chunk(b, Xik, p.ldx, rows, nk, false);
-    __syncthreads();
+    if (nk == W) {
+      // four warps, one per SM sub-partition, each solve 16 rows (solve_block: 8-column
+      // sub-blocks by substitution, their updates on DMMA; the FP64 pipes of the
+      // sub-partitions work in parallel), then the result goes to XS for U
+      double* Xp = Rc + W;        // 4 x [16 x 64] swizzled panels
+      double* Yc = Xp + 4 * 16 * W;  // 1 / L_cc (IEEE)
+      for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+        const int rr = idx & (W - 1), cc = idx >> 6;
+        Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)] = rr < rows ? __ldcg(Xik + (int64_t)cc * p.ldx + rr) : 0.0;
+      }
+      if (threadIdx.x < W) Yc[threadIdx.x] = 1.0 / D[threadIdx.x * df::LDB + threadIdx.x];
+      __syncthreads();
+      if (warp < 4) {
+        const int rr = 16 * warp + (lane & 15);
+        solve_block<0>(Xp + warp * 16 * W, 0, sb::RowMajor<df::LDB>{D}, Yc, lane, Xik, p.ldx, rr,
+                       lane < 16 && rr < rows);
+      }
+      __syncthreads();
+      for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+        const int m = idx >> 6, k = idx & (W - 1);
+        XS[m * df::LDO + k] = Xp[(m >> 4) * 16 * W + sb::xo(m & 15, k)];
+      }
+      __syncthreads();
+    } else {
+      double b[16];
+      load_chunk(b, Xik, p.ldx, rows, nk, false);
+      solve_core(b, D, Rc, XS, df::LDO, nk);
+      store_chunk(b, Xik, p.ldx, rows, nk, false);
+      __syncthreads();
+    }
     if (threadIdx.x == 0) {
       __threadfence();
       st_release(&prog[ib * p.Nb + kb], kb + 1);

@@ -32,6 +32,7 @@
 #include <cstdlib>
 
 #include "ptx.cuh"
+#include "solve_block.cuh"
 #include "tile_ops.hpp"
 
 namespace stfk {
@@ -46,6 +47,8 @@ __device__ __forceinline__ void tr_stamp(unsigned long long* trace, int idx) {
 }
 
 namespace tr {
+using sb::xo;
+using sb::poff;
 constexpr int R = 16;        // rows per CTA (one 128-byte line per column of the panel)
 constexpr int W = 64;        // column block
 constexpr int NMAX = 1024;   // resident panel limit (NMAX * 128 B = 128 KB)
@@ -61,12 +64,6 @@ constexpr int BAR_MMA = 1, BAR_READY = 2, BAR_SOLVED = 3;
 __host__ __device__ constexpr size_t smem_bytes(int n) {
   return 1024 + ((size_t)16 * n + (size_t)NST * STAGE + 2 * DP + 2 * W) * sizeof(double) + 2 * NST * 8;
 }
-// offset of diagonal-block element (r, c), r >= c, in the packed column-major lower triangle
-__device__ __forceinline__ int poff(int r, int c) { return c * W - (c * (c - 1)) / 2 + (r - c); }
-// panel element (r, c): column c is one 128-byte line of 16 rows, 16-byte chunks
-// XOR-swizzled by c & 7 (the TMA 128B pattern), so DMMA fragment loads with the
-// k-permutation k = 8 grp + 2 t + kh are conflict-free
-__device__ __forceinline__ int xo(int r, int c) { return c * 16 + ((((r >> 1) ^ (c & 7)) << 1) | (r & 1)); }
 // L stage element (k, c) written by TMA boxes of [BK][16 c] with the 128B swizzle
 __device__ __forceinline__ int lo(int k, int c) {
   return (c >> 4) * BOXD + k * 16 + (((((c & 15) >> 1) ^ (k & 7)) << 1) | (c & 1));
@@ -91,84 +88,6 @@ __device__ __forceinline__ double ld_cg_early(const double* p) {  // volatile: i
   double v;
   asm volatile("ld.global.cg.f64 %0, [%1];" : "=d"(v) : "l"(p));
   return v;
-}
-
-// Substitution of one 16 x 64 block X <- X L^-T (L = the diagonal block) by the
-// solver warp, in 8 sub-blocks of 8 columns P = 0..7:
-//   (a) lane r < 16 solves row r of sub-block P in registers: x_c = b_c / L_cc
-//       (correctly rounded: div_by with y = RN(1 / L_cc)), b_j -= x_c L_jc (lanes
-//       16..31 repeat rows 0..15 without storing);
-//   (b) the later sub-blocks Q > P are updated on the DMMA pipe:
-//       X[:, Q] -= X[:, P] L[Q, P]^T  (16 x 8 x 8 per Q, fragments from the panel).
-// A DFMA warp instruction costs the FP64 pipe of the sub-partition ~4 clocks for 16
-// useful FMAs here, a DMMA 16 clocks for 256 (tools/solve_lab.cu), so the
-// sub-block updates - 7/8 of the FMAs - run 4x faster on the DMMA path.
-// Every sum keeps a fixed order; results are deterministic.
-template <int P>
-__device__ __forceinline__ void solve_block(double* Xs, int c0, const double* D, const double* Y, int lane,
-                                            double* X, int64_t ldx, int64_t xrow, bool wr) {
-  using namespace tr;
-  if constexpr (P < 8) {
-    const int r = lane & 15;
-    const int cb = c0 + 8 * P;
-    // (a) serial substitution of the 8 columns of sub-block P
-    double b[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) b[i] = Xs[xo(r, cb + i)];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      const int c = 8 * P + i;
-      const double x = div_by(b[i], D[poff(c, c)], Y[c]);
-      b[i] = x;
-#pragma unroll
-      for (int i2 = i + 1; i2 < 8; ++i2) b[i2] = fma(-x, D[poff(8 * P + i2, c)], b[i2]);
-    }
-    if (lane < 16) {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) Xs[xo(r, cb + i)] = b[i];
-    }
-    if (wr) {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) X[(int64_t)(cb + i) * ldx + xrow] = b[i];
-    }
-    __syncwarp();
-    // (b) X[:, Q] -= X[:, P] L[Q, P]^T for Q > P, all DMMAs issued before the stores
-    if constexpr (P < 7) {
-      const int g = lane >> 2, t = lane & 3;
-      double a[2][2];
-#pragma unroll
-      for (int mi = 0; mi < 2; ++mi)
-#pragma unroll
-        for (int ks = 0; ks < 2; ++ks) a[mi][ks] = Xs[xo(8 * mi + g, cb + 4 * ks + t)];
-      double acc[7 - P][2][2];
-#pragma unroll
-      for (int q = 0; q < 7 - P; ++q) {
-        const int Q = P + 1 + q;
-        double bq[2];
-#pragma unroll
-        for (int ks = 0; ks < 2; ++ks) {  // B[k][n] = L(8Q + n, 8P + k), negated: acc = C - A B^T
-          const double v = D[poff(8 * Q + g, 8 * P + 4 * ks + t)];
-          bq[ks] = __longlong_as_double(__double_as_longlong(v) ^ (long long)0x8000000000000000ULL);
-        }
-#pragma unroll
-        for (int mi = 0; mi < 2; ++mi) {
-          acc[q][mi][0] = Xs[xo(8 * mi + g, c0 + 8 * Q + 2 * t)];
-          acc[q][mi][1] = Xs[xo(8 * mi + g, c0 + 8 * Q + 2 * t + 1)];
-#pragma unroll
-          for (int ks = 0; ks < 2; ++ks) dmma_8x8x4(acc[q][mi][0], acc[q][mi][1], a[mi][ks], bq[ks]);
-        }
-      }
-#pragma unroll
-      for (int q = 0; q < 7 - P; ++q)
-#pragma unroll
-        for (int mi = 0; mi < 2; ++mi) {
-          Xs[xo(8 * mi + g, c0 + 8 * (P + 1 + q) + 2 * t)] = acc[q][mi][0];
-          Xs[xo(8 * mi + g, c0 + 8 * (P + 1 + q) + 2 * t + 1)] = acc[q][mi][1];
-        }
-      __syncwarp();
-    }
-    solve_block<P + 1>(Xs, c0, D, Y, lane, X, ldx, xrow, wr);
-  }
 }
 
 // Warp roles are pinned to SM sub-partitions (warp w runs on w % 4): the FP64 pipe
@@ -243,7 +162,7 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
         const int tm = mw * 32 + lane;  // 0..191
         for (int idx = tm; idx < W * W; idx += MMA_THREADS) {
           const int rr = idx & (W - 1), cc = idx >> 6;
-          if (rr >= cc) cpa8(dst + tr::poff(rr, cc), src + (int64_t)cc * ldl + rr);
+          if (rr >= cc) cpa8(dst + sb::poff(rr, cc), src + (int64_t)cc * ldl + rr);
         }
         cpa_commit();
       }
@@ -364,13 +283,13 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
       bar_sync_n(BAR_READY, MMA_THREADS + SOLVE_THREADS);  // X[:, jb] updated; L(jb,jb) staged
       {  // IEEE reciprocals of the 64 pivots (two per lane)
         double* Yw = Rc + (jb & 1) * W;
-        const double d0 = D[tr::poff(lane, lane)], d1 = D[tr::poff(lane + 32, lane + 32)];
+        const double d0 = D[sb::poff(lane, lane)], d1 = D[sb::poff(lane + 32, lane + 32)];
         Yw[lane] = 1.0 / d0;
         Yw[lane + 32] = 1.0 / d1;
         __syncwarp();
       }
       if (lane == 0) tr_stamp(trace, 5 * jb + 4);
-      solve_block<0>(Xs, c0, D, Y, lane, X, ldx, r0 + r, wr);
+      solve_block<0>(Xs, c0, sb::Packed{D}, Y, lane, X, ldx, r0 + r, wr);
       if (mir.n > 0 && wr) {  // fused push (NEXT-3): the finished block into the consumers' replicas
 #pragma unroll 1
         for (int m = 0; m < mir.n && m < 7; ++m) {
