@@ -19,9 +19,17 @@
 #include <cstdlib>
 
 #include "ptx.cuh"
+#include "solve_block.cuh"
 #include "tile_ops.hpp"
 
 namespace stfk {
+
+// diagonal block staged transposed: LdT[c * LD + r] = L(r, c)
+template <int LD>
+struct ColT {
+  const double* p;
+  __device__ __forceinline__ double operator()(int r, int c) const { return p[c * LD + r]; }
+};
 
 // Rows per CTA: 32 (3 stages, latency) or 64 (2 stages, higher DMMA efficiency).
 template <int BM_>
@@ -174,59 +182,95 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
     cp_async_wait<0>();
     __syncthreads();  // ring free
     if (jb + 1 < Nb) prologue_pre(jb + 1);
-    // ---- diagonal solve: S[r][c] = acc, LdT = L(jb,jb) (landed: waited above), Rc[c] = 1 / L_cc
+    // ---- diagonal solve, LdT = L(jb,jb) (landed: waited above), Rc[c] = 1 / L_cc
+    if (nc == tp::W) {
+      // full block: BM/16 warps, one per SM sub-partition, each solve 16 rows
+      // (solve_block: 8-column sub-blocks by substitution, their updates on DMMA)
+      double* Xp = S;  // BM/16 swizzled [16 x 64] panels (S is free here)
 #pragma unroll
-    for (int i = 0; i < tp::FM; ++i)
+      for (int i = 0; i < tp::FM; ++i)
 #pragma unroll
-      for (int j = 0; j < 2; ++j)
+        for (int j = 0; j < 2; ++j)
 #pragma unroll
-        for (int h = 0; h < 2; ++h) S[(wm0 + 8 * i + g) * tp::SS + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
-    if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / LdT[threadIdx.x * tp::SL + threadIdx.x];
-    __syncthreads();
-    // thread (q = tid / BM, r = tid % BM), q < 4, owns row r of the 16-column chunk q.
-    // Chunk q solves its columns in registers, publishes x to S, later chunks
-    // subtract its contribution.
-    const int q = threadIdx.x / tp::BM, r = threadIdx.x % tp::BM;
-    double b[16];
-    if (q < 4) {
+          for (int h = 0; h < 2; ++h) {
+            const int row = wm0 + 8 * i + g, col = wn0 + 8 * j + 2 * t + h;
+            Xp[(row >> 4) * 16 * tp::W + sb::xo(row & 15, col)] = acc[i][j][h];
+          }
+      if (threadIdx.x < tp::W) Rc[threadIdx.x] = 1.0 / LdT[threadIdx.x * tp::SL + threadIdx.x];
+      __syncthreads();
+      if (warp < tp::BM / 16) {
+        const int rr = 16 * warp + (lane & 15);
+        solve_block<0>(Xp + warp * 16 * tp::W, 0, ColT<tp::SL>{LdT}, Rc, lane, X + (int64_t)c0 * ldx + r0, ldx, rr,
+                       lane < 16 && rr < rows);
+      }
+      if (mir.n > 0) {  // fused push (NEXT-3): the finished block into the consumers' replicas
+        __syncthreads();
+        for (int idx = threadIdx.x; idx < tp::BM * tp::W; idx += tp::NT) {
+          const int rr = idx % tp::BM, cc = idx / tp::BM;
+          if (rr < rows) {
+            const double v = Xp[(rr >> 4) * 16 * tp::W + sb::xo(rr & 15, cc)];
+            const int64_t off = (int64_t)(c0 + cc) * ldx + r0 + rr;
 #pragma unroll
-      for (int c = 0; c < 16; ++c) b[c] = S[r * tp::SS + 16 * q + c];
-    }
-    for (int qq = 0; qq < 4; ++qq) {
-      if (q == qq) {
-#pragma unroll
-        for (int c = 0; c < 16; ++c) {
-          const int col = 16 * qq + c;
-          if (col < nc) {
-            b[c] = div_by(b[c], LdT[col * tp::SL + col], Rc[col]);
-#pragma unroll
-            for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], LdT[col * tp::SL + 16 * qq + c2], b[c2]);
+            for (int m = 0; m < 7; ++m)
+              if (m < mir.n) mir.p[m][off] = v;
           }
         }
-#pragma unroll
-        for (int c = 0; c < 16; ++c) S[r * tp::SS + 16 * qq + c] = b[c];
       }
+    } else {
+      // ragged last block: row-chunked substitution, S[r][c] = acc
+  #pragma unroll
+      for (int i = 0; i < tp::FM; ++i)
+  #pragma unroll
+        for (int j = 0; j < 2; ++j)
+  #pragma unroll
+          for (int h = 0; h < 2; ++h) S[(wm0 + 8 * i + g) * tp::SS + wn0 + 8 * j + 2 * t + h] = acc[i][j][h];
+      if (threadIdx.x < nc) Rc[threadIdx.x] = 1.0 / LdT[threadIdx.x * tp::SL + threadIdx.x];
       __syncthreads();
-      if (q > qq && q < 4) {
-#pragma unroll
-        for (int cc = 0; cc < 16; ++cc)
-#pragma unroll
-          for (int c = 0; c < 16; ++c)
-            b[cc] = fma(-S[r * tp::SS + 16 * qq + c], LdT[(16 * qq + c) * tp::SL + 16 * q + cc], b[cc]);
+      // thread (q = tid / BM, r = tid % BM), q < 4, owns row r of the 16-column chunk q.
+      // Chunk q solves its columns in registers, publishes x to S, later chunks
+      // subtract its contribution.
+      const int q = threadIdx.x / tp::BM, r = threadIdx.x % tp::BM;
+      double b[16];
+      if (q < 4) {
+  #pragma unroll
+        for (int c = 0; c < 16; ++c) b[c] = S[r * tp::SS + 16 * q + c];
       }
-    }
-    if (q < 4 && r < rows) {
-#pragma unroll
-      for (int c = 0; c < 16; ++c) {
-        const int col = 16 * q + c;
-        if (col < nc) {
-          const int64_t off = (int64_t)(c0 + col) * ldx + r0 + r;
-          X[off] = b[c];
-          // fused push (NEXT-3): the finished value also goes straight into the
-          // consumers' replicas (peer memory over NVLink / another slot's arena)
-#pragma unroll
-          for (int m = 0; m < 7; ++m)
-            if (m < mir.n) mir.p[m][off] = b[c];
+      for (int qq = 0; qq < 4; ++qq) {
+        if (q == qq) {
+  #pragma unroll
+          for (int c = 0; c < 16; ++c) {
+            const int col = 16 * qq + c;
+            if (col < nc) {
+              b[c] = div_by(b[c], LdT[col * tp::SL + col], Rc[col]);
+  #pragma unroll
+              for (int c2 = c + 1; c2 < 16; ++c2) b[c2] = fma(-b[c], LdT[col * tp::SL + 16 * qq + c2], b[c2]);
+            }
+          }
+  #pragma unroll
+          for (int c = 0; c < 16; ++c) S[r * tp::SS + 16 * qq + c] = b[c];
+        }
+        __syncthreads();
+        if (q > qq && q < 4) {
+  #pragma unroll
+          for (int cc = 0; cc < 16; ++cc)
+  #pragma unroll
+            for (int c = 0; c < 16; ++c)
+              b[cc] = fma(-S[r * tp::SS + 16 * qq + c], LdT[(16 * qq + c) * tp::SL + 16 * q + cc], b[cc]);
+        }
+      }
+      if (q < 4 && r < rows) {
+  #pragma unroll
+        for (int c = 0; c < 16; ++c) {
+          const int col = 16 * q + c;
+          if (col < nc) {
+            const int64_t off = (int64_t)(c0 + col) * ldx + r0 + r;
+            X[off] = b[c];
+            // fused push (NEXT-3): the finished value also goes straight into the
+            // consumers' replicas (peer memory over NVLink / another slot's arena)
+  #pragma unroll
+            for (int m = 0; m < 7; ++m)
+              if (m < mir.n) mir.p[m][off] = b[c];
+          }
         }
       }
     }
