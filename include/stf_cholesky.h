@@ -105,10 +105,13 @@ const char *stf_last_error(void);
  *   "trsm_res_tail" STF_TRSM_RES_TAIL C >= 0: with trsm 3, every TRSM(i,k) of a panel step
  *                           whose trailing order n - k nb <= C uses the resident panel (there
  *                           the factorisation is latency-bound; default 8192)
+ *   "trsm_rows" STF_TRSM_ROWS 32, 64 or 128 (default): rows per CTA of the non-critical
+ *                           row-panel TRSM launches (128: two substitution chains per SM
+ *                           sub-partition, full 64-column blocks only, else 64; same bits)
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA
  *                           graph, memoised per (n, nb, grid, tiles) (default);
  *                           0: eager lowering on streams + events
- *   "streams"  STF_STREAMS  bulk compute streams per GPU slot (default 8)
+ *   "streams"  STF_STREAMS  bulk compute streams per GPU slot (default 32; the pool is sized at init)
  *   "serial"   STF_SERIAL   1: every task on one stream in program order (race check)
  *   "priority" STF_PRIO     1: critical-path tasks on high-priority streams (default 1)
  *   "grid_p"   STF_GRID     rows P of the P x Q grid for COLMAJOR kinds (0 = auto)
@@ -215,6 +218,14 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
  * ready, U done), T = ceil(n/64); trace[6T + 3t ..] the claim / inputs-ready /
  * done stamps of bulk ticket t (0 if unused).  Returns the number of entries
  * written (<= cap) or a negative error.  Not part of the factorisation. */
+/* Debug timeline of the last stf_potrf on one GPU slot, recorded when the
+ * environment had STF_DEBUG_TRACE=1 at plan build (a one-thread stamp kernel
+ * before and after every task on its stream; perturbs timing slightly).  Writes
+ * up to cap_tasks records of 7 int64 (kind as in stf_dag_build, i, j, k, stream index,
+ * %globaltimer ns at start, at end) in program order; returns the number of
+ * tasks of the call (0 if it was not traced). */
+int64_t stf_debug_last_trace(int64_t *out, int64_t cap_tasks);
+
 int64_t stf_debug_potrf_trace(int64_t n, double *A, int64_t lda, int ctas, int64_t *trace, int64_t cap);
 
 /* Debug timeline of the resident-panel TRSM kernel (B[M x n] <- B L^-T, device

@@ -58,7 +58,7 @@ EXPORTS = [
     "stf_cholesky_init", "stf_potrf", "stf_finalize", "stf_last_error",
     "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_infer_edges",
     "stf_fill_spd_tiles", "stf_fill_spd_block",
-    "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace",
+    "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace", "stf_debug_last_trace",
     "stf_debug_trsm_trace",
     "stf_dag_tasks_io", "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
 ]
@@ -103,6 +103,7 @@ stf_mp_blob_size = _decl("stf_mp_blob_size", _i64, [])
 stf_mp_prepare = _decl("stf_mp_prepare", _int, [_i64, _i64, _P(stf_matrix_desc), _vp])
 stf_mp_import = _decl("stf_mp_import", _int, [_vp])
 stf_mp_potrf = _decl("stf_mp_potrf", _int, [])
+stf_debug_last_trace = _decl("stf_debug_last_trace", _i64, [_P(_i64), _i64])
 stf_debug_potrf_trace = _decl("stf_debug_potrf_trace", _i64, [_i64, _vp, _i64, _int, _P(_i64), _i64])
 stf_debug_trsm_trace = _decl("stf_debug_trsm_trace", _i64, [_i64, _i64, _vp, _i64, _vp, _i64, _P(_i64), _i64])
 

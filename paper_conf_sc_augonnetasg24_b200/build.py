@@ -20,7 +20,7 @@ LIB = os.path.join(HERE, "libstf_cholesky.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
-          "-I" + os.path.join(ROOT, "include"), "-I" + CSRC]
+          "-I" + os.path.join(ROOT, "include"), "-I" + CSRC] + os.environ.get("STF_NVCC_DEFS", "").split()
 
 SOURCES = [
     "kernels/gemm_dmma.cu",

@@ -31,18 +31,21 @@ struct ColT {
   __device__ __forceinline__ double operator()(int r, int c) const { return p[c * LD + r]; }
 };
 
-// Rows per CTA: 32 (3 stages, latency) or 64 (2 stages, higher DMMA efficiency).
-template <int BM_>
+// Rows per CTA: 32 (3 stages, latency), 64 (2 stages, higher DMMA efficiency) or
+// 128 (2 half-depth stages: eight solver warps, two per SM sub-partition, so two
+// substitution chains interleave on each FP64 pipe; full 64-column blocks only).
+// A pipeline stage holds KD of the 64 k-columns of one update block.
+template <int BM_, int KD_ = 64>
 struct TP {
-  static constexpr int BM = BM_, W = 64, NT = 256, STAGES = (BM_ == 32) ? 3 : 2;
+  static constexpr int BM = BM_, W = 64, NT = 256, STAGES = (BM_ == 32) ? 3 : 2, KD = KD_, R = 64 / KD_;
   static constexpr int SA = BM + 4;  // As[k][m] stride (= 4 mod 16 -> conflict-free fragment loads)
   static constexpr int SB = 68;      // Bs[k][n] stride
   static constexpr int SS = 65;      // solve scratch stride
   static constexpr int SL = 66;      // LdT stride (16-byte aligned columns for cp.async; warp-broadcast reads)
   static constexpr int FM = BM / 16; // m-fragments per warp (2 x 4 warp grid, warp tile BM/2 x 16)
-  static constexpr int STAGE = W * SA + W * SB;                     // doubles per pipeline stage
+  static constexpr int STAGE = KD * SA + KD * SB;                   // doubles per pipeline stage
   static constexpr int SOLVE = BM * SS + W * SL + W;                // S, LdT, Rc
-  static constexpr int SMEM_BYTES = (STAGES * STAGE + SOLVE) * 8;  // ~210 KB / ~207 KB
+  static constexpr int SMEM_BYTES = (STAGES * STAGE + SOLVE) * 8;  // ~210 / ~207 / ~203 KB
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
@@ -57,31 +60,31 @@ __device__ __forceinline__ double negd_tp(double x) {
   return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
 }
 
-// dst[k * ld + r] = G(r, k) for r < rows (<= R), k < kc (<= W); zero-filled otherwise.
+// dst[k * ld + r] = G(r, k) for r < rows (<= R), k < kc (<= KD); zero-filled otherwise.
 // Fast path (full block, 16-byte aligned columns) uses cp.async; else scalar loads.
-template <int R>
+template <int R, int KD = 64>
 __device__ __forceinline__ void stage_block(double* dst, int ld, const double* G, int64_t ldg, int rows, int kc,
                                             bool fast) {
-  using tp = TP<32>;
+  constexpr int NT = 256;
   if (fast) {
     constexpr int CH = R / 2;  // 16-byte chunks per column
-    for (int idx = threadIdx.x; idx < CH * tp::W; idx += tp::NT) {
+    for (int idx = threadIdx.x; idx < CH * KD; idx += NT) {
       const int k = idx / CH, c = idx % CH;
       cp_async16(dst + k * ld + 2 * c, G + (int64_t)k * ldg + 2 * c);
     }
   } else {
-    for (int idx = threadIdx.x; idx < R * tp::W; idx += tp::NT) {
+    for (int idx = threadIdx.x; idx < R * KD; idx += NT) {
       const int k = idx / R, r = idx % R;
       dst[k * ld + r] = (r < rows && k < kc) ? __ldcg(G + (int64_t)k * ldg + r) : 0.0;
     }
   }
 }
 
-template <int BMT>
+template <int BMT, int KDT = 64>
 __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __restrict__ L, int64_t ldl, int n,
                                                              double* __restrict__ X, int64_t ldx, int M,
                                                              const Mirrors mir) {
-  using tp = TP<BMT>;
+  using tp = TP<BMT, KDT>;
   extern __shared__ __align__(16) double smt[];
   const int r0 = blockIdx.x * tp::BM;
   const int rows = min(tp::BM, M - r0);
@@ -95,18 +98,20 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
   double* LdT = S + tp::BM * tp::SS;         // LdT[p * SL + c] = L(c0 + c, c0 + p); upper part unused
   double* Rc = LdT + tp::W * tp::SL;
 
-  // Stage (jb, pb) = operands of the update of column block jb by block pb; it
-  // lives in ring slot pb % STAGES and is one cp.async group.  X block pb may be
-  // staged only after it has been solved, so the first STAGES-1 stages of jb+1
-  // are issued in two halves: those with pb < jb before the solve of jb (overlapping
-  // their latency with it), the one with pb == jb after it.  Every prologue commits
-  // exactly STAGES-1 groups and every update iteration one group.
-  auto issue = [&](int jb, int pb) {
+  // Stage (jb, s) = operands of the update of column block jb by k-columns
+  // [s KD, (s + 1) KD) (block pb = s / R); it lives in ring slot s % STAGES and is
+  // one cp.async group.  X block pb may be staged only after it has been solved,
+  // so the first STAGES-1 stages of jb+1 are issued in two halves: those with
+  // pb < jb before the solve of jb (overlapping their latency with it), those
+  // with pb == jb after it.  Every prologue commits exactly STAGES-1 stage groups
+  // (plus the diagonal block's) and every update iteration one group.
+  auto issue = [&](int jb, int s) {
     const int c0 = jb * tp::W, nc = min(tp::W, n - c0);
-    double* As = smt + (pb % tp::STAGES) * tp::STAGE;
-    double* Bs = As + tp::W * tp::SA;
-    stage_block<tp::BM>(As, tp::SA, Xr + (int64_t)pb * tp::W * ldx, ldx, rows, tp::W, rows_fast);
-    stage_block<tp::W>(Bs, tp::SB, L + (int64_t)pb * tp::W * ldl + c0, ldl, nc, tp::W, lal && nc == tp::W);
+    double* As = smt + (s % tp::STAGES) * tp::STAGE;
+    double* Bs = As + tp::KD * tp::SA;
+    stage_block<tp::BM, tp::KD>(As, tp::SA, Xr + (int64_t)s * tp::KD * ldx, ldx, rows, tp::KD, rows_fast);
+    stage_block<tp::W, tp::KD>(Bs, tp::SB, L + (int64_t)s * tp::KD * ldl + c0, ldl, nc, tp::KD,
+                               lal && nc == tp::W);
   };
   // diagonal block L(jb, jb) -> LdT (cp.async when full and aligned)
   auto issue_diag = [&](int jb) {
@@ -126,7 +131,7 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
   };
   auto prologue_pre = [&](int jn) {
     for (int p = 0; p < tp::STAGES - 1; ++p)
-      if (p < jn - 1) {
+      if (p < (jn - 1) * tp::R) {
         issue(jn, p);
         cp_async_commit();
       }
@@ -135,8 +140,8 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
     issue_diag(jn);
     cp_async_commit();
     for (int p = 0; p < tp::STAGES - 1; ++p)
-      if (p >= jn - 1) {
-        if (p < jn) issue(jn, p);
+      if (p >= (jn - 1) * tp::R) {
+        if (p < jn * tp::R) issue(jn, p);
         cp_async_commit();
       }
   };
@@ -157,17 +162,17 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
           const int r = wm0 + 8 * i + g, c = wn0 + 8 * j + 2 * t + h;
           acc[i][j][h] = (r < rows && c < nc) ? __ldcg(Xr + (int64_t)(c0 + c) * ldx + r) : 0.0;
         }
-    // left-looking update over pb < jb, one barrier per stage
-    for (int pb = 0; pb < jb; ++pb) {
+    // left-looking update over the k-columns of blocks pb < jb, one barrier per stage
+    for (int st = 0; st < jb * tp::R; ++st) {
       cp_async_wait<tp::STAGES - 2>();
       __syncthreads();
-      const int pf = pb + tp::STAGES - 1;  // refill the slot consumed at pb - 1
-      if (pf < jb) issue(jb, pf);
+      const int pf = st + tp::STAGES - 1;  // refill the slot consumed at st - 1
+      if (pf < jb * tp::R) issue(jb, pf);
       cp_async_commit();
-      const double* As = smt + (pb % tp::STAGES) * tp::STAGE;
-      const double* Bs = As + tp::W * tp::SA;
+      const double* As = smt + (st % tp::STAGES) * tp::STAGE;
+      const double* Bs = As + tp::KD * tp::SA;
 #pragma unroll 4
-      for (int k0 = 0; k0 < tp::W; k0 += 4) {
+      for (int k0 = 0; k0 < tp::KD; k0 += 4) {
         double a[tp::FM], b[2];
 #pragma unroll
         for (int i = 0; i < tp::FM; ++i) a[i] = As[(k0 + t) * tp::SA + wm0 + 8 * i + g];
@@ -216,7 +221,7 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
           }
         }
       }
-    } else {
+    } else if constexpr (tp::BM <= 64) {
       // ragged last block: row-chunked substitution, S[r][c] = acc
   #pragma unroll
       for (int i = 0; i < tp::FM; ++i)
@@ -285,13 +290,17 @@ cudaError_t trsm_panel_init_attrs() {
                                        TP<32>::SMEM_BYTES);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(trsm_panel_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, TP<64>::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(trsm_panel_kernel<128, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             TP<128, 32>::SMEM_BYTES);
   return e;
 }
 
 static int trsm_rows() {
   static int v = [] {
     const char* e = getenv("STF_TRSM_ROWS");
-    return (e && atoi(e) == 32) ? 32 : 64;
+    const int r = e ? atoi(e) : 64;
+    return (r == 32 || r == 128) ? r : 64;
   }();
   return v;
 }
@@ -301,11 +310,12 @@ cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double
   Mirrors mir{};
   if (mirrors) mir = *mirrors;
   if (M <= 0 || n <= 0) return cudaSuccess;
-  const int bm = rows_per_cta == 32 || rows_per_cta == 64 ? rows_per_cta : trsm_rows();
+  int bm = rows_per_cta == 32 || rows_per_cta == 64 || rows_per_cta == 128 ? rows_per_cta : trsm_rows();
+  if (bm == 128 && n % 64 != 0) bm = 64;  // the 128-row form solves full 64-column blocks only
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((M + bm - 1) / bm);
   cfg.blockDim = dim3(256);
-  cfg.dynamicSmemBytes = bm == 32 ? TP<32>::SMEM_BYTES : TP<64>::SMEM_BYTES;
+  cfg.dynamicSmemBytes = bm == 32 ? TP<32>::SMEM_BYTES : bm == 64 ? TP<64>::SMEM_BYTES : TP<128, 32>::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributePriority;
@@ -314,6 +324,7 @@ cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double
   cfg.numAttrs = 1;
   ++launch_count();
   if (bm == 32) return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<32>, L, ldl, n, B, ldb, M, mir);
+  if (bm == 128) return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<128, 32>, L, ldl, n, B, ldb, M, mir);
   return cudaLaunchKernelEx(&cfg, trsm_panel_kernel<64>, L, ldl, n, B, ldb, M, mir);
 }
 

@@ -131,8 +131,11 @@ struct Builder {
       for (int64_t j = 0; j <= i; ++j) p.buffers.push_back(Buffer{(int32_t)i, (int32_t)j, p.owner(i, j), false});
     (void)NT;
     if (p.opt.with_load) {
-      for (int64_t j = 0; j < T; ++j)
-        for (int64_t i = j; i < T; ++i) {
+      // Tile columns in order (the order in which the panel steps need them), or
+      // tile rows (leading principal blocks first) with load_order = 1.
+      for (int64_t a = 0; a < T; ++a)
+        for (int64_t b = p.opt.load_order ? 0 : a; b < (p.opt.load_order ? a + 1 : T); ++b) {
+          const int64_t i = p.opt.load_order ? a : b, j = p.opt.load_order ? b : a;
           const int own = p.owner(i, j);
           const int64_t w = Plan::tile_id(i, j);
           Task t{K_LOAD, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own), {-1, -1}, w};
@@ -175,7 +178,10 @@ struct Builder {
         for (int64_t i = j; i < T; ++i) {
           const int own = p.owner(i, j);
           const int64_t d = Plan::tile_id(i, j);
-          Task t{K_STORE, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own), {d, -1}, -1};
+          // the other copy stream than the slot's loads: a write-back starts as soon
+          // as its tile is final instead of queueing behind every load
+          Task t{K_STORE, (int32_t)i, (int32_t)j, 0, own, 0, copy_stream(own + (p.opt.store_own_stream ? 1 : 0)),
+                 {d, -1}, -1};
           Access acc[1] = {{d, READ}};
           submit(t, acc, 1);
           p.nstores++;

@@ -82,7 +82,7 @@ struct Options {
   int64_t trsm = 3;      // TRSM tile kernel: 3 resident panel, 2 row-panel, 1 dataflow, 0 recursive
   int64_t trsm_split = 4;  // row panel: non-critical TRSMs as `trsm_split` column blocks (panel + GEMM updates)
   int64_t graph = 1;
-  int64_t streams = 8;
+  int64_t streams = 32;
   int64_t serial = 0;
   int64_t priority = 1;
   int64_t grid_p = 0;
@@ -91,13 +91,15 @@ struct Options {
   int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
   int64_t mem_cap_tiles = 0;  // HOST_COLMAJOR on one GPU: device tile frames (0 = whole matrix resident)
   int64_t trsm_res_tail = 8192;  // trsm 3: every TRSM(i,k) resident-panel once the trailing order n - k nb <= this
+  int64_t trsm_rows = 128;  // row panel: rows per CTA of the non-critical TRSM panels (32, 64 or 128)
 };
 
 // options that change the plan or its lowering (part of the memo key)
 bool same_plan_options(const Options& a, int64_t a_graph, const Options& b) {
   return a.streams == b.streams && a.serial == b.serial && a_graph == b.graph && a.priority == b.priority &&
          a.dataflow == b.dataflow && a.trsm == b.trsm && a.trsm_split == b.trsm_split && a.push == b.push &&
-         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.trsm_res_tail == b.trsm_res_tail;
+         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.trsm_res_tail == b.trsm_res_tail &&
+         a.trsm_rows == b.trsm_rows;
 }
 
 // A plan bound to physical buffers, plus its lowering artefacts.
@@ -124,6 +126,7 @@ struct Exec {
   int64_t graph_nodes = 0;
   int graph_fallback = 0;  // capture failed, eager lowering used
   unsigned skip_mask = 0;  // STF_DEBUG_SKIP: task kinds whose kernels are not launched (timing what-ifs)
+  unsigned long long* trace = nullptr;  // STF_DEBUG_TRACE: per task %globaltimer at start / end (slot 0's device)
   int64_t updates = 0;     // successful cudaGraphExecUpdate re-binds
   bool rebound = false;
   int64_t launches = 0;
@@ -170,6 +173,7 @@ struct Context {
   Options opt;
   std::list<std::unique_ptr<Exec>> cache;  // MRU first
   stf_plan_stats last{};
+  std::vector<int64_t> last_trace;  // STF_DEBUG_TRACE: (kind, i, j, k, stream, t0_ns, t1_ns) per task
   cudaStream_t origin = nullptr;  // capture / launch stream on slot 0's device
   int origin_dev = 0;
   std::vector<cudaEvent_t> fork_join;  // per slot-stream, for fork/join around a call
@@ -217,6 +221,8 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.prio_mode = (int)env_int("STF_PRIO_MODE", 0);
   po.with_load = load;
   po.with_store = store;
+  po.load_order = env_int("STF_LOAD_ORDER", 0);            // experiment knobs (not part of the ABI)
+  po.store_own_stream = env_int("STF_STORE_STREAM", 1) != 0;
   po.lookahead = o.lookahead != 0;
   po.push = o.push != 0 && o.trsm >= 2;
   return po;
@@ -293,8 +299,8 @@ struct Lowerer {
           for (int64_t pp = 0; pp < parts; ++pp) {
             stfk::Mirrors mp = mir;
             for (int m = 0; m < mp.n; ++m) mp.p[m] = mir.p[m] + pp * w * nb;
-            CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)w, L + pp * w * nb + pp * w, nb, B + pp * w * nb, nb, 0,
-                                      &mp),
+            CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)w, L + pp * w * nb + pp * w, nb, B + pp * w * nb, nb,
+                                      (int)X.opt.trsm_rows, &mp),
                      "TRSM launch");
             if (pp + 1 < parts)
               CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)(nb - (pp + 1) * w), (int)w, B + pp * w * nb, nb,
@@ -302,8 +308,8 @@ struct Lowerer {
                        "TRSM GEMM");
           }
         } else if (X.opt.trsm >= 2) {
-          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, 0,
-                                    &mir),
+          CUDA_TRY(stfk::trsm_panel(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb,
+                                    (int)X.opt.trsm_rows, &mir),
                    "TRSM launch");
         } else if (X.opt.trsm == 1)
           CUDA_TRY(stfk::trsm_tile(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, ws),
@@ -457,8 +463,10 @@ struct Lowerer {
           while (!recorded[*q].load(std::memory_order_acquire)) std::this_thread::yield();
         CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
       }
+      if (X.trace) CUDA_TRY(stfk::stamp(s, X.trace + 2 * t), "trace stamp");
       int r = body(task, t, s, prio_of(task));
       if (r) return r;
+      if (X.trace) CUDA_TRY(stfk::stamp(s, X.trace + 2 * t + 1), "trace stamp");
       if (X.mp) {  // publish remote replicas written by this task (COPY target, fused-push mirrors)
         auto signal = [&](int64_t b) -> int {
           const int dst = P.buffers[(size_t)b].slot;
@@ -670,6 +678,11 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
       CUDA_TRY(stfk::dataflow_prepare((int)X.nb, (int)X.nb, false), "dataflow tables");
     }
   }
+  if (getenv("STF_DEBUG_TRACE") && atoi(getenv("STF_DEBUG_TRACE")) && X.ngpus == 1 && !X.mp) {
+    cudaSetDevice(C.slots[0].device);
+    CUDA_TRY(cudaMalloc(&X.trace, P.tasks.size() * 2 * sizeof(unsigned long long)), "trace alloc");
+    X.allocs.push_back({C.slots[0].device, X.trace});
+  }
   // events only where a successor runs on another stream
   std::vector<int64_t> soff, succ;
   P.graph.build_successors(soff, succ);
@@ -868,9 +881,10 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.trsm = env_int("STF_TRSM", 3);
   C.opt.trsm_split = env_int("STF_TRSM_SPLIT", 4);
   C.opt.trsm_res_tail = env_int("STF_TRSM_RES_TAIL", 8192);
+  C.opt.trsm_rows = env_int("STF_TRSM_ROWS", 128);
   C.opt.push = env_int("STF_PUSH", 0);
   C.opt.mem_cap_tiles = env_int("STF_MEM_CAP_TILES", 0);
-  C.opt.streams = env_int("STF_STREAMS", 8);
+  C.opt.streams = env_int("STF_STREAMS", 32);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
   C.opt.threads = env_int("STF_THREADS", 8);
@@ -1002,6 +1016,10 @@ int stf_set_option(const char* name, int64_t value) {
     if (value < 0) return fail(-105, "trsm_res_tail must be >= 0");
     C.opt.trsm_res_tail = value;
   }
+  else if (n == "trsm_rows") {
+    if (value != 32 && value != 64 && value != 128) return fail(-105, "trsm_rows must be 32, 64 or 128");
+    C.opt.trsm_rows = value;
+  }
   else if (n == "push") C.opt.push = value != 0;
   else if (n == "mem_cap_tiles") {
     if (value != 0 && value < 3) return fail(-105, "mem_cap_tiles must be 0 (no cap) or >= 3 (a GEMM holds 3 tiles)");
@@ -1033,6 +1051,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "lookahead") *value = C.opt.lookahead;
   else if (n == "trsm_split") *value = C.opt.trsm_split;
   else if (n == "trsm_res_tail") *value = C.opt.trsm_res_tail;
+  else if (n == "trsm_rows") *value = C.opt.trsm_rows;
   else if (n == "push") *value = C.opt.push;
   else if (n == "mem_cap_tiles") *value = C.opt.mem_cap_tiles;
   else if (n == "threads") *value = C.opt.threads;
@@ -1182,11 +1201,32 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
   fill_stats(*X, hit, &C.last);
   C.last.device_ms = C.device_ms;
   C.last.graph_reuse = reuse;
+  C.last_trace.clear();
+  if (X->trace && info >= 0) {  // debug timeline of this call (run() has synchronised)
+    const auto& tasks = X->plan.tasks;
+    std::vector<unsigned long long> ts(tasks.size() * 2);
+    cudaSetDevice(C.slots[0].device);
+    if (cudaMemcpy(ts.data(), X->trace, ts.size() * 8, cudaMemcpyDeviceToHost) == cudaSuccess)
+      for (size_t t = 0; t < tasks.size(); ++t) {
+        const stf::Task& k = tasks[t];
+        const int64_t rec[7] = {k.kind, k.i, k.j, k.k, k.stream, (int64_t)ts[2 * t], (int64_t)ts[2 * t + 1]};
+        C.last_trace.insert(C.last_trace.end(), rec, rec + 7);
+      }
+  }
   if (info < 0) {
     // a failed call leaves device state unknown: drop the plan
     C.cache.remove_if([&](const std::unique_ptr<Exec>& p) { return p.get() == X; });
   }
   return info;
+}
+
+int64_t stf_debug_last_trace(int64_t* out, int64_t cap_tasks) {
+  Context& C = ctx();
+  std::lock_guard<std::mutex> g(C.mu);
+  const int64_t n = (int64_t)C.last_trace.size() / 7;
+  if (out)
+    std::copy(C.last_trace.begin(), C.last_trace.begin() + 7 * std::min(n, std::max<int64_t>(cap_tasks, 0)), out);
+  return n;
 }
 
 int stf_last_stats(stf_plan_stats* out) {
@@ -1349,7 +1389,7 @@ int stf_kernel_trsm(int64_t M, int64_t n, const double* L, int64_t ldl, double* 
     return 0;
   }
   if (ctx().opt.trsm >= 2) {
-    CUDA_TRY(stfk::trsm_panel(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm (row panel)");
+    CUDA_TRY(stfk::trsm_panel(0, 0, (int)M, (int)n, L, ldl, B, ldb, (int)ctx().opt.trsm_rows), "trsm (row panel)");
     CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
     return 0;
   }

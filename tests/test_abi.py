@@ -83,9 +83,9 @@ def test_init_without_gpu_fails_cleanly():
     assert b"CUDA" in _abi.stf_last_error() or b"device" in _abi.stf_last_error()
 
 
-OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (3, 1), "streams": (8, 3), "serial": (0, 1),
+OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (3, 1), "streams": (32, 3), "serial": (0, 1),
            "priority": (1, 0), "grid_p": (0, 2), "lookahead": (1, 0), "threads": (8, 2), "trsm_split": (4, 2), "push": (0, 1),
-           "trsm_res_tail": (8192, 0)}
+           "trsm_res_tail": (8192, 0), "trsm_rows": (128, 64)}
 
 
 def test_options_roundtrip_without_gpu():

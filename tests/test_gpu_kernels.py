@@ -21,17 +21,19 @@ def abi():
     return _abi
 
 
-@pytest.fixture(params=[(1, 3), (1, 2), (1, 1), (0, 0)], ids=["dataflow+resident", "dataflow+rowpanel", "dataflow",
-                                                              "recursive"])
+@pytest.fixture(params=[(1, 3, 64), (1, 2, 64), (1, 2, 128), (1, 1, 64), (0, 0, 64)],
+                ids=["dataflow+resident", "dataflow+rowpanel", "dataflow+rowpanel128", "dataflow", "recursive"])
 def variant(request, abi):
-    """(POTRF, TRSM) implementations: POTRF dataflow (1) / recursive (0);
+    """(POTRF, TRSM, rows) implementations: POTRF dataflow (1) / recursive (0);
     TRSM resident panel (3, product default; row panel where unsupported) /
-    row panel (2) / dataflow (1) / recursive (0)."""
+    row panel (2, 64 or 128 rows per CTA) / dataflow (1) / recursive (0)."""
     abi.stf_set_option(b"dataflow", request.param[0])
     abi.stf_set_option(b"trsm", request.param[1])
+    abi.stf_set_option(b"trsm_rows", request.param[2])
     yield request.param
     abi.stf_set_option(b"dataflow", 1)
     abi.stf_set_option(b"trsm", 3)
+    abi.stf_set_option(b"trsm_rows", 128)
 
 
 def _even(x):

@@ -34,6 +34,19 @@ def test_parity_trsm_variants(stf, trsm, split):
     assert relF(M.to_dense().numpy(), Lo) <= 1e-10
 
 
+@pytest.mark.parametrize("rows", [32, 128])
+def test_trsm_panel_rows_same_bits(stf, rows):  # 128 is the default
+    """The row-panel TRSM at 32 / 128 rows per CTA (128: half-depth stages, two
+    solver warps per SM sub-partition) keeps every sum in the same order as the
+    64-row form, so the whole factorisation is bit-identical."""
+    for n, nb, split in [(2048, 512, 4), (3072, 1024, 4), (1536, 512, 2)]:
+        ref = _bits(stf, n, nb, trsm=2, trsm_split=split, trsm_rows=64)
+        got = _bits(stf, n, nb, trsm=2, trsm_split=split, trsm_rows=rows)
+        assert np.array_equal(ref, got), (n, nb, split)
+        Lo, _ = oracle.potrf(synth.spd_matrix(3, n))
+        assert relF(got, Lo) <= 1e-10
+
+
 def test_parity_recursive_panel_kernels(stf):
     """The recursive (GEMM-based) POTRF/TRSM variant through the whole path."""
     _options(stf, dataflow=0, trsm=0)
@@ -54,7 +67,8 @@ def _reset_options(request):
     yield
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
-        _options(s, graph=1, serial=0, priority=1, streams=8, grid_p=0, dataflow=1, trsm=3, threads=8, lookahead=1, trsm_split=4, push=0)
+        _options(s, graph=1, serial=0, priority=1, streams=32, grid_p=0, dataflow=1, trsm=3, threads=8, lookahead=1, trsm_split=4, push=0,
+                 trsm_rows=128)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
@@ -180,7 +194,7 @@ def _bits(stf, n, nb, p=1, q=1, seed=3, **opts):
     M, info = _factor_spd(stf, n, nb, p, q, seed)
     assert info == 0
     out = M.to_dense().numpy().copy()
-    _options(stf, graph=1, serial=0, priority=1, streams=8, threads=8)
+    _options(stf, graph=1, serial=0, priority=1, streams=32, threads=8)
     return out
 
 

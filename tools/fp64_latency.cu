@@ -51,6 +51,16 @@ __global__ void lat(double* out, long long* clk, double x0) {
     t1 = clock64();
     if (threadIdx.x == 0) clk[6] = (t1 - t0) / N;
   }
+  // rsqrt chain
+  t0 = clock64();
+  for (int i = 0; i < N; ++i) x = rsqrt(x) + 0.5;
+  t1 = clock64();
+  if (threadIdx.x == 0) clk[7] = (t1 - t0) / N;
+  // DMUL chain
+  t0 = clock64();
+  for (int i = 0; i < N; ++i) x = x * 0.999999;
+  t1 = clock64();
+  if (threadIdx.x == 0) clk[8] = (t1 - t0) / N;
   out[threadIdx.x] = x;
 }
 
@@ -62,7 +72,7 @@ int main() {
   lat<<<1, 256>>>(out, clk, 1.7);
   lat<<<1, 256>>>(out, clk, 1.7);
   cudaDeviceSynchronize();
-  const char* names[] = {"DFMA", "sqrt", "1/x", "x/y", "__syncthreads(256)", "sync+smem publish", "bar.sync 64"};
-  for (int i = 0; i < 7; ++i) printf("%-22s %lld clk\n", names[i], clk[i]);
+  const char* names[] = {"DFMA", "sqrt", "1/x", "x/y", "__syncthreads(256)", "sync+smem publish", "bar.sync 64", "rsqrt", "DMUL"};
+  for (int i = 0; i < 9; ++i) printf("%-22s %lld clk\n", names[i], clk[i]);
   return 0;
 }
