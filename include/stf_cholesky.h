@@ -219,11 +219,11 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
  * done stamps of bulk ticket t (0 if unused).  Returns the number of entries
  * written (<= cap) or a negative error.  Not part of the factorisation. */
 /* Debug timeline of the last stf_potrf on one GPU slot, recorded when the
- * environment had STF_DEBUG_TRACE=1 at plan build (a one-thread stamp kernel
- * before and after every task on its stream; perturbs timing slightly).  Writes
- * up to cap_tasks records of 7 int64 (kind as in stf_dag_build, i, j, k, stream index,
- * %globaltimer ns at start, at end) in program order; returns the number of
- * tasks of the call (0 if it was not traced). */
+ * environment had STF_DEBUG_TRACE=1 at plan build (timing events recorded
+ * before and after every task on its stream; no SM work).  Writes up to
+ * cap_tasks records of 7 int64 (kind as in stf_dag_build, i, j, k, stream index,
+ * ns since the first task's start, at start and at end; -1 if unavailable) in
+ * program order; returns the number of tasks of the call (0 if not traced). */
 int64_t stf_debug_last_trace(int64_t *out, int64_t cap_tasks);
 
 int64_t stf_debug_potrf_trace(int64_t n, double *A, int64_t lda, int ctas, int64_t *trace, int64_t cap);

@@ -219,16 +219,6 @@ cudaError_t transpose_copy(cudaStream_t stream, double* dst, int64_t ldd, const 
 
 __global__ void info_reset_kernel(unsigned long long* info) { *info = ULLONG_MAX; }
 
-// debug timeline (STF_DEBUG_TRACE): one thread stores %globaltimer (ns)
-__global__ void stamp_kernel(unsigned long long* dst) {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  *dst = t;
-}
-cudaError_t stamp(cudaStream_t stream, unsigned long long* dst) {
-  stamp_kernel<<<1, 1, 0, stream>>>(dst);
-  return cudaGetLastError();
-}
 
 cudaError_t info_reset(cudaStream_t stream, unsigned long long* info) {
   ++launch_count();

@@ -76,7 +76,6 @@ cudaError_t transpose_copy(cudaStream_t stream, double* dst, int64_t ldd, const 
 
 // Fill a device int64 sentinel used by potrf_lower's info.
 cudaError_t info_reset(cudaStream_t stream, unsigned long long* info);
-cudaError_t stamp(cudaStream_t stream, unsigned long long* dst);  // debug timeline
 
 // Number of kernels enqueued by the launchers above, all host threads
 // (monotonic; the runtime reports per-call deltas as gpu_launches).

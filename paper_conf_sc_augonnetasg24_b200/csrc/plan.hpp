@@ -52,8 +52,10 @@ struct PlanOptions {
   int prio_mode = 0;       // level assignment variant (0 default; see plan.cpp)
   bool with_load = false;  // LOAD tasks first (COLMAJOR descriptors)
   bool with_store = false; // STORE tasks (write-back) at the end of program order
-  int load_order = 0;      // LOAD order: 0 tile columns (j outer), 1 tile rows (i outer)
   bool store_own_stream = true;  // STOREs on the other copy stream than the slot's LOADs
+  bool order_asap = false;  // re-submit the tasks in order of earliest start (see plan.cpp);
+                            // the runtime sets it for COLMAJOR calls (LOAD/STORE tasks)
+  double copy_cost = 0;     // order_asap: a tile copy in GEMM-tile times (0: 2.7, nb = 1024)
   bool lookahead = true;   // false: a FENCE task (RW on every tile) closes each panel step, so
                            // step k+1 starts only when step k is complete (ablation, NEXT-1)
   bool push = false;       // TRSM(i,k) writes L_ik into its consumers' replicas itself (fused

@@ -126,7 +126,7 @@ struct Exec {
   int64_t graph_nodes = 0;
   int graph_fallback = 0;  // capture failed, eager lowering used
   unsigned skip_mask = 0;  // STF_DEBUG_SKIP: task kinds whose kernels are not launched (timing what-ifs)
-  unsigned long long* trace = nullptr;  // STF_DEBUG_TRACE: per task %globaltimer at start / end (slot 0's device)
+  std::vector<cudaEvent_t> trace;  // STF_DEBUG_TRACE: per task timing events at start / end (one GPU slot)
   int64_t updates = 0;     // successful cudaGraphExecUpdate re-binds
   bool rebound = false;
   int64_t launches = 0;
@@ -158,6 +158,8 @@ struct Exec {
         cudaSetDevice(events_dev[t]);
         cudaEventDestroy(events[t]);
       }
+    for (auto& ev : trace)
+      if (ev) cudaEventDestroy(ev);
     for (auto& a : allocs) {
       cudaSetDevice(a.first);
       cudaFree(a.second);
@@ -221,8 +223,10 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.prio_mode = (int)env_int("STF_PRIO_MODE", 0);
   po.with_load = load;
   po.with_store = store;
-  po.load_order = env_int("STF_LOAD_ORDER", 0);            // experiment knobs (not part of the ABI)
-  po.store_own_stream = env_int("STF_STORE_STREAM", 1) != 0;
+  // submission in order of earliest start for plans with host/device transfers
+  // (STF_ORDER_ASAP: -1 auto = COLMAJOR calls, 0 never, 1 always)
+  const int64_t asap = env_int("STF_ORDER_ASAP", -1);
+  po.order_asap = asap < 0 ? load : asap != 0;
   po.lookahead = o.lookahead != 0;
   po.push = o.push != 0 && o.trsm >= 2;
   return po;
@@ -463,10 +467,11 @@ struct Lowerer {
           while (!recorded[*q].load(std::memory_order_acquire)) std::this_thread::yield();
         CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
       }
-      if (X.trace) CUDA_TRY(stfk::stamp(s, X.trace + 2 * t), "trace stamp");
+      // debug timeline: timing events (external record nodes when captured), no SM work
+      if (!X.trace.empty()) CUDA_TRY(cudaEventRecordWithFlags(X.trace[2 * t], s, cudaEventRecordExternal), "trace");
       int r = body(task, t, s, prio_of(task));
       if (r) return r;
-      if (X.trace) CUDA_TRY(stfk::stamp(s, X.trace + 2 * t + 1), "trace stamp");
+      if (!X.trace.empty()) CUDA_TRY(cudaEventRecordWithFlags(X.trace[2 * t + 1], s, cudaEventRecordExternal), "trace");
       if (X.mp) {  // publish remote replicas written by this task (COPY target, fused-push mirrors)
         auto signal = [&](int64_t b) -> int {
           const int dst = P.buffers[(size_t)b].slot;
@@ -584,6 +589,13 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   const int64_t T = X.n / X.nb;
   const bool colmajor = X.kind != STF_DESC_TILED_2DBC;
   stf::PlanOptions po = plan_options(X.opt, X.P, X.Q, X.ngpus, colmajor, colmajor);
+  // tile copy time in GEMM-tile times for the early-start order: PCIe ~55 GB/s vs
+  // a 2 nb^3 tile update at ~35 TF/s (2.7 at nb = 1024); device copies ~free.
+  // The order pays off with tiles of order >= 1024 (n = 32768: e2e 396 -> 350 ms);
+  // with small tiles the captured program order was faster (n = 8192, nb = 256:
+  // 23 vs 60 ms), so it is used there (STF_ORDER_ASAP = 1 forces it).
+  po.copy_cost = X.kind == STF_DESC_HOST_COLMAJOR ? 2.7 * 1024.0 / (double)X.nb : 0.05;
+  if (env_int("STF_ORDER_ASAP", -1) < 0) po.order_asap = colmajor && X.nb >= 1024;
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
     po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames
@@ -680,8 +692,8 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   }
   if (getenv("STF_DEBUG_TRACE") && atoi(getenv("STF_DEBUG_TRACE")) && X.ngpus == 1 && !X.mp) {
     cudaSetDevice(C.slots[0].device);
-    CUDA_TRY(cudaMalloc(&X.trace, P.tasks.size() * 2 * sizeof(unsigned long long)), "trace alloc");
-    X.allocs.push_back({C.slots[0].device, X.trace});
+    X.trace.assign(P.tasks.size() * 2, nullptr);
+    for (auto& ev : X.trace) CUDA_TRY(cudaEventCreate(&ev), "trace event");
   }
   // events only where a successor runs on another stream
   std::vector<int64_t> soff, succ;
@@ -844,6 +856,21 @@ bool host_pinned(const void* ptr) {
     return false;
   }
   return a.type == cudaMemoryTypeHost;
+}
+
+// HOST_COLMAJOR calls are lowered eagerly onto the streams: pageable memory
+// cannot be captured, and in-core with pinned memory the captured graph ran the
+// early-start submission order ~10% slower end to end than the streams
+// (n = 32768: 386 vs 350 ms, profiles/r01/e2e_order.txt) - for tiles of order
+// >= 1024 only: with smaller tiles the host cannot issue the many short tasks fast
+// enough (n = 8192, nb = 256: 38.9 ms eager vs 23 ms captured in program order).
+// STF_HOST_GRAPH=1 always captures.  Out-of-core plans keep the graph when pinned.
+bool host_eager(const Context& C, const stf_matrix_desc* d, int64_t n, int64_t nb, int ngpus) {
+  if (d->kind != STF_DESC_HOST_COLMAJOR) return false;
+  if (!host_pinned(d->ptr)) return true;
+  const int64_t T = nb > 0 ? n / nb : 0;
+  const bool ooc = ngpus == 1 && C.opt.mem_cap_tiles > 0 && C.opt.mem_cap_tiles < T * (T + 1) / 2;
+  return !ooc && nb >= 1024 && !env_int("STF_HOST_GRAPH", 0);
 }
 
 int ensure_kernel_attrs(int dev) {
@@ -1168,7 +1195,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
     e->key_ptrs = ptrs;
     e->key_ld = A_desc->ld;
     e->key_dev = A_desc->device;
-    if (A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr)) e->opt.graph = 0;  // pageable: no capture
+    if (host_eager(C, A_desc, n, nb, ngpus)) e->opt.graph = 0;
     if (const char* sk = getenv("STF_DEBUG_SKIP")) {
       std::string v(sk);
       const char* names[] = {"potrf", "trsm", "syrk", "gemm", "copy", "trsm_as_gemm", "trsm_as_half_gemm"};
@@ -1189,7 +1216,7 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
       e.reset(new Exec());
       e->n = n; e->nb = nb; e->uplo = up; e->kind = A_desc->kind; e->ngpus = ngpus; e->P = P; e->Q = Q;
       e->opt = C.opt; e->key_graph = C.opt.graph; e->key_ptrs = ptrs; e->key_ld = A_desc->ld; e->key_dev = A_desc->device;
-      if (A_desc->kind == STF_DESC_HOST_COLMAJOR && !host_pinned(A_desc->ptr)) e->opt.graph = 0;
+      if (host_eager(C, A_desc, n, nb, ngpus)) e->opt.graph = 0;
       g_err.clear();
       r = prepare(C, *e, A_desc);
     }
@@ -1202,16 +1229,20 @@ int stf_potrf(int64_t n, int64_t nb, char uplo, stf_matrix_desc* A_desc, int ngp
   C.last.device_ms = C.device_ms;
   C.last.graph_reuse = reuse;
   C.last_trace.clear();
-  if (X->trace && info >= 0) {  // debug timeline of this call (run() has synchronised)
+  if (!X->trace.empty() && info >= 0) {  // debug timeline of this call (run() has synchronised)
     const auto& tasks = X->plan.tasks;
-    std::vector<unsigned long long> ts(tasks.size() * 2);
     cudaSetDevice(C.slots[0].device);
-    if (cudaMemcpy(ts.data(), X->trace, ts.size() * 8, cudaMemcpyDeviceToHost) == cudaSuccess)
-      for (size_t t = 0; t < tasks.size(); ++t) {
-        const stf::Task& k = tasks[t];
-        const int64_t rec[7] = {k.kind, k.i, k.j, k.k, k.stream, (int64_t)ts[2 * t], (int64_t)ts[2 * t + 1]};
-        C.last_trace.insert(C.last_trace.end(), rec, rec + 7);
+    for (size_t t = 0; t < tasks.size(); ++t) {
+      const stf::Task& k = tasks[t];
+      float a = 0.f, b = 0.f;  // ms since the first task's start event
+      if (cudaEventElapsedTime(&a, X->trace[0], X->trace[2 * t]) != cudaSuccess ||
+          cudaEventElapsedTime(&b, X->trace[0], X->trace[2 * t + 1]) != cudaSuccess) {
+        cudaGetLastError();
+        a = b = -1.f;
       }
+      const int64_t rec[7] = {k.kind, k.i, k.j, k.k, k.stream, (int64_t)(a * 1e6), (int64_t)(b * 1e6)};
+      C.last_trace.insert(C.last_trace.end(), rec, rec + 7);
+    }
   }
   if (info < 0) {
     // a failed call leaves device state unknown: drop the plan

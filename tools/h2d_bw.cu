@@ -8,6 +8,15 @@
 #include <vector>
 #include <cuda_runtime.h>
 
+// occupies every SM (4 CTAs x 256 threads each, FP64 FMA chains) for ~ms milliseconds
+__global__ void busy(double* out, long long cycles) {
+  const long long t0 = clock64();
+  double x = threadIdx.x;
+  while (clock64() - t0 < cycles)
+    for (int i = 0; i < 64; ++i) x = fma(x, 0.9999, 1e-7);
+  if (x == 12345.0) out[0] = x;
+}
+
 int main(int argc, char** argv) {
   const long n = argc > 1 ? atol(argv[1]) : 32768, nb = argc > 2 ? atol(argv[2]) : 1024, T = n / nb;
   const long ntiles = T * (T + 1) / 2, tb = nb * nb * 8;
@@ -62,6 +71,33 @@ int main(int argc, char** argv) {
       run("2D tiles", ns, 0, h2d);
       run("contig", ns, 1, h2d);
     }
+  // copies while every SM is busy (the e2e situation): does the copy need SMs?
+  {
+    cudaStream_t sb;
+    cudaStreamCreateWithFlags(&sb, cudaStreamNonBlocking);
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+    for (int h2d = 1; h2d >= 0; --h2d) {
+      cudaDeviceSynchronize();
+      busy<<<sms * 4, 256, 0, sb>>>(reinterpret_cast<double*>(d), 2000000000LL / 10 * 3);  // ~300 ms
+      cudaEventRecord(e0, st[0]);
+      long t = 0;
+      for (long j = 0; j < T; ++j)
+        for (long i = j; i < T; ++i, ++t) {
+          double* dt = d + t * nb * nb;
+          double* ht = h + i * nb + j * nb * n;
+          if (h2d) cudaMemcpy2DAsync(dt, nb * 8, ht, n * 8, nb * 8, nb, cudaMemcpyHostToDevice, st[0]);
+          else cudaMemcpy2DAsync(ht, n * 8, dt, nb * 8, nb * 8, nb, cudaMemcpyDeviceToHost, st[0]);
+        }
+      cudaEventRecord(e1, st[0]);
+      cudaEventSynchronize(e1);
+      float ms = 0;
+      cudaEventElapsedTime(&ms, e0, e1);
+      printf("%s 2D tiles while all SMs busy: %8.2f ms  %6.1f GB/s\n", h2d ? "H2D" : "D2H", ms,
+             ntiles * tb / (ms * 1e-3) / 1e9);
+      cudaDeviceSynchronize();
+    }
+  }
   // both directions at once (the e2e overlap): H2D tiles on st[0], D2H tiles on st[1]
   cudaDeviceSynchronize();
   auto t0 = std::chrono::steady_clock::now();

@@ -38,7 +38,7 @@ cnt = _abi.stf_debug_last_trace(None, 0)
 buf = (ctypes.c_int64 * (7 * cnt))()
 _abi.stf_debug_last_trace(buf, cnt)
 R = np.frombuffer(buf, dtype=np.int64).reshape(cnt, 7)
-t0 = R[:, 5].min()
+t0 = R[R[:, 5] >= 0, 5].min()
 R = R.copy()
 R[:, 5:] -= t0
 names = ["POTRF", "TRSM", "SYRK", "GEMM", "COPY", "LOAD", "STORE", "FENCE"]
