@@ -129,3 +129,22 @@ def test_fused_push_replaces_panel_copies(T, p, q, known):
     if T <= 8:
         Ro = oracle.transitive_closure(len(ot), oracle.stf_edges([acc for _, _, acc in ot]))
         assert np.array_equal(R[np.ix_(comp, comp)], Ro)
+
+
+@pytest.mark.parametrize("T,p,q", [(6, 1, 1), (8, 2, 2), (8, 2, 4), (5, 1, 2)])
+def test_earliest_start_order_same_dag(T, p, q, monkeypatch):
+    """The early-start re-submission (plan.cpp reorder_asap, used for COLMAJOR
+    calls) is a topological order of the program-order DAG, and re-applying the
+    STF rule in that order yields the same DAG (edges identical up to the task
+    relabelling): only the stream-order chains change."""
+    e0, k0, ijk0, st0 = stf.dag(T, p, q)
+    monkeypatch.setenv("STF_ORDER_ASAP", "1")
+    e1, k1, ijk1, st1 = stf.dag(T, p, q)
+    keys0 = [(k, *x) for k, x in zip(k0, ijk0)]
+    keys1 = [(k, *x) for k, x in zip(k1, ijk1)]
+    assert len(set(keys0)) == len(keys0) and sorted(keys0) == sorted(keys1)
+    pos = {key: t for t, key in enumerate(keys1)}
+    perm = [pos[key] for key in keys0]
+    assert all(a < b for a, b in e1)  # submission order is topological
+    assert {(perm[a], perm[b]) for a, b in e0} == set(e1)
+    assert st1["critical_path"] == st0["critical_path"] and st1["edges"] == st0["edges"]

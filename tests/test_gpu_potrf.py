@@ -298,6 +298,24 @@ def test_colmajor_descriptors(stf, where, order, ngpus):
     assert np.all(got[np.triu_indices(n, 1)] == 12345.0)
 
 
+@pytest.mark.parametrize("ngpus", [1, 2])
+def test_host_colmajor_early_start_order_same_bits(stf, ngpus):
+    """nb >= 1024 HOST_COLMAJOR calls are re-submitted in earliest-start order and
+    lowered onto the streams; same DAG, so the same bits as the
+    device-resident tiles."""
+    import torch
+
+    n, nb = 4096, 1024
+    ref = _bits(stf, n, nb, 1, ngpus, seed=7)
+    A = synth.spd_matrix(7, n)
+    t = torch.from_numpy(np.ascontiguousarray(A)).pin_memory().t()  # column-major view
+    assert stf.potrf(t, nb, ngpus=ngpus) == 0
+    st = stf.last_stats()
+    assert st["graph_nodes"] == 0 and st["host_loads"] == 10  # eager lowering, lower tiles loaded
+    got = np.tril(t.numpy())
+    assert np.array_equal(got, np.tril(ref))
+
+
 def test_n_zero(stf):
     import torch
 
