@@ -78,12 +78,7 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
 // refill of a stage is issued by the LAST warp to finish reading it (shared-memory
 // arrival counter), i.e. at the earliest possible moment, with the next k-tile
 // STAGES ahead; consumers wait only on the TMA "full" mbarriers.
-// TPC > 1 (plain GEMM only): the CTA computes TPC consecutive N-tiles with ONE
-// continuous stage ring (the next tile's first k-stages load during this tile's
-// last ones, its C is prefetched into L2), so the per-tile start-up - launch,
-// first TMA round trip, C load - is paid once per TPC tiles (fixed cost measured
-// at ~2.2% of a K = 1024 tile: 8192^2 x K runs at 97.4% of peak as K -> inf).
-template <int WM, int WN, class g, int TPC = 1>
+template <int WM, int WN, class g>
 __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         double* __restrict__ C, int64_t ldc, int M, int N, int K, int lower) {
@@ -115,13 +110,10 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
     }
   } else {
     tm = blockIdx.x;
-    tn = blockIdx.y * TPC;
+    tn = blockIdx.y;
   }
-  const int m0 = tm * g::BM, n00 = tn * g::BN;
+  const int m0 = tm * g::BM, n0 = tn * g::BN;
   const int KT = (K + g::BK - 1) / g::BK;
-  // tiles of this CTA (TPC > 1: the last CTA column may hold fewer)
-  const int ntile = (TPC == 1) ? 1 : min(TPC, (N - n00 + g::BN - 1) / g::BN);
-  const int KTT = ntile * KT;  // k-stages over all tiles of the CTA
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
@@ -132,8 +124,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
       released[s] = 0;
     }
     fence_barrier_init();
-    for (int kt = 0; kt < g::STAGES && kt < KTT; ++kt)
-      load_stage<g>(smem, kt, &tmA, &tmB, m0, n00 + (kt / KT) * g::BN, kt % KT, full);
+    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, m0, n0, kt, full);
   }
   __syncthreads();
 
@@ -142,21 +133,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
   const int gq = lane >> 2, tq = lane & 3;
 
   // In lower mode, warps of a diagonal CTA whose warp tile is strictly upper idle.
-  const bool warp_dead = lower && (m0 + wm0 + WM <= n00 + wn0);  // warp tile strictly above the diagonal
-
-  // Per-lane fragment offsets: swz_off(w0 + 8f + gq, 2tq + kh) depends on f only
-  // through the box (f >> 1, an immediate) and the chunk bit 2 (f & 1).
-  uint32_t offA[2][2], offB[2][2];
-#pragma unroll
-  for (int p = 0; p < 2; ++p)
-#pragma unroll
-    for (int kh = 0; kh < 2; ++kh) {
-      offA[p][kh] = swz_off<g>(wm0 + 8 * p + gq, 2 * tq + kh);
-      offB[p][kh] = g::A_BYTES + swz_off<g>(wn0 + 8 * p + gq, 2 * tq + kh);
-    }
-
-  for (int u = 0; u < ntile; ++u) {
-  const int n0 = n00 + u * g::BN;
+  const bool warp_dead = lower && (m0 + wm0 + WM <= n0 + wn0);  // warp tile strictly above the diagonal
 
   // acc = C, loaded straight into the accumulators (64 independent loads in
   // flight, latency hidden behind the first TMA wait); the mainloop adds
@@ -175,22 +152,19 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
       }
   }
 
-  for (int kk = 0; kk < KT; ++kk) {
-    const int kt = u * KT + kk;
-    const int s = kt % g::STAGES;
-    if (TPC > 1 && u + 1 < ntile && kk == KT / 2) {  // next tile's C into L2 (no registers)
+  // Per-lane fragment offsets: swz_off(w0 + 8f + gq, 2tq + kh) depends on f only
+  // through the box (f >> 1, an immediate) and the chunk bit 2 (f & 1).
+  uint32_t offA[2][2], offB[2][2];
 #pragma unroll
-      for (int j = 0; j < WN / 8; ++j)
+  for (int p = 0; p < 2; ++p)
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int n = n0 + g::BN + wn0 + 8 * j + 2 * tq + h;
-#pragma unroll
-          for (int r = 0; r < WM; r += 16) {  // one 128-byte line per 16 rows
-            const int m = m0 + wm0 + r + gq;
-            if (n < N && m < M) asm volatile("prefetch.global.L2 [%0];" ::"l"(C + (int64_t)n * ldc + m));
-          }
-        }
+    for (int kh = 0; kh < 2; ++kh) {
+      offA[p][kh] = swz_off<g>(wm0 + 8 * p + gq, 2 * tq + kh);
+      offB[p][kh] = g::A_BYTES + swz_off<g>(wn0 + 8 * p + gq, 2 * tq + kh);
     }
+
+  for (int kt = 0; kt < KT; ++kt) {
+    const int s = kt % g::STAGES;
     mbar_wait(&full[s], (kt / g::STAGES) & 1);
     const uint8_t* st = smem + s * g::STAGE_BYTES;
     if (!warp_dead) {
@@ -216,14 +190,13 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
       }
     }
     __syncwarp();  // this warp's reads of stage s are complete (their values fed its DMMAs)
-    if (lane == 0 && kt + g::STAGES < KTT) {
+    if (lane == 0 && kt + g::STAGES < KT) {
       __threadfence_block();
       if (atomicAdd(&released[s], 1) == NCW - 1) {  // last reader of stage s refills it
         released[s] = 0;
         __threadfence_block();
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        const int kn = kt + g::STAGES;
-        load_stage<g>(smem, s, &tmA, &tmB, m0, n00 + (kn / KT) * g::BN, kn % KT, full);
+        load_stage<g>(smem, s, &tmA, &tmB, m0, n0, kt + g::STAGES, full);
       }
     }
   }
@@ -242,7 +215,6 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
       }
     }
   }
-  }  // tiles of the CTA
 }
 
 // ------------------------------------------------------------------ host side
@@ -296,11 +268,6 @@ static int gemm_narrow() {
   static int v = env_or("STF_GEMM_NARROW", 2);
   return v;
 }
-// N-tiles per CTA of the plain (non-SYRK) 128 x 64 GEMM: STF_GEMM_TPC (1 or 2)
-static int gemm_tpc() {
-  static int v = env_or("STF_GEMM_TPC", 1) == 2 ? 2 : 1;
-  return v;
-}
 
 template <class G>
 static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tmA, const CUtensorMap& tmB, double* C,
@@ -338,10 +305,6 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
     cfg.dynamicSmemBytes = CfgN64::SMEM_BYTES;
     if (gemm_narrow() == 2) {  // 8 warps of 32 x 32, 2 CTAs (16 warps) per SM
       cfg.blockDim = dim3(256, 1, 1);
-      if (!lower && gemm_tpc() == 2) {
-        cfg.gridDim = dim3(tM, (tN + 1) / 2, 1);
-        return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64, 2>, tmA, tmB, C, ldc, M, N, K, lower);
-      }
       return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64>, tmA, tmB, C, ldc, M, N, K, lower);
     }
     cfg.blockDim = dim3(128, 1, 1);  // 4 warps of 64 x 32
@@ -369,9 +332,6 @@ cudaError_t gemm_init_attrs() {
                              CfgN64::SMEM_BYTES);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, CfgN64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             CfgN64::SMEM_BYTES);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, CfgN64, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              CfgN64::SMEM_BYTES);
   return e;
 }
