@@ -3,6 +3,7 @@
 
 #include <algorithm>
 #include <climits>
+#include <queue>
 #include <set>
 #include <utility>
 #include <vector>
@@ -15,6 +16,21 @@ int streams_per_slot(const PlanOptions& opt) {
 }
 
 namespace {
+
+// High-priority streams: the panel chain POTRF(k) -> TRSM(k+1,k) -> SYRK(k+1,k)
+// (level 5) alone on stream 0, so stream order never puts a chain task behind
+// another task (measured at n = 8192: POTRF(1) started 1.06 ms after SYRK(1,0)
+// while it queued behind the bulk TRSMs sharing its stream); the tasks that feed
+// the next chain TRSM(k+2,k+1) - TRSM(k+2,k) and GEMM(k+2,k+1,k) - alone on
+// stream 1; the other urgent tasks (level 4: TRSM(i,k), the next column's
+// updates) on streams 2.. by row.
+template <class TaskLike>
+int crit_stream(const TaskLike& t, int crit_streams) {
+  if (crit_streams <= 1 || t.prio >= 5) return 0;
+  const bool feeds_chain = t.i == t.k + 2 && (t.kind == K_TRSM || (t.kind == K_GEMM && t.j == t.k + 1));
+  if (crit_streams == 2 || feeds_chain) return 1;
+  return 2 + (int)(t.i % (crit_streams - 2));
+}
 
 struct Builder {
   Plan& p;
@@ -38,10 +54,7 @@ struct Builder {
 
   int compute_stream(const Task& t) const {
     if (p.opt.serial) return 0;
-    if (p.opt.priority && t.prio >= 4) {
-      if (t.kind == K_POTRF) return 0;
-      return (int)(t.i % p.opt.crit_streams);
-    }
+    if (p.opt.priority && t.prio >= 4) return crit_stream(t, p.opt.crit_streams);
     return p.opt.crit_streams + (int)((t.i * T + t.j) % p.opt.bulk_streams);
   }
 
@@ -305,7 +318,7 @@ struct OocBuilder {
     };
     auto compute_stream = [&](const CT& c) -> int {
       if (serial) return 0;
-      if (priority && c.prio >= 4) return c.kind == K_POTRF ? 0 : (int)(c.i % crit_streams);
+      if (priority && c.prio >= 4) return crit_stream(c, crit_streams);
       return crit_streams + (int)((c.i * T + c.j) % bulk_streams);
     };
     for (size_t q = 0; q < seq.size(); ++q) {
@@ -425,6 +438,100 @@ static void reorder_asap(Plan& plan, const std::vector<std::vector<Access>>& acc
   plan.graph = std::move(g);
 }
 
+// Submission order by simulated list scheduling (order_mode 2): each GPU slot
+// runs at most `width` compute tasks at a time, transfers one at a time per copy
+// stream; among ready compute tasks the one with the longest remaining path
+// (bottom level, in the cost units of reorder_asap) starts first.  Tasks are
+// re-submitted in order of simulated start, so the bounded look-ahead of the
+// graph executor / stream queues sees the tasks the GPU will run next - the
+// panel chain before the bulk updates of the same step.  A topological order,
+// so the DAG is unchanged (see reorder_asap).
+static void reorder_list(Plan& plan, const std::vector<std::vector<Access>>& accs, int64_t ndata, int width) {
+  const size_t n = plan.tasks.size();
+  const double copy_cost = plan.opt.copy_cost > 0 ? plan.opt.copy_cost : 2.7;
+  auto is_copy = [](int32_t k) { return k == K_COPY || k == K_LOAD || k == K_STORE; };
+  auto cost = [&](const Task& t) -> double {
+    switch (t.kind) {
+      case K_POTRF: return 5.0;
+      case K_TRSM: return 2.0;
+      case K_SYRK:
+      case K_GEMM: return 1.0;
+      case K_COPY:
+      case K_LOAD:
+      case K_STORE: return copy_cost;
+      default: return 0.01;
+    }
+  };
+  std::vector<int64_t> soff, succ;
+  plan.graph.build_successors(soff, succ);
+  std::vector<double> bl(n, 0.0);
+  for (size_t t = n; t-- > 0;) {
+    double m = 0.0;
+    for (int64_t e = soff[t]; e < soff[t + 1]; ++e) m = std::max(m, bl[(size_t)succ[(size_t)e]]);
+    bl[t] = cost(plan.tasks[t]) + m;
+  }
+  std::vector<int64_t> npred(n, 0);
+  for (size_t t = 0; t < n; ++t) npred[t] = plan.graph.preds_end((int64_t)t) - plan.graph.preds_begin((int64_t)t);
+  int nslots = 1;
+  for (const Task& t : plan.tasks) nslots = std::max(nslots, t.slot + 1);
+  auto cmp_ready = [&](size_t a, size_t b) { return bl[a] < bl[b] || (bl[a] == bl[b] && a > b); };
+  std::vector<std::priority_queue<size_t, std::vector<size_t>, decltype(cmp_ready)>> ready;
+  for (int s = 0; s < nslots; ++s) ready.emplace_back(cmp_ready);
+  std::vector<int> busy((size_t)nslots, 0);
+  typedef std::pair<double, size_t> Ev;  // (finish time, task)
+  std::priority_queue<Ev, std::vector<Ev>, std::greater<Ev>> events;
+  std::vector<double> qfree;
+  std::vector<double> start(n, 0.0);
+  double now = 0.0;
+  auto release = [&](size_t t) {
+    const Task& k = plan.tasks[t];
+    if (is_copy(k.kind)) {
+      const size_t key = (size_t)k.slot * 64 + (size_t)k.stream;
+      if (qfree.size() <= key) qfree.resize(key + 1, 0.0);
+      start[t] = std::max(now, qfree[key]);
+      qfree[key] = start[t] + cost(k);
+      events.push(Ev(qfree[key], t));
+    } else {
+      ready[(size_t)k.slot].push(t);
+    }
+  };
+  for (size_t t = 0; t < n; ++t)
+    if (npred[t] == 0) release(t);
+  size_t done = 0;
+  while (done < n) {
+    for (int s = 0; s < nslots; ++s)
+      while (busy[(size_t)s] < width && !ready[(size_t)s].empty()) {
+        const size_t t = ready[(size_t)s].top();
+        ready[(size_t)s].pop();
+        start[t] = now;
+        busy[(size_t)s]++;
+        events.push(Ev(now + cost(plan.tasks[t]), t));
+      }
+    if (events.empty()) break;  // cannot happen for a DAG
+    const Ev ev = events.top();
+    events.pop();
+    now = ev.first;
+    const size_t t = ev.second;
+    ++done;
+    if (!is_copy(plan.tasks[t].kind)) busy[(size_t)plan.tasks[t].slot]--;
+    for (int64_t e = soff[t]; e < soff[t + 1]; ++e) {
+      const size_t u = (size_t)succ[(size_t)e];
+      if (--npred[u] == 0) release(u);
+    }
+  }
+  std::vector<size_t> ord(n);
+  for (size_t t = 0; t < n; ++t) ord[t] = t;
+  std::stable_sort(ord.begin(), ord.end(), [&](size_t a, size_t b) { return start[a] < start[b]; });
+  std::vector<Task> tasks(n);
+  TaskGraph g(ndata);
+  for (size_t r = 0; r < n; ++r) {
+    tasks[r] = plan.tasks[ord[r]];
+    g.submit(accs[ord[r]].data(), (int)accs[ord[r]].size());
+  }
+  plan.tasks.swap(tasks);
+  plan.graph = std::move(g);
+}
+
 void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
   plan.T = T;
   plan.opt = opt;
@@ -451,7 +558,8 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
     plan.graph = TaskGraph(NT + NT * opt.nslots + 1);
     Builder b(plan, T);
     b.run();
-    if (opt.order_asap) reorder_asap(plan, b.accs, NT + NT * opt.nslots + 1);
+    if (opt.order_mode == 2) reorder_list(plan, b.accs, NT + NT * opt.nslots + 1, opt.sched_width);
+    else if (opt.order_asap) reorder_asap(plan, b.accs, NT + NT * opt.nslots + 1);
   }
   // longest chain of compute tasks (COPY/LOAD/STORE weigh 0)
   std::vector<int64_t> depth(plan.tasks.size(), 0);

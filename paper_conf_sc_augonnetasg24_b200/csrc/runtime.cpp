@@ -206,7 +206,7 @@ Context& ctx() {
   return c;
 }
 
-constexpr int kCritStreams = 4;
+constexpr int kCritStreams = 6;  // 0: panel chain, 1: its feeders, 2..5: other urgent tasks by row
 constexpr int kCopyStreams = 2;
 constexpr size_t kCacheMax = 4;
 
@@ -227,6 +227,8 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   // (STF_ORDER_ASAP: -1 auto = COLMAJOR calls, 0 never, 1 always)
   const int64_t asap = env_int("STF_ORDER_ASAP", -1);
   po.order_asap = asap < 0 ? load : asap != 0;
+  po.order_mode = (int)env_int("STF_ORDER_MODE", 0);
+  po.sched_width = (int)std::max<int64_t>(1, env_int("STF_SCHED_WIDTH", 3));
   po.lookahead = o.lookahead != 0;
   po.push = o.push != 0 && o.trsm >= 2;
   return po;
@@ -252,6 +254,13 @@ struct Lowerer {
     if (!X.opt.priority) return lo;
     const int v = hi + (5 - t.prio);
     return v > lo ? lo : v;
+  }
+
+  static cudaError_t trace_record(cudaEvent_t ev, cudaStream_t s) {
+    cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(s, &st);
+    return st == cudaStreamCaptureStatusActive ? cudaEventRecordWithFlags(ev, s, cudaEventRecordExternal)
+                                               : cudaEventRecord(ev, s);
   }
 
   int body(const stf::Task& t, size_t tidx, cudaStream_t s, int prio) {
@@ -468,10 +477,10 @@ struct Lowerer {
         CUDA_TRY(cudaStreamWaitEvent(s, X.events[(size_t)*q], 0), "stream wait event");
       }
       // debug timeline: timing events (external record nodes when captured), no SM work
-      if (!X.trace.empty()) CUDA_TRY(cudaEventRecordWithFlags(X.trace[2 * t], s, cudaEventRecordExternal), "trace");
+      if (!X.trace.empty()) CUDA_TRY(trace_record(X.trace[2 * t], s), "trace");
       int r = body(task, t, s, prio_of(task));
       if (r) return r;
-      if (!X.trace.empty()) CUDA_TRY(cudaEventRecordWithFlags(X.trace[2 * t + 1], s, cudaEventRecordExternal), "trace");
+      if (!X.trace.empty()) CUDA_TRY(trace_record(X.trace[2 * t + 1], s), "trace");
       if (X.mp) {  // publish remote replicas written by this task (COPY target, fused-push mirrors)
         auto signal = [&](int64_t b) -> int {
           const int dst = P.buffers[(size_t)b].slot;
@@ -596,6 +605,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   // 23 vs 60 ms), so it is used there (STF_ORDER_ASAP = 1 forces it).
   po.copy_cost = X.kind == STF_DESC_HOST_COLMAJOR ? 2.7 * 1024.0 / (double)X.nb : 0.05;
   if (env_int("STF_ORDER_ASAP", -1) < 0) po.order_asap = colmajor && X.nb >= 1024;
+
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
     po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames

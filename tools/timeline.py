@@ -57,6 +57,16 @@ if host:
     ld = R[R[:, 0] == 5]
     print("LOAD end ms by column:", " ".join("%d:%.1f" % (j, ld[ld[:, 2] == j][:, 6].max() / 1e6)
                                             for j in range(0, n // nb, max(1, n // nb // 16))))
+# the critical chain POTRF(k) -> TRSM(k+1,k) -> SYRK(k+1,k) -> POTRF(k+1): start / end (ms)
+if n // nb <= 32:
+    def find(kind, i, j, k):
+        sel = R[(R[:, 0] == kind) & (R[:, 1] == i) & (R[:, 2] == j) & (R[:, 3] == k)]
+        return (sel[0, 5] / 1e6, sel[0, 6] / 1e6) if len(sel) else (float("nan"),) * 2
+    for k in range(min(n // nb, 12)):
+        p_ = find(0, k, k, k)
+        t_ = find(1, k + 1, k, k)
+        s_ = find(2, k + 1, k + 1, k)
+        print("k=%2d POTRF %.3f-%.3f  TRSM(k+1) %.3f-%.3f  SYRK(k+1) %.3f-%.3f" % (k, *p_, *t_, *s_))
 # flop-weighted activity profile: GEMM/SYRK/TRSM flops completed per bin (task flops spread over its span)
 span = R[:, 6].max()
 edges = np.linspace(0, span, bins + 1)
