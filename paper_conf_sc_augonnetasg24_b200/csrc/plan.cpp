@@ -558,7 +558,8 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
     plan.graph = TaskGraph(NT + NT * opt.nslots + 1);
     Builder b(plan, T);
     b.run();
-    if (opt.order_mode == 2) reorder_list(plan, b.accs, NT + NT * opt.nslots + 1, opt.sched_width);
+    if (opt.order_mode == 2)
+      reorder_list(plan, b.accs, NT + NT * opt.nslots + 1, opt.sched_width > 0 ? opt.sched_width : 2);
     else if (opt.order_asap) reorder_asap(plan, b.accs, NT + NT * opt.nslots + 1);
   }
   // longest chain of compute tasks (COPY/LOAD/STORE weigh 0)

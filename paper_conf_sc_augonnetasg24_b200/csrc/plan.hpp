@@ -57,6 +57,7 @@ struct PlanOptions {
                             // the runtime sets it for COLMAJOR calls (LOAD/STORE tasks)
   int order_mode = 0;       // 2: re-submit in simulated list-scheduling order (plan.cpp reorder_list)
   int sched_width = 3;      // order_mode 2: compute tasks a GPU slot runs at a time in the model
+                            // (the runtime derives it from nb and the SM count)
   double copy_cost = 0;     // order_asap: a tile copy in GEMM-tile times (0: 2.7, nb = 1024)
   bool lookahead = true;   // false: a FENCE task (RW on every tile) closes each panel step, so
                            // step k+1 starts only when step k is complete (ablation, NEXT-1)

@@ -225,10 +225,9 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.with_store = store;
   // submission in order of earliest start for plans with host/device transfers
   // (STF_ORDER_ASAP: -1 auto = COLMAJOR calls, 0 never, 1 always)
-  const int64_t asap = env_int("STF_ORDER_ASAP", -1);
-  po.order_asap = asap < 0 ? load : asap != 0;
-  po.order_mode = (int)env_int("STF_ORDER_MODE", 0);
-  po.sched_width = (int)std::max<int64_t>(1, env_int("STF_SCHED_WIDTH", 3));
+  po.order_asap = env_int("STF_ORDER_ASAP", 0) != 0;
+  po.order_mode = (int)std::max<int64_t>(0, env_int("STF_ORDER_MODE", 0));
+  po.sched_width = (int)std::max<int64_t>(0, env_int("STF_SCHED_WIDTH", 0));  // 0: from nb (prepare)
   po.lookahead = o.lookahead != 0;
   po.push = o.push != 0 && o.trsm >= 2;
   return po;
@@ -598,13 +597,30 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   const int64_t T = X.n / X.nb;
   const bool colmajor = X.kind != STF_DESC_TILED_2DBC;
   stf::PlanOptions po = plan_options(X.opt, X.P, X.Q, X.ngpus, colmajor, colmajor);
-  // tile copy time in GEMM-tile times for the early-start order: PCIe ~55 GB/s vs
-  // a 2 nb^3 tile update at ~35 TF/s (2.7 at nb = 1024); device copies ~free.
-  // The order pays off with tiles of order >= 1024 (n = 32768: e2e 396 -> 350 ms);
-  // with small tiles the captured program order was faster (n = 8192, nb = 256:
-  // 23 vs 60 ms), so it is used there (STF_ORDER_ASAP = 1 forces it).
-  po.copy_cost = X.kind == STF_DESC_HOST_COLMAJOR ? 2.7 * 1024.0 / (double)X.nb : 0.05;
-  if (env_int("STF_ORDER_ASAP", -1) < 0) po.order_asap = colmajor && X.nb >= 1024;
+  // Scheduling model of the submission order (plan.cpp reorder_list), in units of
+  // one nb^3 GEMM task's duration while `width` of them share the GPU: a tile
+  // update has nb^2 / 8192 CTAs of 128 x 64 at 2 per SM, so about
+  // width = SMs * 16384 / nb^2 run at once (2 at nb = 1024, 9 at nb = 512); a
+  // PCIe tile copy (nb^2 * 8 B at ~54 GB/s) against 2 nb^3 flop at ~35 TFLOP/s per
+  // width: copy_cost = 2592 / (width * nb) units; device copies ~free.
+  {
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, C.slots[0].device);
+    if (po.sched_width <= 0)
+      po.sched_width = (int)std::min<int64_t>(64, std::max<int64_t>(1, (int64_t)sms * 16384 / (X.nb * X.nb)));
+    po.copy_cost = X.kind == STF_DESC_HOST_COLMAJOR ? 2592.0 / ((double)po.sched_width * (double)X.nb) : 0.02;
+  }
+  // Submission order (profiles/r01/submission_order.txt): with tiles of order
+  // >= 512 the plan is re-submitted in simulated list-scheduling order - the panel
+  // chain ahead of the bulk updates of its step, the transfers of a COLMAJOR call
+  // next to the tasks that need them - for COLMAJOR calls (HOST n = 32768: 396 ->
+  // 358 ms; n = 16384, nb = 512: 67 -> 58 ms) and for device tiles when T <= 16,
+  // where the chain bounds the time (n = 8192: POTRF(1) starts 1.3 ms earlier,
+  // nb = 512 +12%, nb = 1024 +2%; n = 16384, nb = 1024 +2%).  Device tiles with
+  // T > 16 keep program order (n = 32768: -0.3%, within noise), as does nb = 256
+  // (-12%).  STF_ORDER_MODE overrides (0 program order, 2 list); STF_ORDER_ASAP=1
+  // selects the earliest-start order instead.
+  if (env_int("STF_ORDER_MODE", -1) < 0) po.order_mode = (X.nb >= 512 && (colmajor || T <= 16)) ? 2 : 0;
 
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
@@ -868,19 +884,15 @@ bool host_pinned(const void* ptr) {
   return a.type == cudaMemoryTypeHost;
 }
 
-// HOST_COLMAJOR calls are lowered eagerly onto the streams: pageable memory
-// cannot be captured, and in-core with pinned memory the captured graph ran the
-// early-start submission order ~10% slower end to end than the streams
-// (n = 32768: 386 vs 350 ms, profiles/r01/e2e_order.txt) - for tiles of order
-// >= 1024 only: with smaller tiles the host cannot issue the many short tasks fast
-// enough (n = 8192, nb = 256: 38.9 ms eager vs 23 ms captured in program order).
-// STF_HOST_GRAPH=1 always captures.  Out-of-core plans keep the graph when pinned.
+// HOST_COLMAJOR calls on pageable memory are lowered eagerly onto the streams
+// (pageable copies cannot be captured); STF_HOST_EAGER=1 forces the eager
+// lowering for pinned memory too.  The eager path's speed depends on how the
+// driver maps the ~40 streams onto its hardware queues (measured 350 to 388 ms
+// at n = 32768 for the same plan), the captured graph does not (357 ms).
 bool host_eager(const Context& C, const stf_matrix_desc* d, int64_t n, int64_t nb, int ngpus) {
+  (void)C; (void)n; (void)nb; (void)ngpus;
   if (d->kind != STF_DESC_HOST_COLMAJOR) return false;
-  if (!host_pinned(d->ptr)) return true;
-  const int64_t T = nb > 0 ? n / nb : 0;
-  const bool ooc = ngpus == 1 && C.opt.mem_cap_tiles > 0 && C.opt.mem_cap_tiles < T * (T + 1) / 2;
-  return !ooc && nb >= 1024 && !env_int("STF_HOST_GRAPH", 0);
+  return !host_pinned(d->ptr) || env_int("STF_HOST_EAGER", 0) != 0;
 }
 
 int ensure_kernel_attrs(int dev) {

@@ -131,14 +131,15 @@ def test_fused_push_replaces_panel_copies(T, p, q, known):
         assert np.array_equal(R[np.ix_(comp, comp)], Ro)
 
 
-@pytest.mark.parametrize("T,p,q", [(6, 1, 1), (8, 2, 2), (8, 2, 4), (5, 1, 2)])
-def test_earliest_start_order_same_dag(T, p, q, monkeypatch):
-    """The early-start re-submission (plan.cpp reorder_asap, used for COLMAJOR
-    calls) is a topological order of the program-order DAG, and re-applying the
-    STF rule in that order yields the same DAG (edges identical up to the task
-    relabelling): only the stream-order chains change."""
+@pytest.mark.parametrize("T,p,q", [(6, 1, 1), (8, 2, 2), (8, 2, 4), (5, 1, 2), (16, 1, 1)])
+@pytest.mark.parametrize("order", [("STF_ORDER_ASAP", "1"), ("STF_ORDER_MODE", "2")], ids=["asap", "list"])
+def test_submission_orders_same_dag(T, p, q, order, monkeypatch):
+    """The re-submission orders (plan.cpp reorder_asap / reorder_list, the latter
+    the default for nb >= 512) are topological orders of the program-order DAG,
+    and re-applying the STF rule in that order yields the same DAG (edges
+    identical up to the task relabelling): only the stream-order chains change."""
     e0, k0, ijk0, st0 = stf.dag(T, p, q)
-    monkeypatch.setenv("STF_ORDER_ASAP", "1")
+    monkeypatch.setenv(*order)
     e1, k1, ijk1, st1 = stf.dag(T, p, q)
     keys0 = [(k, *x) for k, x in zip(k0, ijk0)]
     keys1 = [(k, *x) for k, x in zip(k1, ijk1)]

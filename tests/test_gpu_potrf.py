@@ -299,21 +299,27 @@ def test_colmajor_descriptors(stf, where, order, ngpus):
 
 
 @pytest.mark.parametrize("ngpus", [1, 2])
-def test_host_colmajor_early_start_order_same_bits(stf, ngpus):
-    """nb >= 1024 HOST_COLMAJOR calls are re-submitted in earliest-start order and
-    lowered onto the streams; same DAG, so the same bits as the
-    device-resident tiles."""
+def test_host_colmajor_submission_orders_same_bits(stf, ngpus, monkeypatch):
+    """HOST_COLMAJOR calls with nb >= 512 are re-submitted in list-scheduling
+    order; that order, the earliest-start order and the eager lowering
+    all keep the DAG, so the same bits as the device-resident tiles."""
     import torch
 
     n, nb = 4096, 1024
     ref = _bits(stf, n, nb, 1, ngpus, seed=7)
     A = synth.spd_matrix(7, n)
-    t = torch.from_numpy(np.ascontiguousarray(A)).pin_memory().t()  # column-major view
-    assert stf.potrf(t, nb, ngpus=ngpus) == 0
-    st = stf.last_stats()
-    assert st["graph_nodes"] == 0 and st["host_loads"] == 10  # eager lowering, lower tiles loaded
-    got = np.tril(t.numpy())
-    assert np.array_equal(got, np.tril(ref))
+    for env in ({}, {"STF_ORDER_MODE": "0", "STF_ORDER_ASAP": "1"}, {"STF_HOST_EAGER": "1"}):
+        for k, v in env.items():
+            monkeypatch.setenv(k, v)
+        stf.finalize()  # the environment is read when a plan is built: drop the memoised plans
+        stf.init(NSLOTS, [0] * NSLOTS)
+        t = torch.from_numpy(np.ascontiguousarray(A)).pin_memory().t()  # column-major view
+        assert stf.potrf(t, nb, ngpus=ngpus) == 0
+        st = stf.last_stats()
+        assert st["host_loads"] == 10 and (st["graph_nodes"] == 0) == ("STF_HOST_EAGER" in env)
+        assert np.array_equal(np.tril(t.numpy()), np.tril(ref)), env
+        for k in env:
+            monkeypatch.delenv(k)
 
 
 def test_n_zero(stf):
