@@ -10,8 +10,8 @@ prof gemm_tile gemm_nt 0 1024 1024 1024
 prof gemm_full gemm_nt 0 8192 8192 1024
 prof syrk_tile gemm_nt 1 1024 1024 1024
 prof trsm_res_tile trsm_res 2 1024 1024 0
-prof trsm_panel_tile trsm_panel 2 1024 1024 0 STF_TRSM=2
-prof trsm_w256 trsm_panel 2 1024 256 0 STF_TRSM=2
+prof trsm_panel_tile trsm_panel 2 1024 1024 0 "STF_TRSM=2 STF_TRSM_ROWS=128"
+prof trsm_w256 trsm_panel 2 1024 256 0 "STF_TRSM=2 STF_TRSM_ROWS=128"
 prof potrf_tile dataflow 3 1024 1024 0
 timeout 900 ncu --graph-profiling graph --nvtx --nvtx-include "stf_potrf/" --clock-control none \
   --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,lts__t_bytes.sum,sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed \
