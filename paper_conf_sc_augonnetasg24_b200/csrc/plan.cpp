@@ -446,8 +446,18 @@ static void reorder_asap(Plan& plan, const std::vector<std::vector<Access>>& acc
 // graph executor / stream queues sees the tasks the GPU will run next - the
 // panel chain before the bulk updates of the same step.  A topological order,
 // so the DAG is unchanged (see reorder_asap).
-static void reorder_list(Plan& plan, const std::vector<std::vector<Access>>& accs, int64_t ndata, int width) {
+static void reorder_list(Plan& plan, const std::vector<std::vector<Access>>& accs, int64_t ndata, int width,
+                         int64_t tail_steps) {
   const size_t n = plan.tasks.size();
+  // tail_steps > 0: only the tasks from POTRF(T - tail_steps) on (a suffix of the
+  // program order) are re-ordered; the prefix keeps program order
+  size_t first = 0;
+  if (tail_steps > 0 && tail_steps < plan.T)
+    for (size_t t = 0; t < n; ++t)
+      if (plan.tasks[t].kind == K_POTRF && plan.tasks[t].k == plan.T - tail_steps) {
+        first = t;
+        break;
+      }
   const double copy_cost = plan.opt.copy_cost > 0 ? plan.opt.copy_cost : 2.7;
   auto is_copy = [](int32_t k) { return k == K_COPY || k == K_LOAD || k == K_STORE; };
   auto cost = [&](const Task& t) -> double {
@@ -521,7 +531,7 @@ static void reorder_list(Plan& plan, const std::vector<std::vector<Access>>& acc
   }
   std::vector<size_t> ord(n);
   for (size_t t = 0; t < n; ++t) ord[t] = t;
-  std::stable_sort(ord.begin(), ord.end(), [&](size_t a, size_t b) { return start[a] < start[b]; });
+  std::stable_sort(ord.begin() + (ptrdiff_t)first, ord.end(), [&](size_t a, size_t b) { return start[a] < start[b]; });
   std::vector<Task> tasks(n);
   TaskGraph g(ndata);
   for (size_t r = 0; r < n; ++r) {
@@ -559,7 +569,7 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
     Builder b(plan, T);
     b.run();
     if (opt.order_mode == 2)
-      reorder_list(plan, b.accs, NT + NT * opt.nslots + 1, opt.sched_width > 0 ? opt.sched_width : 2);
+      reorder_list(plan, b.accs, NT + NT * opt.nslots + 1, opt.sched_width > 0 ? opt.sched_width : 2, opt.order_tail);
     else if (opt.order_asap) reorder_asap(plan, b.accs, NT + NT * opt.nslots + 1);
   }
   // longest chain of compute tasks (COPY/LOAD/STORE weigh 0)

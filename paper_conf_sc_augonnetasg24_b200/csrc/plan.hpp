@@ -56,6 +56,7 @@ struct PlanOptions {
   bool order_asap = false;  // re-submit the tasks in order of earliest start (see plan.cpp);
                             // the runtime sets it for COLMAJOR calls (LOAD/STORE tasks)
   int order_mode = 0;       // 2: re-submit in simulated list-scheduling order (plan.cpp reorder_list)
+  int64_t order_tail = 0;   // order_mode 2: re-order only the last order_tail panel steps (0: all)
   int sched_width = 3;      // order_mode 2: compute tasks a GPU slot runs at a time in the model
                             // (the runtime derives it from nb and the SM count)
   double copy_cost = 0;     // order_asap: a tile copy in GEMM-tile times (0: 2.7, nb = 1024)

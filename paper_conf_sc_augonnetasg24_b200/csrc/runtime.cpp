@@ -227,6 +227,7 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   // (STF_ORDER_ASAP: -1 auto = COLMAJOR calls, 0 never, 1 always)
   po.order_asap = env_int("STF_ORDER_ASAP", 0) != 0;
   po.order_mode = (int)std::max<int64_t>(0, env_int("STF_ORDER_MODE", 0));
+  po.order_tail = std::max<int64_t>(0, env_int("STF_ORDER_TAIL", 0));
   po.sched_width = (int)std::max<int64_t>(0, env_int("STF_SCHED_WIDTH", 0));  // 0: from nb (prepare)
   po.lookahead = o.lookahead != 0;
   po.push = o.push != 0 && o.trsm >= 2;

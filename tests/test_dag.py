@@ -149,3 +149,19 @@ def test_submission_orders_same_dag(T, p, q, order, monkeypatch):
     assert all(a < b for a, b in e1)  # submission order is topological
     assert {(perm[a], perm[b]) for a, b in e0} == set(e1)
     assert st1["critical_path"] == st0["critical_path"] and st1["edges"] == st0["edges"]
+
+
+def test_list_order_submits_the_panel_chain_early(monkeypatch):
+    """List-scheduling order (default for T <= 16 and COLMAJOR calls): POTRF(k+1)
+    is submitted as soon as its chain allows, ahead of bulk updates of step k that
+    are not its ancestors (in program order it comes after all of them)."""
+    T = 8
+    monkeypatch.setenv("STF_ORDER_MODE", "2")
+    e, k, ijk, st = stf.dag(T, 1, 1)
+    pos = {(kd, *x): t for t, (kd, x) in enumerate(zip(k, ijk))}
+    for step in range(T - 2):
+        assert pos[("POTRF", step + 1, step + 1, step + 1)] < pos[("GEMM", T - 1, T - 2, step)]
+    monkeypatch.setenv("STF_ORDER_MODE", "0")
+    e0, k0, ijk0, _ = stf.dag(T, 1, 1)
+    pos0 = {(kd, *x): t for t, (kd, x) in enumerate(zip(k0, ijk0))}
+    assert pos0[("POTRF", 1, 1, 1)] > pos0[("GEMM", T - 1, T - 2, 0)]
