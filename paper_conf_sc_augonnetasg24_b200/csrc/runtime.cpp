@@ -618,10 +618,13 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   // 358 ms; n = 16384, nb = 512: 67 -> 58 ms) and for device tiles when T <= 16,
   // where the chain bounds the time (n = 8192: POTRF(1) starts 1.3 ms earlier,
   // nb = 512 +12%, nb = 1024 +2%; n = 16384, nb = 1024 +2%).  Device tiles with
-  // T > 16 keep program order (n = 32768: -0.3%, within noise), as does nb = 256
-  // (-12%).  STF_ORDER_MODE overrides (0 program order, 2 list); STF_ORDER_ASAP=1
-  // selects the earliest-start order instead.
-  if (env_int("STF_ORDER_MODE", -1) < 0) po.order_mode = (X.nb >= 512 && (colmajor || T <= 16)) ? 2 : 0;
+  // T > 16 re-order only the last 8 panel steps, where the chain bounds the time
+  // again (n = 32768: +0.2%; all steps: -0.3%; n = 65536 +-0).  nb = 256 keeps
+  // program order (-12%).  STF_ORDER_MODE / STF_ORDER_TAIL override (mode 0
+  // program order, 2 list; tail 0 = all steps); STF_ORDER_ASAP=1 selects the
+  // earliest-start order instead.
+  if (env_int("STF_ORDER_MODE", -1) < 0) po.order_mode = X.nb >= 512 ? 2 : 0;
+  if (env_int("STF_ORDER_TAIL", -1) < 0) po.order_tail = (!colmajor && T > 16) ? 8 : 0;
 
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
