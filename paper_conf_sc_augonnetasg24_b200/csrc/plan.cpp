@@ -2,6 +2,7 @@
 #include "plan.hpp"
 
 #include <algorithm>
+#include <cstdlib>
 #include <climits>
 #include <queue>
 #include <set>
@@ -275,8 +276,89 @@ struct OocBuilder {
     }
   }
 
-  void run(int crit_streams, int bulk_streams, int load_stream, int store_stream, bool serial, bool priority) {
-    make_sequence();
+  // 2D-blocked order (ooc_order 1).  A tall super-column of width w re-reads
+  // about 1/w panel tiles per update; when the trailing column alone fills the
+  // budget, w is 1.  Here the block [j0, j1] is processed in row chunks of
+  // height r: the diagonal triangle first (all updates from k < j0, then
+  // factored right-looking inside), then each chunk of rows below it: updates
+  // from k < j0 (k outer: r + w panel tiles per k for r w GEMMs), then its
+  // TRSMs against the block's diagonal and the block-internal updates.  Every
+  // tile still receives its updates k = 0, 1, ... in order and then its TRSM,
+  // so L is bit-identical.  (w, r) minimise 1/w + 1/r under
+  // w(w+1)/2 + r w <= 3F/5 (the other frames stream panel tiles; 3/5 gave
+  // the fewest loads over F = 33..396 at T = 32 among 30..70%); a single
+  // chunk is the tall super-column.
+  void choose_block(int64_t j0, int64_t& w_out, int64_t& r_out) const {
+    const int64_t B = std::max<int64_t>(F * 3 / 5, 1);
+    double best = 1e30;
+    w_out = 1;
+    r_out = T - j0 - 1;
+    for (int64_t w = 1; w <= T - j0; ++w) {
+      const int64_t rest = T - j0 - w;  // rows below the block
+      const int64_t tri = w * (w + 1) / 2;
+      if (tri > B && w > 1) break;
+      int64_t r = rest == 0 ? 0 : std::min(rest, std::max<int64_t>((B - tri) / w, 1));
+      const double cost = 1.0 / (double)w + (rest > 0 ? 1.0 / (double)r : 0.0);
+      if (cost < best - 1e-12) {
+        best = cost;
+        w_out = w;
+        r_out = r;
+      }
+    }
+  }
+
+  void make_sequence_2d() {
+    int64_t j0 = 0;
+    while (j0 < T) {
+      int64_t w, r;
+      choose_block(j0, w, r);
+      const int64_t j1 = j0 + w - 1;
+      // diagonal triangle of the block
+      for (int64_t k = 0; k < j0; ++k)
+        for (int64_t j = j0; j <= j1; ++j) {
+          const int d = (int)(j - j0);
+          seq.push_back({K_SYRK, (int32_t)j, (int32_t)j, (int32_t)k, d == 0 ? 5 : d == 1 ? 3 : 2, id(j, k), -1, id(j, j)});
+          for (int64_t i = j + 1; i <= j1; ++i)
+            seq.push_back({K_GEMM, (int32_t)i, (int32_t)j, (int32_t)k, d == 0 ? 4 : d == 1 ? 2 : 1, id(i, k), id(j, k),
+                           id(i, j)});
+        }
+      for (int64_t j = j0; j <= j1; ++j) {
+        seq.push_back({K_POTRF, (int32_t)j, (int32_t)j, (int32_t)j, 5, -1, -1, id(j, j)});
+        for (int64_t i = j + 1; i <= j1; ++i)
+          seq.push_back({K_TRSM, (int32_t)i, (int32_t)j, (int32_t)j, i == j + 1 ? 5 : 4, id(j, j), -1, id(i, j)});
+        for (int64_t jj = j + 1; jj <= j1; ++jj) {
+          seq.push_back({K_SYRK, (int32_t)jj, (int32_t)jj, (int32_t)j, jj == j + 1 ? 5 : 3, id(jj, j), -1, id(jj, jj)});
+          for (int64_t i = jj + 1; i <= j1; ++i)
+            seq.push_back({K_GEMM, (int32_t)i, (int32_t)jj, (int32_t)j, jj == j + 1 ? 4 : 2, id(i, j), id(jj, j),
+                           id(i, jj)});
+        }
+      }
+      // row chunks below it
+      for (int64_t i0 = j1 + 1; i0 < T; i0 += r) {
+        const int64_t i1 = std::min(T - 1, i0 + r - 1);
+        for (int64_t k = 0; k < j0; ++k)
+          for (int64_t j = j0; j <= j1; ++j)
+            for (int64_t i = i0; i <= i1; ++i)
+              seq.push_back({K_GEMM, (int32_t)i, (int32_t)j, (int32_t)k, j == j0 ? 2 : 1, id(i, k), id(j, k), id(i, j)});
+        for (int64_t j = j0; j <= j1; ++j) {
+          for (int64_t i = i0; i <= i1; ++i)
+            seq.push_back({K_TRSM, (int32_t)i, (int32_t)j, (int32_t)j, 4, id(j, j), -1, id(i, j)});
+          for (int64_t jj = j + 1; jj <= j1; ++jj)
+            for (int64_t i = i0; i <= i1; ++i)
+              seq.push_back({K_GEMM, (int32_t)i, (int32_t)jj, (int32_t)j, jj == j + 1 ? 2 : 1, id(i, j), id(jj, j),
+                             id(i, jj)});
+        }
+      }
+      j0 = j1 + 1;
+    }
+  }
+
+  void run(int crit_streams, int bulk_streams, int load_stream, int store_stream, bool serial, bool priority,
+           int order) {
+    if (order == 1)
+      make_sequence_2d();
+    else
+      make_sequence();
     const int64_t NT = p.ntiles();
     p.buffers.clear();
     for (int64_t f = 0; f < F; ++f) p.buffers.push_back(Buffer{-1, -1, 0, false});
@@ -561,7 +643,10 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
     const int base = plan.opt.serial ? 1 : plan.opt.crit_streams + plan.opt.bulk_streams;
     OocBuilder b(plan, T, opt.frames);
     b.run(plan.opt.crit_streams, plan.opt.bulk_streams, base, base + (plan.opt.copy_streams > 1 ? 1 : 0),
-          plan.opt.serial, plan.opt.priority);
+          plan.opt.serial, plan.opt.priority,
+          // auto: 2D-blocked while less than half the tiles fit (measured at n = 32768,
+          // nb = 1024: F = 33 / 66 / 132 +58% / +42% / +2%, F = 264 -1.6%)
+          plan.opt.ooc_order >= 0 ? plan.opt.ooc_order : (2 * opt.frames < NT ? 1 : 0));
   } else {
     plan.opt.frames = 0;
     // dense datum ids: home tiles + at most one replica per (tile, slot)

@@ -90,6 +90,7 @@ struct Options {
   int64_t threads = 8;  // eager backend: host submission threads (one per slot group)
   int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
   int64_t mem_cap_tiles = 0;  // HOST_COLMAJOR on one GPU: device tile frames (0 = whole matrix resident)
+  int64_t ooc_order = -1;     // out-of-core program order: 0 tall super-columns, 1 2D-blocked, -1 auto
   int64_t trsm_res_tail = 8192;  // trsm 3: every TRSM(i,k) resident-panel once the trailing order n - k nb <= this
   int64_t trsm_rows = 128;  // row panel: rows per CTA of the non-critical TRSM panels (32, 64 or 128)
 };
@@ -98,7 +99,7 @@ struct Options {
 bool same_plan_options(const Options& a, int64_t a_graph, const Options& b) {
   return a.streams == b.streams && a.serial == b.serial && a_graph == b.graph && a.priority == b.priority &&
          a.dataflow == b.dataflow && a.trsm == b.trsm && a.trsm_split == b.trsm_split && a.push == b.push &&
-         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.trsm_res_tail == b.trsm_res_tail &&
+         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.ooc_order == b.ooc_order && a.trsm_res_tail == b.trsm_res_tail &&
          a.trsm_rows == b.trsm_rows;
 }
 
@@ -629,6 +630,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
     po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames
+  po.ooc_order = (int)X.opt.ooc_order;
   stf::build_plan(X.plan, T, po);
   const stf::Plan& P = X.plan;
   const size_t tile_bytes = (size_t)(X.nb * X.nb) * sizeof(double);
@@ -937,6 +939,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.trsm_rows = env_int("STF_TRSM_ROWS", 128);
   C.opt.push = env_int("STF_PUSH", 0);
   C.opt.mem_cap_tiles = env_int("STF_MEM_CAP_TILES", 0);
+  C.opt.ooc_order = env_int("STF_OOC_ORDER", -1);
   C.opt.streams = env_int("STF_STREAMS", 32);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
@@ -1078,6 +1081,11 @@ int stf_set_option(const char* name, int64_t value) {
     if (value != 0 && value < 3) return fail(-105, "mem_cap_tiles must be 0 (no cap) or >= 3 (a GEMM holds 3 tiles)");
     C.opt.mem_cap_tiles = value;
   }
+  else if (n == "ooc_order") {
+    if (value < -1 || value > 1)
+      return fail(-105, "ooc_order must be -1 (auto), 0 (tall super-columns) or 1 (2D-blocked)");
+    C.opt.ooc_order = value;
+  }
   else if (n == "threads") {
     if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
     C.opt.threads = value;
@@ -1107,6 +1115,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "trsm_rows") *value = C.opt.trsm_rows;
   else if (n == "push") *value = C.opt.push;
   else if (n == "mem_cap_tiles") *value = C.opt.mem_cap_tiles;
+  else if (n == "ooc_order") *value = C.opt.ooc_order;
   else if (n == "threads") *value = C.opt.threads;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;
@@ -1320,6 +1329,7 @@ int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t* edges, int64_t 
   const bool ooc = ctx().opt.mem_cap_tiles > 0 && p * q == 1 && ctx().opt.mem_cap_tiles < T * (T + 1) / 2;
   stf::PlanOptions po = plan_options(o, p, q, p * q, ooc, ooc);
   if (ooc) po.frames = ctx().opt.mem_cap_tiles;
+  po.ooc_order = (int)ctx().opt.ooc_order;
   stf::build_plan(plan, T, po);
   double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   int64_t e = 0;

@@ -102,3 +102,26 @@ def test_out_of_core_rejected_on_several_gpus(stf):
         assert e.value.code == -105
     finally:
         stf.set_option("mem_cap_tiles", 0)
+
+
+@pytest.mark.parametrize("ooc_order", [0, 1])
+def test_out_of_core_orders_bit_equal(stf, ooc_order):
+    """Both program orders of the out-of-core plan (tall super-columns, 2D-blocked
+    row chunks) give the in-core call's bits; the 2D order loads fewer tiles."""
+    n, nb, cap = 4096, 256, 20
+    A = synth.spd_matrix(9, n)
+    ref, _, _ = _factor(stf, A, nb, 0)
+    stf.set_option("ooc_order", ooc_order)
+    try:
+        got, info, st = _factor(stf, A, nb, cap)
+    finally:
+        stf.set_option("ooc_order", -1)
+    assert info == 0 and st["frames"] == cap
+    assert np.array_equal(np.tril(got), np.tril(ref))
+    stf.set_option("ooc_order", 1 - ooc_order)
+    try:
+        _, _, st_other = _factor(stf, A, nb, cap)
+    finally:
+        stf.set_option("ooc_order", -1)
+    two_d, tall = (st, st_other) if ooc_order == 1 else (st_other, st)
+    assert two_d["host_loads"] < tall["host_loads"]

@@ -20,15 +20,17 @@ import synth
 NB = 4  # tile order for the emulation (values are irrelevant to the schedule)
 
 
-def _plan(T, p, q, frames=0, lookahead=1):
+def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1):
     stf.set_option("mem_cap_tiles", frames)
     stf.set_option("lookahead", lookahead)
+    stf.set_option("ooc_order", ooc_order)
     try:
         edges, kinds, ijk, st = stf.dag(T, p, q)
         io, nbuf = stf.dag_io(len(kinds))
     finally:
         stf.set_option("mem_cap_tiles", 0)
         stf.set_option("lookahead", 1)
+        stf.set_option("ooc_order", -1)
     return edges, kinds, ijk, io, nbuf, st
 
 
@@ -105,10 +107,12 @@ def test_distributed_plan_any_topological_order(T, p, q, lookahead):
         assert np.array_equal(got, ref), (seed, np.abs(got - ref).max())
 
 
-@pytest.mark.parametrize("T,frames", [(4, 3), (4, 5), (6, 3), (6, 4), (6, 7), (6, 12), (8, 6), (8, 20), (9, 10)])
-def test_out_of_core_plan_any_topological_order(T, frames):
+@pytest.mark.parametrize("ooc_order", [0, 1, -1])
+@pytest.mark.parametrize("T,frames", [(4, 3), (4, 5), (6, 3), (6, 4), (6, 7), (6, 12), (8, 6), (8, 20), (9, 10),
+                                      (12, 9), (12, 30)])
+def test_out_of_core_plan_any_topological_order(T, frames, ooc_order):
     A = synth.spd_matrix(11, T * NB)
-    edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames)
+    edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames, ooc_order=ooc_order)
     NT = T * (T + 1) // 2
     assert st["frames"] == frames and nbuf == frames
     assert "COPY" not in kinds
@@ -162,3 +166,17 @@ def test_out_of_core_traffic_left_looking():
     assert st_big["host_loads"] <= 3 * NT
     _, _, _, _, _, st_none = _plan(T, 1, 1, frames=NT)  # cap >= matrix: no out-of-core plan
     assert st_none["frames"] == 0 and st_none["host_loads"] == 0
+
+
+def test_out_of_core_2d_order_cuts_panel_reloads():
+    """The 2D-blocked order (row chunks under each column block) re-reads fewer
+    panel tiles than tall super-columns once a trailing column alone fills the
+    frames (T = 32: the bench's n = 32768, nb = 1024), and never loads a tile
+    less than once or writes one back more than once per eviction."""
+    T = 32
+    NT = T * (T + 1) // 2
+    for frames, gain in ((33, 0.75), (66, 0.75), (132, 0.95)):
+        st0 = _plan(T, 1, 1, frames=frames, ooc_order=0)[5]
+        st1 = _plan(T, 1, 1, frames=frames, ooc_order=1)[5]
+        assert NT <= st1["host_loads"] <= gain * st0["host_loads"], (frames, st0["host_loads"], st1["host_loads"])
+        assert st1["host_stores"] == NT
