@@ -241,6 +241,7 @@ struct OocBuilder {
     int64_t r0, r1, w;  // tile ids read (or -1) and written
   };
   std::vector<CT> seq;
+  std::vector<std::vector<Access>> accs;  // per task, for a re-ordered re-submission
 
   OocBuilder(Plan& plan, int64_t T_, int64_t F_) : p(plan), T(T_), F(F_) {}
 
@@ -394,6 +395,7 @@ struct OocBuilder {
       Task s{K_STORE, ij[0], ij[1], 0, 0, 0, store_stream, {f, -1}, -1};
       Access acc[2] = {{f, READ}, {host(tile_in[(size_t)f]), WRITE}};
       p.graph.submit(acc, 2);
+      accs.emplace_back(acc, acc + 2);
       p.tasks.push_back(s);
       p.nstores++;
       dirty[(size_t)f] = 0;
@@ -430,6 +432,7 @@ struct OocBuilder {
         Task l{K_LOAD, ij[0], ij[1], 0, 0, priority ? c.prio : 0, load_stream, {-1, -1}, f};
         Access acc[2] = {{host(t), READ}, {f, WRITE}};
         p.graph.submit(acc, 2);
+        accs.emplace_back(acc, acc + 2);
         p.tasks.push_back(l);
         p.nloads++;
         frame_of[(size_t)t] = f;
@@ -447,6 +450,7 @@ struct OocBuilder {
       if (t.in[1] >= 0) acc[n++] = {t.in[1], READ};
       acc[n++] = {t.out, RW};
       p.graph.submit(acc, n);
+      accs.emplace_back(acc, acc + n);
       p.tasks.push_back(t);
       dirty[(size_t)t.out] = 1;
       // refresh the next-use keys of the tiles just used
@@ -647,6 +651,8 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
           // auto: 2D-blocked while less than half the tiles fit (measured at n = 32768,
           // nb = 1024: F = 33 / 66 / 132 +58% / +42% / +2%, F = 264 -1.6%)
           plan.opt.ooc_order >= 0 ? plan.opt.ooc_order : (2 * opt.frames < NT ? 1 : 0));
+    if (opt.order_mode == 2 && opt.ooc_reorder)
+      reorder_list(plan, b.accs, opt.frames + NT + 1, opt.sched_width > 0 ? opt.sched_width : 2, 0);
   } else {
     plan.opt.frames = 0;
     // dense datum ids: home tiles + at most one replica per (tile, slot)

@@ -66,6 +66,7 @@ struct PlanOptions {
                            // push, NEXT-3) instead of COPY tasks at the first remote read
   int64_t frames = 0;      // > 0 (one slot, with_load/with_store): memory-capped out-of-core
                            // plan (NEXT-4) over this many device tile frames; see plan.cpp
+  bool ooc_reorder = true;  // order_mode 2 also re-orders out-of-core plans (loads by simulated start)
   int ooc_order = -1;      // out-of-core program order: 0 tall super-columns, 1 2D-blocked,
                            // -1 2D-blocked while fewer than half the tiles fit (plan.cpp)
 };

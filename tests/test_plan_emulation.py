@@ -107,10 +107,15 @@ def test_distributed_plan_any_topological_order(T, p, q, lookahead):
         assert np.array_equal(got, ref), (seed, np.abs(got - ref).max())
 
 
+@pytest.mark.parametrize("list_order", [False, True])
 @pytest.mark.parametrize("ooc_order", [0, 1, -1])
 @pytest.mark.parametrize("T,frames", [(4, 3), (4, 5), (6, 3), (6, 4), (6, 7), (6, 12), (8, 6), (8, 20), (9, 10),
                                       (12, 9), (12, 30)])
-def test_out_of_core_plan_any_topological_order(T, frames, ooc_order):
+def test_out_of_core_plan_any_topological_order(T, frames, ooc_order, list_order, monkeypatch):
+    """list_order: the plan re-submitted in simulated list-scheduling order
+    (STF_ORDER_MODE=2, what the runtime does at nb >= 512)."""
+    if list_order:
+        monkeypatch.setenv("STF_ORDER_MODE", "2")
     A = synth.spd_matrix(11, T * NB)
     edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames, ooc_order=ooc_order)
     NT = T * (T + 1) // 2
