@@ -131,8 +131,9 @@ const char *stf_last_error(void);
  *   "ooc_order" STF_OOC_ORDER  program order of an out-of-core plan: 1 2D-blocked (column
  *                           blocks swept in row chunks: fewer panel re-reads when a trailing
  *                           column alone fills the frames); 0 tall super-columns; -1 (default)
- *                           1 while the cap is below half the tiles, else 0.  Every order
- *                           gives bit-identical L.
+ *                           1 when the plan is re-submitted in list-scheduling order (nb >=
+ *                           512), else 1 while the cap is below half the tiles, else 0.  Every
+ *                           order gives bit-identical L.
  * Returns 0 or -105. */
 int stf_set_option(const char *name, int64_t value);
 int stf_get_option(const char *name, int64_t *value);

@@ -287,10 +287,11 @@ struct OocBuilder {
   // tile still receives its updates k = 0, 1, ... in order and then its TRSM,
   // so L is bit-identical.  (w, r) minimise 1/w + 1/r under
   // w(w+1)/2 + r w <= 3F/5 (the other frames stream panel tiles; 3/5 gave
-  // the fewest loads over F = 33..396 at T = 32 among 30..70%); a single
+  // the fewest loads over F = 33..396 at T = 32 among 30..70%, and time within
+  // 3% of the best of 40..80% at F = 33, 66, 132); a single
   // chunk is the tall super-column.
   void choose_block(int64_t j0, int64_t& w_out, int64_t& r_out) const {
-    const int64_t B = std::max<int64_t>(F * 3 / 5, 1);
+    const int64_t B = std::max<int64_t>(F * p.opt.ooc_budget_pct / 100, 1);
     double best = 1e30;
     w_out = 1;
     r_out = T - j0 - 1;
@@ -648,9 +649,11 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
     OocBuilder b(plan, T, opt.frames);
     b.run(plan.opt.crit_streams, plan.opt.bulk_streams, base, base + (plan.opt.copy_streams > 1 ? 1 : 0),
           plan.opt.serial, plan.opt.priority,
-          // auto: 2D-blocked while less than half the tiles fit (measured at n = 32768,
-          // nb = 1024: F = 33 / 66 / 132 +58% / +42% / +2%, F = 264 -1.6%)
-          plan.opt.ooc_order >= 0 ? plan.opt.ooc_order : (2 * opt.frames < NT ? 1 : 0));
+          // auto: 2D-blocked for re-ordered plans (n = 32768, nb = 1024: F = 33..396 all
+          // ahead of the tall order); in program order only while less than half the
+          // tiles fit (F = 33 / 66 / 132 +58% / +42% / +2%, F = 264 -1.6%)
+          plan.opt.ooc_order >= 0 ? plan.opt.ooc_order
+                                  : ((opt.order_mode == 2 && opt.ooc_reorder) || 2 * opt.frames < NT ? 1 : 0));
     if (opt.order_mode == 2 && opt.ooc_reorder)
       reorder_list(plan, b.accs, opt.frames + NT + 1, opt.sched_width > 0 ? opt.sched_width : 2, 0);
   } else {

@@ -67,8 +67,10 @@ struct PlanOptions {
   int64_t frames = 0;      // > 0 (one slot, with_load/with_store): memory-capped out-of-core
                            // plan (NEXT-4) over this many device tile frames; see plan.cpp
   bool ooc_reorder = true;  // order_mode 2 also re-orders out-of-core plans (loads by simulated start)
+  int ooc_budget_pct = 60;  // 2D order: % of the frames a block (triangle + row chunk) may fill
   int ooc_order = -1;      // out-of-core program order: 0 tall super-columns, 1 2D-blocked,
-                           // -1 2D-blocked while fewer than half the tiles fit (plan.cpp)
+                           // -1 auto: 2D-blocked if re-ordered, else while fewer than half
+                           // the tiles fit (plan.cpp)
 };
 
 // A "buffer" is one physical nb x nb tile instance: home tiles are buffers
