@@ -339,7 +339,7 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
     roof["kernels_alone"] = kern
     # dominant kernel: the GEMM tile update (GEMM+SYRK are (T-1)(T-2)/T^2 + (T-1)/T^2 of the flops)
     T = n // nb
-    tr = load_traffic()
+    tr = load_traffic(nb)
     dom = {"name": "gemm_nt_dmma (GEMM/SYRK tile update C -= A B^T)",
            "flop_share": round(((T - 1) * (T - 2) + (T - 1)) / T ** 2, 4),
            "launches_per_step": T * (T - 1) * (T - 2) // 6 + T * (T - 1) // 2,
@@ -351,8 +351,9 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
         roof["traffic"] = gt["traffic_bytes"]
         roof["traffic_src"] = gt["src"]
     roof["traffic_note"] = ("traffic = DRAM bytes of one whole-DAG graph launch (ncu --graph-profiling graph, "
-                            "committed under profiles/); algorithmic minimum 8.86 GB at n=32768 (lower tiles read "
-                            "and written once); per-kernel DRAM traffic of the GEMM tile in dominant_kernel")
+                            "committed under profiles/, null when none was captured at this n, nb); algorithmic "
+                            "minimum %.2f GB (lower tiles read and written once); per-kernel DRAM traffic of the GEMM "
+                            "tile in dominant_kernel (nb=1024 capture only)" % (2 * 8 * nb * nb * T * (T + 1) / 2 / 1e9))
 
     cpu = None
     if N == 1 and not args.no_cpu:
@@ -435,11 +436,13 @@ def load_graph_traffic(n, nb):
     return best
 
 
-def load_traffic():
-    """dram bytes per GEMM launch from the committed ncu --set full summary, if present."""
+def load_traffic(nb):
+    """dram bytes per GEMM launch from the committed ncu --set full summary, if
+    present and captured at this tile size (nb=1024)."""
     p = os.path.join(ROOT, "profiles", "gemm_traffic.json")
     try:
-        return json.load(open(p)).get("traffic_bytes_per_launch")
+        d = json.load(open(p))
+        return d.get("traffic_bytes_per_launch") if "nb=%d)" % nb in d.get("kernel", "") else None
     except (OSError, ValueError):
         return None
 

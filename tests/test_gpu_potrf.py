@@ -122,7 +122,7 @@ def oracle_8192():
     return A, L
 
 
-@pytest.mark.parametrize("nb", [256, 512, 1024])
+@pytest.mark.parametrize("nb", [256, 512, 1024, 2048])  # 2048: CFG4's tile (BASELINE configs[4])
 def test_parity_cfg1_nb_sweep(stf, oracle_8192, nb):
     A, Lo = oracle_8192
     M, info = _factor_spd(stf, 8192, nb, seed=1)
