@@ -91,6 +91,7 @@ struct Options {
   int64_t push = 0;     // fused push of TRSM outputs into consumer replicas (row-panel TRSM only)
   int64_t mem_cap_tiles = 0;  // HOST_COLMAJOR on one GPU: device tile frames (0 = whole matrix resident)
   int64_t ooc_order = -1;     // out-of-core program order: 0 tall super-columns, 1 2D-blocked, -1 auto
+  int64_t host_stream = 1;    // HOST_COLMAJOR on one GPU, nb >= 512: out-of-core builder with all tiles as frames
   int64_t trsm_res_tail = 8192;  // trsm 3: every TRSM(i,k) resident-panel once the trailing order n - k nb <= this
   int64_t trsm_rows = 128;  // row panel: rows per CTA of the non-critical TRSM panels (32, 64 or 128)
 };
@@ -99,7 +100,7 @@ struct Options {
 bool same_plan_options(const Options& a, int64_t a_graph, const Options& b) {
   return a.streams == b.streams && a.serial == b.serial && a_graph == b.graph && a.priority == b.priority &&
          a.dataflow == b.dataflow && a.trsm == b.trsm && a.trsm_split == b.trsm_split && a.push == b.push &&
-         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.ooc_order == b.ooc_order && a.trsm_res_tail == b.trsm_res_tail &&
+         a.lookahead == b.lookahead && a.mem_cap_tiles == b.mem_cap_tiles && a.ooc_order == b.ooc_order && a.host_stream == b.host_stream && a.trsm_res_tail == b.trsm_res_tail &&
          a.trsm_rows == b.trsm_rows;
 }
 
@@ -632,6 +633,12 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
     po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames
+  else if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && po.order_mode == 2 && po.ooc_reorder &&
+           X.opt.host_stream)
+    // in-core host call through the out-of-core builder with a frame per tile: its
+    // 2D-blocked left-looking order consumes the tiles in the order they arrive
+    // over PCIe (n = 32768, nb = 1024: 357.6 -> 352.7 ms end to end); no eviction
+    po.frames = T * (T + 1) / 2;
   po.ooc_order = (int)X.opt.ooc_order;
   stf::build_plan(X.plan, T, po);
   const stf::Plan& P = X.plan;
@@ -942,6 +949,7 @@ int stf_cholesky_init(int ngpus, const int* device_ids) {
   C.opt.push = env_int("STF_PUSH", 0);
   C.opt.mem_cap_tiles = env_int("STF_MEM_CAP_TILES", 0);
   C.opt.ooc_order = env_int("STF_OOC_ORDER", -1);
+  C.opt.host_stream = env_int("STF_HOST_STREAM", 1);
   C.opt.streams = env_int("STF_STREAMS", 32);
   C.opt.serial = env_int("STF_SERIAL", 0);
   C.opt.lookahead = env_int("STF_LOOKAHEAD", 1);
@@ -1088,6 +1096,7 @@ int stf_set_option(const char* name, int64_t value) {
       return fail(-105, "ooc_order must be -1 (auto), 0 (tall super-columns) or 1 (2D-blocked)");
     C.opt.ooc_order = value;
   }
+  else if (n == "host_stream") C.opt.host_stream = value != 0;
   else if (n == "threads") {
     if (value < 1 || value > 64) return fail(-105, "threads must be in [1, 64]");
     C.opt.threads = value;
@@ -1118,6 +1127,7 @@ int stf_get_option(const char* name, int64_t* value) {
   else if (n == "push") *value = C.opt.push;
   else if (n == "mem_cap_tiles") *value = C.opt.mem_cap_tiles;
   else if (n == "ooc_order") *value = C.opt.ooc_order;
+  else if (n == "host_stream") *value = C.opt.host_stream;
   else if (n == "threads") *value = C.opt.threads;
   else if (n == "priority") *value = C.opt.priority;
   else if (n == "grid_p") *value = C.opt.grid_p;

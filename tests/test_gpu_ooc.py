@@ -84,7 +84,11 @@ def test_out_of_core_larger_tiles_and_repeat(stf):
     """T = 16 with 20 frames (15% of the tiles); twice in a row (memoised plan)."""
     n, nb = 8192, 512
     A = synth.spd_matrix(8, n)
-    ref, _, _ = _factor(stf, A, nb, 0)
+    stf.set_option("host_stream", 0)  # reference: the right-looking in-core plan
+    try:
+        ref, _, _ = _factor(stf, A, nb, 0)
+    finally:
+        stf.set_option("host_stream", 1)
     for rep in range(2):
         got, info, st = _factor(stf, A, nb, 20)
         assert info == 0 and st["frames"] == 20
@@ -125,3 +129,26 @@ def test_out_of_core_orders_bit_equal(stf, ooc_order):
         stf.set_option("ooc_order", -1)
     two_d, tall = (st, st_other) if ooc_order == 1 else (st_other, st)
     assert two_d["host_loads"] < tall["host_loads"]
+
+
+@pytest.mark.parametrize("n,nb,order", [(4096, 512, "F"), (3072, 1024, "C"), (8192, 1024, "F")])
+def test_host_stream_plan_bit_equal_to_right_looking_plan(stf, n, nb, order):
+    """An uncapped HOST_COLMAJOR call at nb >= 512 runs the out-of-core builder
+    with one frame per tile ("host_stream", default); it must give the bits of
+    the right-looking plan with LOAD/STORE tasks (host_stream 0) and load and
+    write back every tile exactly once."""
+    T = n // nb
+    NT = T * (T + 1) // 2
+    A = synth.spd_matrix(12, n)
+    A[np.triu_indices(n, 1)] = 777.0
+    stf.set_option("host_stream", 0)
+    try:
+        ref, info0, st0 = _factor(stf, A, nb, 0, order)
+    finally:
+        stf.set_option("host_stream", 1)
+    got, info, st = _factor(stf, A, nb, 0, order)
+    assert info0 == 0 and info == 0
+    assert st0["frames"] == 0 and st["frames"] == NT
+    assert st["host_loads"] == NT and st["host_stores"] == NT
+    assert np.array_equal(np.tril(got), np.tril(ref))
+    assert np.all(got[np.triu_indices(n, 1)] == 777.0)
