@@ -194,6 +194,27 @@ struct Builder {
         for (int64_t i = j; i < T; ++i) store(i, j);
   }
 
+  // the same tasks in another program order (dev_order 1): seq holds
+  // (kind, i, j, k) in any order in which every tile receives its updates
+  // k = 0, 1, ... and then its TRSM, so the STF rule infers the same DAG
+  template <class Seq>
+  void run_seq(const Seq& seq) {
+    p.buffers.clear();
+    for (int64_t i = 0; i < T; ++i)
+      for (int64_t j = 0; j <= i; ++j) p.buffers.push_back(Buffer{(int32_t)i, (int32_t)j, p.owner(i, j), false});
+    auto key = [&](int64_t i, int64_t j) { return i * T + j; };
+    const bool prio = p.opt.priority;
+    auto level = [&](int64_t d) -> int { return d <= 1 ? 4 : d == 2 ? 3 : d <= 4 ? 2 : d <= 8 ? 1 : 0; };
+    auto P = [&](int lv) { return prio ? lv : 0; };
+    for (const auto& c : seq) {
+      const int64_t i = c.i, j = c.j, k = c.k;
+      if (c.kind == K_POTRF) compute(K_POTRF, k, k, k, P(5), -1, -1, k, k);
+      else if (c.kind == K_TRSM) compute(K_TRSM, i, k, k, P(i == k + 1 ? 5 : 4), key(k, k), -1, i, k);
+      else if (c.kind == K_SYRK) compute(K_SYRK, i, i, k, P(i == k + 1 ? 5 : level(i - k)), key(i, k), -1, i, i);
+      else compute(K_GEMM, i, j, k, P(level(j - k)), key(i, k), key(j, k), i, j);
+    }
+  }
+
   // write-back of the final tile (i, j); on the other copy stream than the slot's
   // loads, so a write-back starts as soon as its tile is final instead of queueing
   // behind every load
@@ -661,7 +682,13 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
     // dense datum ids: home tiles + at most one replica per (tile, slot)
     plan.graph = TaskGraph(NT + NT * opt.nslots + 1);
     Builder b(plan, T);
-    b.run();
+    if (opt.dev_order == 1 && !opt.with_load && !opt.with_store && opt.lookahead) {
+      OocBuilder ob(plan, T, NT);  // 2D-blocked left-looking order, block budget from all tiles
+      ob.make_sequence_2d();
+      b.run_seq(ob.seq);
+    } else {
+      b.run();
+    }
     if (opt.order_mode == 2)
       reorder_list(plan, b.accs, NT + NT * opt.nslots + 1, opt.sched_width > 0 ? opt.sched_width : 2, opt.order_tail);
     else if (opt.order_asap) reorder_asap(plan, b.accs, NT + NT * opt.nslots + 1);

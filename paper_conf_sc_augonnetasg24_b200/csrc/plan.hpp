@@ -68,6 +68,7 @@ struct PlanOptions {
                            // plan (NEXT-4) over this many device tile frames; see plan.cpp
   bool ooc_reorder = true;  // order_mode 2 also re-orders out-of-core plans (loads by simulated start)
   int ooc_budget_pct = 60;  // 2D order: % of the frames a block (triangle + row chunk) may fill
+  int dev_order = 0;        // device-resident plans: 0 right-looking program order, 1 2D-blocked left-looking
   int ooc_order = -1;      // out-of-core program order: 0 tall super-columns, 1 2D-blocked,
                            // -1 auto: 2D-blocked if re-ordered, else while fewer than half
                            // the tiles fit (plan.cpp)

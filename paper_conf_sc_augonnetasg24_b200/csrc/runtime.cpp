@@ -233,6 +233,7 @@ stf::PlanOptions plan_options(const Options& o, int P, int Q, int nslots, bool l
   po.sched_width = (int)std::max<int64_t>(0, env_int("STF_SCHED_WIDTH", 0));  // 0: from nb (prepare)
   po.lookahead = o.lookahead != 0;
   po.ooc_reorder = env_int("STF_OOC_REORDER", 1) != 0;
+  po.dev_order = (int)env_int("STF_DEV_ORDER", 0);
   po.ooc_budget_pct = (int)std::min<int64_t>(95, std::max<int64_t>(10, env_int("STF_OOC_BUDGET_PCT", 60)));
   po.push = o.push != 0 && o.trsm >= 2;
   return po;

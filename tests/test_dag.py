@@ -132,7 +132,8 @@ def test_fused_push_replaces_panel_copies(T, p, q, known):
 
 
 @pytest.mark.parametrize("T,p,q", [(6, 1, 1), (8, 2, 2), (8, 2, 4), (5, 1, 2), (16, 1, 1)])
-@pytest.mark.parametrize("order", [("STF_ORDER_ASAP", "1"), ("STF_ORDER_MODE", "2")], ids=["asap", "list"])
+@pytest.mark.parametrize("order", [("STF_ORDER_ASAP", "1"), ("STF_ORDER_MODE", "2"), ("STF_DEV_ORDER", "1")],
+                         ids=["asap", "list", "left_looking"])
 def test_submission_orders_same_dag(T, p, q, order, monkeypatch):
     """The re-submission orders (plan.cpp reorder_asap / reorder_list, the latter
     the default for nb >= 512) are topological orders of the program-order DAG,
