@@ -135,7 +135,7 @@ const char *stf_last_error(void);
  *                           512), else 1 while the cap is below half the tiles, else 0.  Every
  *                           order gives bit-identical L.
  *   "host_stream" STF_HOST_STREAM  1 (default): an uncapped HOST_COLMAJOR call on one GPU with
- *                           nb >= 512 is planned by the out-of-core builder with one frame per
+ *                           nb >= 512 and n/nb >= 16 is planned by the out-of-core builder with one frame per
  *                           tile (2D-blocked left-looking order, no eviction); 0: the
  *                           right-looking plan with its LOAD/STORE tasks.  Same bits.
  * Returns 0 or -105. */

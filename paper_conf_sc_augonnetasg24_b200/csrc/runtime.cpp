@@ -635,11 +635,15 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
       X.opt.mem_cap_tiles < T * (T + 1) / 2)
     po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames
   else if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && po.order_mode == 2 && po.ooc_reorder &&
-           X.opt.host_stream)
+           X.opt.host_stream && T >= 16) {  // T = 8 (n = 8192, nb = 1024): -1.5%, T = 16 +0.2%, T = 32 +2.7..5%
     // in-core host call through the out-of-core builder with a frame per tile: its
     // 2D-blocked left-looking order consumes the tiles in the order they arrive
-    // over PCIe (n = 32768, nb = 1024: 357.6 -> 352.7 ms end to end); no eviction
+    // over PCIe; nothing is evicted, so a block may fill most of the frames
+    // (n = 32768, nb = 1024: right-looking plan 357.6 ms, block budget 60% 352.7 ms,
+    // 75..99% 345.8 ms; one block of all tiles would be the right-looking order)
     po.frames = T * (T + 1) / 2;
+    po.ooc_budget_pct = (int)std::min<int64_t>(99, std::max<int64_t>(10, env_int("STF_HOST_STREAM_BUDGET_PCT", 90)));
+  }
   po.ooc_order = (int)X.opt.ooc_order;
   stf::build_plan(X.plan, T, po);
   const stf::Plan& P = X.plan;
