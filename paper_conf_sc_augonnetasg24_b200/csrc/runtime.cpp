@@ -632,8 +632,13 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   if (env_int("STF_ORDER_TAIL", -1) < 0) po.order_tail = (!colmajor && T > 16) ? 8 : 0;
 
   if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && X.opt.mem_cap_tiles > 0 &&
-      X.opt.mem_cap_tiles < T * (T + 1) / 2)
+      X.opt.mem_cap_tiles < T * (T + 1) / 2) {
     po.frames = X.opt.mem_cap_tiles;  // NEXT-4: out-of-core plan over this many device frames
+    // with three quarters of the tiles resident or more, wide blocks (90%) keep the
+    // right-looking concurrency; below, eviction pressure favours 60% (n = 32768,
+    // nb = 1024: F = 450 / 396 +2.1% / +2.0% at 90%, F = 264 -6%)
+    if (env_int("STF_OOC_BUDGET_PCT", -1) < 0 && 4 * po.frames >= 3 * (T * (T + 1) / 2)) po.ooc_budget_pct = 90;
+  }
   else if (X.kind == STF_DESC_HOST_COLMAJOR && X.ngpus == 1 && po.order_mode == 2 && po.ooc_reorder &&
            X.opt.host_stream && T >= 16) {  // T = 8 (n = 8192, nb = 1024): -1.5%, T = 16 +0.2%, T = 32 +2.7..5%
     // in-core host call through the out-of-core builder with a frame per tile: its
