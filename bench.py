@@ -15,8 +15,12 @@ ranks contribute 0 device time to the max-over-ranks.
 One step = one synchronous stf_potrf of the whole matrix (every §8(a) row: DAG,
 placement, replica pushes, POTRF/TRSM/SYRK/GEMM kernels, completion) on
 device-resident 2D-block-cyclic tiles (TILED_2DBC).  The
-matrix is regenerated on the device before every step (untimed); it is 4.4 GB
-of tiles at the default n = 32768, far larger than the 126 MB L2.
+workload is north_star's target matrix, n = 65536, nb = 1024 (BASELINE
+configs[3]; 17.4 GB of lower tiles, fits one B200), at every N.  The matrix is
+regenerated on the device before every step (untimed); it is far larger than
+the 126 MB L2.  After the timed steps one more call factors the P2 matrix
+A = L0 L0^T on the same plan and every tile is compared with L0
+bit for bit on the box (`check`).
 `value` = n^3/3 * steps / sum(device time), device time measured with CUDA
 events on the library's launch stream around the graph launch.
 
@@ -137,6 +141,49 @@ def max_over_ranks(x: float, dist_on: bool) -> float:
     return float(t.item())
 
 
+def workload_name(n, nb):
+    cfg = {(65536, 1024): "configs[3]", (32768, 1024): "configs[2]", (131072, 2048): "configs[4]",
+           (8192, 512): "configs[1]", (1024, 256): "configs[0]"}.get((n, nb), "custom")
+    return "n=%d nb=%d FP64 SPD (seeded, diagonally dominant), %s" % (n, nb, cfg)
+
+
+def p2_check(tiles, n, nb, owned=None):
+    """Load the P2 dyadic matrix A = L0 L0^T (harness-side torch
+    fp64 matmuls build it exactly in any order) into the tiles this process holds.
+    `tiles` maps (i, j) -> the row-major (nb, nb) tensor holding tile (i, j)
+    transposed.  Returns L0 per device for p2_compare after the factorisation."""
+    import torch
+    from synth.spd import dyadic_unit_lower_block_torch
+
+    by_dev = {}
+    for ij, t in tiles.items():
+        by_dev.setdefault(t.device, []).append(ij)
+    L0s = {}
+    for dev in by_dev:
+        L0 = torch.empty((n, n), dtype=torch.float64, device=dev)
+        for r in range(0, n, 4096):
+            L0[r:r + 4096] = dyadic_unit_lower_block_torch(101, n, r, 0, min(4096, n - r), n, device=dev)
+        L0s[dev] = L0
+        for (i, j) in by_dev[dev]:
+            K = (j + 1) * nb
+            tiles[(i, j)].copy_((L0[i * nb:(i + 1) * nb, :K] @ L0[j * nb:(j + 1) * nb, :K].T).T)
+        torch.cuda.synchronize(dev)
+    return L0s
+
+
+def p2_compare(tiles, L0s, nb):
+    import torch
+
+    bad = 0
+    for (i, j), t in tiles.items():
+        got = t.T
+        ref = L0s[t.device][i * nb:(i + 1) * nb, j * nb:(j + 1) * nb]
+        if i == j:
+            got, ref = torch.tril(got), torch.tril(ref)
+        bad += not torch.equal(got, ref)
+    return len(tiles), bad
+
+
 def reference_arm(args, rank, world):
     if rank != 0:
         return 0
@@ -163,7 +210,7 @@ def reference_arm(args, rank, world):
         "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1000 * tot / len(ts), 3),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": "n=%d nb=%d FP64 SPD (seeded, diagonally dominant), configs[2]" % (n, nb),
+        "config": {"workload": workload_name(n, nb),
                    "n": n, "nb": nb, "grid": "%dx%d" % grid_for(args.gpus), "sample_n": m, "l2": "n/a (CPU)"},
         "cpu_baseline": {"value": round(value, 4), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
         "e2e": {"value": round(value, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -227,6 +274,15 @@ def run_ours(args, rank, world):
             torch.cuda.synchronize(d)
         clk = clocks.stop()
         total_ms = sum(steps_ms)
+        check = None
+        if not args.no_check:
+            L0s = p2_check(M.tiles, n, nb)
+            info = M.potrf()
+            ntile, bad = p2_compare(M.tiles, L0s, nb)
+            del L0s
+            check = {"input": "P2 dyadic A = L0 L0^T (m=25, seed 101), same plan, after the timed steps",
+                     "info": info, "tiles_checked": ntile, "tiles_mismatched": bad, "bit_exact": bad == 0 and info == 0}
+            torch.cuda.empty_cache()
     if dist_on:
         total_ms = max_over_ranks(total_ms, True)
         dist.barrier()
@@ -235,7 +291,10 @@ def run_ours(args, rank, world):
             dist.destroy_process_group()
         return 0
 
-    report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "single", args.steps * stats["kernel_launches"])
+    del M
+    torch.cuda.empty_cache()
+    report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "single", args.steps * stats["kernel_launches"],
+           check)
     stf.finalize()
     if dist_on:
         dist.destroy_process_group()
@@ -279,6 +338,21 @@ def run_mp(args, rank, world, P, Q):
     mine = [step() for _ in range(args.steps)]
     clk = clocks.stop() if rank == 0 else None
     stats = stf.last_stats()
+    check = None
+    if not args.no_check:
+        L0s = p2_check(A.tiles, n, nb)
+        dist.barrier()
+        info = A.potrf()
+        dist.barrier()
+        ntile, bad = p2_compare(A.tiles, L0s, nb)
+        del L0s
+        torch.cuda.empty_cache()
+        got = [None] * world
+        dist.all_gather_object(got, (info, ntile, bad))
+        bad_all = sum(g[2] for g in got)
+        check = {"input": "P2 dyadic A = L0 L0^T (m=25, seed 101), same plan, after the timed steps",
+                 "info": max(g[0] for g in got), "tiles_checked": sum(g[1] for g in got), "tiles_mismatched": bad_all,
+                 "bit_exact": bad_all == 0 and all(g[0] == 0 for g in got)}
     steps_ms = [max_over_ranks(x, True) for x in mine]  # per step: the slowest rank
     total_ms = sum(steps_ms)
     launches = torch.tensor([float(stats["kernel_launches"])], dtype=torch.float64,
@@ -293,14 +367,17 @@ def run_mp(args, rank, world, P, Q):
         devices = list(range(N)) if args.virtual == 0 else [0] * N
         stf.init(N, devices)
         stats = dict(stats, graph_nodes=sum(nodes), kernel_launches=int(launches.item()))
-        report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "mp", args.steps * int(launches.item()))
+        del A
+        torch.cuda.empty_cache()
+        report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "mp", args.steps * int(launches.item()),
+               check)
         stf.finalize()
     dist.barrier()
     dist.destroy_process_group()
     return 0
 
 
-def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, gpu_launches):
+def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, gpu_launches, check=None):
     import torch
 
     n, nb = args.n, args.nb
@@ -366,11 +443,12 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
         "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": N, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": "n=%d nb=%d FP64 SPD (seeded, diagonally dominant), configs[2]" % (n, nb),
+        "config": {"workload": workload_name(n, nb),
                    "n": n, "nb": nb, "grid": "%dx%d" % (P, Q), "descriptor": "TILED_2DBC (device-resident tiles)",
                    "l2": "inputs larger than L2 (%.1f GB of tiles) and regenerated before every step" %
                          (n // nb * (n // nb + 1) / 2 * nb * nb * 8 / 1e9),
-                   "graph": stf.get_option("graph"), "streams": stf.get_option("streams"),
+                   "graph": bool(stats["graph"]), "graph_fallback": bool(stats["graph_fallback"]),
+                   "streams": stf.get_option("streams"),
                    "virtual_slots": bool(args.virtual),
                    "processes": ("one per GPU (stf_mp_*, CUDA-IPC replicas, device-side flags)" if mode == "mp"
                                  else "one process drives all %d GPU(s) (stf_potrf)" % N)},
@@ -379,7 +457,10 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
         "roofline": roof,
         "cpu_baseline": cpu,
         "e2e": e2e,
-        "plan": {k: stats[k] for k in ("tasks", "transfers", "edges", "critical_path", "graph_nodes", "kernel_launches")},
+        "plan": {k: stats[k] for k in ("tasks", "dag_tasks", "edges", "critical_path", "graph_nodes", "kernel_launches",
+                                       "transfers", "transfer_bytes", "pushed", "replicas_max", "data_plane",
+                                       "devices", "slots", "peer_transfers", "build_ms")},
+        "check": check,
         "first_call_ms": round(first_ms, 1) if first_ms else None,
         "step_ms": [round(x, 3) for x in steps_ms],
     }
@@ -453,7 +534,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", "--order", dest="n", type=int, default=32768)
+    ap.add_argument("--n", "--order", dest="n", type=int, default=65536)
     ap.add_argument("--nb", "--tile", dest="nb", type=int, default=1024)
     ap.add_argument("--virtual-slots", dest="virtual", type=int, default=0, help="map all slots onto cuda:0")
     ap.add_argument("--mode", default=None, choices=["single", "mp"],
@@ -461,6 +542,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-check", action="store_true", help="skip the post-timing P2 bit-exactness check")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--ref-cap", type=int, default=0, help="cap on the reference sample order (0 = none)")
     ap.add_argument("--ref-seconds", type=float, default=0.0, help="oracle seconds per reference step (0 = auto)")

@@ -30,7 +30,12 @@
  * valid until the next library call on that thread.
  *
  * Threading: calls are serialised by an internal mutex; stf_potrf is not
- * re-entrant.  Ownership: the caller owns A (and every tile) in all modes and
+ * re-entrant.  Stream ordering: a factorisation starts after all work the caller
+ * enqueued before the call on the legacy default stream and on the calling
+ * thread's per-thread default stream of every participating device (the library
+ * records events there and its launch stream waits on them); work on other caller
+ * streams must be synchronised by the caller.  It returns after all of its own
+ * device work has completed.  Ownership: the caller owns A (and every tile) in all modes and
  * must not touch it during a call; the library owns its streams, events,
  * graphs, replicas and workspaces from stf_cholesky_init to stf_finalize.
  */
@@ -94,50 +99,70 @@ int stf_finalize(void);
 const char *stf_last_error(void);
 
 /* ---------------------------------------------------------------- options
- * Execution options (defaults from the environment at init):
+ * Execution options.  Each is read once from the environment at init (the
+ * variable in the second column) and settable here; every option except
+ * "threads" and "grid_p" is part of the memo key of a plan, so a plan or graph
+ * built under one value is never reused under another.  Out-of-range values
+ * (from either source) are rejected with -105.
  *   "dataflow" STF_DATAFLOW POTRF tile kernel: 1 single-launch dataflow (default), 0 recursive
  *   "trsm"     STF_TRSM     TRSM tile kernel: 3 (default) = resident panel for the critical
  *                           TRSM(k+1,k) when nb <= 1024 and nb % 64 == 0, row panel otherwise;
  *                           2 row panel, 1 dataflow, 0 recursive
  *   "trsm_split" STF_TRSM_SPLIT P in [1,16]: non-critical row-panel TRSMs run right-looking
- *                           over P column blocks (panel kernel + GEMM updates; default 4);
- *                           1: one panel launch
+ *                           over P column blocks (panel kernel + GEMM updates; default 4)
  *   "trsm_res_tail" STF_TRSM_RES_TAIL C >= 0: with trsm 3, every TRSM(i,k) of a panel step
- *                           whose trailing order n - k nb <= C uses the resident panel (there
- *                           the factorisation is latency-bound; default 8192)
- *   "trsm_rows" STF_TRSM_ROWS 32, 64 or 128 (default): rows per CTA of the non-critical
- *                           row-panel TRSM launches (128: two substitution chains per SM
- *                           sub-partition, full 64-column blocks only, else 64; same bits)
- *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA
- *                           graph, memoised per (n, nb, grid, tiles) (default);
- *                           0: eager lowering on streams + events
- *   "streams"  STF_STREAMS  bulk compute streams per GPU slot (default 32; the pool is sized at init)
- *   "serial"   STF_SERIAL   1: every task on one stream in program order (race check)
+ *                           whose trailing order n - k nb <= C uses the resident panel (default 8192)
+ *   "trsm_rows" STF_TRSM_ROWS 32, 64 or 128 (default): rows per CTA of the row-panel TRSM
+ *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA graph,
+ *                           memoised per (n, nb, grid, tiles, options) (default); 0: eager
+ *                           lowering on streams + events.  A capture the driver rejects falls
+ *                           back to eager (stf_plan_stats.graph_fallback = 1)
+ *   "streams"  STF_STREAMS  bulk compute streams per GPU slot (default 32; pool sized at init)
+ *   "stream_pool" STF_STREAM_POOL 0 (default): 6 high-priority + "streams" bulk + 2 copy streams
+ *                           per slot; 1: one compute stream + one copy stream per slot; 2: one
+ *                           stream per slot for everything (ablations of PAPER.md:401, :407)
+ *   "serial"   STF_SERIAL   1: every compute task on one stream in program order (race check)
  *   "priority" STF_PRIO     1: critical-path tasks on high-priority streams (default 1)
+ *   "prio_mode" STF_PRIO_MODE  priority level assignment variant (0 default; 1..3 ablations)
  *   "grid_p"   STF_GRID     rows P of the P x Q grid for COLMAJOR kinds (0 = auto)
  *   "push"     STF_PUSH     1: TRSM(i,k) writes L_ik into its consumers' replicas from its own
  *                           epilogue (fused push over NVLink, NEXT-3); 0: COPY tasks (default)
  *   "threads"  STF_THREADS  eager backend: host submission threads, slots split round-robin
  *                           (default 8, capped at ngpus; the graph backend captures on one thread)
  *   "lookahead" STF_LOOKAHEAD 1: pure STF DAG (default); 0: a fence task closes every
- *                           panel step (no look-ahead; ablation of PAPER.md:399)
+ *                           panel step (no look-ahead; ablation of PAPER.md:399).  Rejected
+ *                           (-105) for out-of-core plans and in multi-process mode
+ *   "order_mode" STF_ORDER_MODE submission order: -1 auto (default: list scheduling for
+ *                           nb >= 512, else program order), 0 program order, 2 list scheduling
+ *   "order_tail" STF_ORDER_TAIL with list scheduling, re-order only the last C panel steps
+ *                           (-1 auto: 8 for device tiles with T > 16, else all; 0 all)
+ *   "order_asap" STF_ORDER_ASAP 1: earliest-start submission order (with order_mode 0)
+ *   "sched_width" STF_SCHED_WIDTH list-scheduling model width (0 auto from nb and the SM count)
+ *   "dev_order" STF_DEV_ORDER 1: device-resident plans in the 2D-blocked left-looking order
  *   "mem_cap_tiles" STF_MEM_CAP_TILES  0 (default) or >= 3: a HOST_COLMAJOR call on one GPU
  *                           keeps at most this many nb x nb tiles on the device (out-of-core,
  *                           NEXT-4): tiles are loaded on demand and dirty
- *                           tiles written back on eviction (Belady order, left-looking
- *                           super-columns).  A cap >= T(T+1)/2 tiles means no cap.  Rejected
- *                           (-105) for HOST_COLMAJOR calls on more than one GPU; ignored for
- *                           device-resident kinds, whose matrix is on the device already.
- *   "ooc_order" STF_OOC_ORDER  program order of an out-of-core plan: 1 2D-blocked (column
- *                           blocks swept in row chunks: fewer panel re-reads when a trailing
- *                           column alone fills the frames); 0 tall super-columns; -1 (default)
- *                           1 when the plan is re-submitted in list-scheduling order (nb >=
- *                           512), else 1 while the cap is below half the tiles, else 0.  Every
- *                           order gives bit-identical L.
+ *                           tiles written back on eviction (Belady order).  A cap >= T(T+1)/2
+ *                           tiles means no cap.  Rejected (-105) for HOST_COLMAJOR calls on
+ *                           more than one GPU; ignored for device-resident kinds
+ *   "ooc_order" STF_OOC_ORDER  program order of an out-of-core plan: 1 2D-blocked, 0 tall
+ *                           super-columns, -1 (default) auto.  Every order gives bit-identical L
+ *   "ooc_reorder" STF_OOC_REORDER 1 (default): out-of-core plans re-submitted in list order
+ *   "ooc_budget_pct" STF_OOC_BUDGET_PCT block budget of the 2D order in % of the frames
+ *                           (-1 auto: 90 once 3/4 of the tiles fit, else 60)
  *   "host_stream" STF_HOST_STREAM  1 (default): an uncapped HOST_COLMAJOR call on one GPU with
- *                           nb >= 512 and n/nb >= 16 is planned by the out-of-core builder with one frame per
+ *                           nb >= 512 and n/nb >= 16 (list order, lookahead, default stream
+ *                           pool) is planned by the out-of-core builder with one frame per
  *                           tile (2D-blocked left-looking order, no eviction); 0: the
- *                           right-looking plan with its LOAD/STORE tasks.  Same bits.
+ *                           right-looking plan with its LOAD/STORE tasks.  Same bits
+ *   "host_stream_budget_pct" STF_HOST_STREAM_BUDGET_PCT block budget of that plan (default 90)
+ *   "host_eager" STF_HOST_EAGER 1: HOST_COLMAJOR calls on pinned memory lowered eagerly
+ *   "pdl"      STF_PDL      1: programmatic dependent launch between same-stream chain kernels
+ *   "debug_skip" STF_DEBUG_SKIP bit mask (or names potrf,trsm,syrk,gemm,copy,trsm_as_gemm,
+ *                           trsm_as_half_gemm) of task kinds NOT launched: timing what-ifs only,
+ *                           results invalid
+ *   "debug_trace" STF_DEBUG_TRACE 1: timing events around every task (one slot), see
+ *                           stf_debug_last_trace in stf_harness.h
  * Returns 0 or -105. */
 int stf_set_option(const char *name, int64_t value);
 int stf_get_option(const char *name, int64_t *value);
@@ -163,6 +188,14 @@ typedef struct stf_plan_stats {
   int64_t host_loads;     /* LOAD tasks: tiles copied from the caller's matrix (COLMAJOR kinds) */
   int64_t host_stores;    /* STORE tasks: tiles written back to the caller's matrix */
   int64_t frames;         /* device tile frames of an out-of-core plan ("mem_cap_tiles"), else 0 */
+  int64_t pushed;         /* replicas written by fused epilogue pushes (part of transfers) */
+  int64_t replicas_max;   /* largest number of replica tiles held by one slot */
+  int64_t data_plane;     /* 0 COPY tasks (copy engine), 1 fused epilogue push */
+  int64_t graph_fallback; /* 1: the graph capture was rejected and the eager backend ran */
+  int64_t graph;          /* 1: the call ran as one CUDA graph launch, 0: eager streams */
+  int64_t devices;        /* distinct CUDA devices spanned by the call's slots */
+  int64_t slots;          /* GPU slots of the call (ngpus) */
+  int64_t peer_transfers; /* transfers whose source and destination are distinct devices */
 } stf_plan_stats;
 
 int stf_last_stats(stf_plan_stats *out);
@@ -172,13 +205,21 @@ int stf_last_stats(stf_plan_stats *out);
  * order) into edges[2*cap].  kinds[cap_tasks] receives per-task codes
  * (0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM, 4 COPY, 5 LOAD, 6 STORE, 7 FENCE) and ijk[3*cap_tasks]
  * the (i, j, k) indices (for COPY: tile i, j and destination slot k).  Any output pointer
- * may be NULL.  Fills *stats.  Uses the current "push", "lookahead" and "mem_cap_tiles"
- * options (the latter, for p = q = 1: the out-of-core plan of a HOST_COLMAJOR call).
- * Needs no GPU. */
+ * may be NULL.  Fills *stats.  Uses the current options ("order_mode" / "order_tail" auto
+ * mean program order; "mem_cap_tiles" with p = q = 1: the out-of-core plan of a
+ * HOST_COLMAJOR call).  Returns 0, -1, -4 or -105.  Needs no GPU. */
 int stf_dag_build(int64_t T, int p, int q, int64_t cap, int64_t *edges, int64_t cap_tasks, int32_t *kinds,
                   int64_t *ijk, stf_plan_stats *stats);
 
-/* Buffers of the tasks of the last stf_dag_build on this thread: io[3*t] and
+/* The plan stf_potrf(n, nb, 'L', desc of `kind`, ngpus) would execute with the
+ * current options on a p x q grid of GPUs with `sms` SMs each (0: 148), built on
+ * the host only (same code path as the call: submission order, host_stream /
+ * out-of-core builders, stream assignment), exported like stf_dag_build.
+ * Returns 0, -2, -4 or -105.  Needs no GPU. */
+int stf_dag_build_call(int64_t n, int64_t nb, int kind, int ngpus, int p, int q, int sms, int64_t cap, int64_t *edges,
+                       int64_t cap_tasks, int32_t *kinds, int64_t *ijk, stf_plan_stats *stats);
+
+/* Buffers of the tasks of the last stf_dag_build(_call) on this thread: io[3*t] and
  * io[3*t+1] = buffer ids read (-1 unused), io[3*t+2] = buffer written (-1 for
  * STORE/FENCE).  Buffers: home tiles 0..T(T+1)/2-1 (tile (i,j) -> i(i+1)/2 + j)
  * then replicas; in an out-of-core plan the device frames 0..frames-1 (LOAD
@@ -193,60 +234,8 @@ int stf_dag_tasks_io(int64_t cap_tasks, int64_t *io);
 int64_t stf_infer_edges(int64_t ntasks, const int32_t *nacc, const int64_t *data, const int32_t *modes, int64_t cap,
                         int64_t *edges);
 
-/* ---------------------------------------------------------------- harness helpers
- * Fill the seeded SPD metric matrix (SURVEY.md §8(d) generator; same bits as
- * synth/spd.py) into a TILED_2DBC descriptor (lower tiles) on the devices.
- * Synchronous.  Not part of the factorisation. */
-int stf_fill_spd_tiles(int64_t n, int64_t nb, const stf_matrix_desc *A_desc, int ngpus, uint64_t seed);
-
-/* Same generator into an arbitrary column-major device block: rows r0.., cols c0..
- * of the order-n matrix into dst (ld), on the current CUDA device, stream 0. */
-int stf_fill_spd_block(double *dst, int64_t ld, int64_t n, int64_t r0, int64_t c0, int64_t rows, int64_t cols,
-                       uint64_t seed);
-
-/* Direct tile-kernel entry points (device pointers, current device, default
- * stream, synchronous) used by the kernel-level parity tests and the roofline
- * measurement:  C -= A B^T (lower: SYRK);  B <- B L^-T;  A <- chol(A). */
-int stf_kernel_gemm_nt(int64_t M, int64_t N, int64_t K, const double *A, int64_t lda, const double *B, int64_t ldb,
-                       double *C, int64_t ldc, int lower);
-int stf_kernel_trsm(int64_t M, int64_t n, const double *L, int64_t ldl, double *B, int64_t ldb);
-int stf_kernel_potrf(int64_t n, double *A, int64_t lda, int64_t *info);
-
-/* Kernel timing for the roofline: `reps` launches of one tile kernel on a
- * library-owned stream of the current device, each bracketed by CUDA events
- * recorded on that same stream; *avg_ms = mean launch duration.  Inputs are
- * generated on the device (SPD generator) and regenerated (untimed) before
- * each POTRF launch.  kind: 0 GEMM C[MxN] -= A[MxK] B[NxK]^T, 1 SYRK (N = M),
- * 2 TRSM B[MxN] <- B L^-T (K ignored), 3 POTRF of an M x M tile.
- * Returns 0 / -4 / -101 / -103.  Not part of the factorisation. */
-int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double *avg_ms);
-
-/* Debug timeline of the dataflow POTRF tile kernel (one launch on the current
- * device, A: n x n column-major device matrix, ctas <= 0: default grid).
- * trace[0 .. 6T) holds %globaltimer stamps (ns) of the critical-path CTA per
- * 64-block step kb (P start, P published, S inputs ready, S published, U inputs
- * ready, U done), T = ceil(n/64); trace[6T + 3t ..] the claim / inputs-ready /
- * done stamps of bulk ticket t (0 if unused).  Returns the number of entries
- * written (<= cap) or a negative error.  Not part of the factorisation. */
-/* Debug timeline of the last stf_potrf on one GPU slot, recorded when the
- * environment had STF_DEBUG_TRACE=1 at plan build (timing events recorded
- * before and after every task on its stream; no SM work).  Writes up to
- * cap_tasks records of 7 int64 (kind as in stf_dag_build, i, j, k, stream index,
- * ns since the first task's start, at start and at end; -1 if unavailable) in
- * program order; returns the number of tasks of the call (0 if not traced). */
-int64_t stf_debug_last_trace(int64_t *out, int64_t cap_tasks);
-
-int64_t stf_debug_potrf_trace(int64_t n, double *A, int64_t lda, int ctas, int64_t *trace, int64_t cap);
-
-/* Debug timeline of the resident-panel TRSM kernel (B[M x n] <- B L^-T, device
- * pointers, current device; requires 64 <= n <= 1024, n % 64 == 0).  With
- * T = n/64, trace[5 kb + e] holds the %globaltimer stamps (ns) of CTA 0 for
- * column block kb: e = 0 MMA step start, 1 MMA waits for the previous block's
- * solution, 2 it is available, 3 updated block handed to the solver, 4 solver
- * starts; trace[5T + kb] the solver's end.  Returns the number of entries
- * written (<= cap) or a negative error.  Not part of the factorisation. */
-int64_t stf_debug_trsm_trace(int64_t M, int64_t n, const double *L, int64_t ldl, double *B, int64_t ldb,
-                             int64_t *trace, int64_t cap);
+/* Harness entry points (input generation, direct tile kernels, kernel timing,
+ * debug timelines) are declared in stf_harness.h; the same library exports them. */
 
 /* ---------------------------------------------------------------- multi-process mode
  * One process per GPU (e.g. torch.distributed / torchrun): process `rank` owns

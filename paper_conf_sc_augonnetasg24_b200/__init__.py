@@ -68,6 +68,23 @@ def dag(T: int, p: int = 1, q: int = 1):
     return edges, kinds, ijk, st.as_dict()
 
 
+def dag_call(n: int, nb: int, kind: int = STF_DESC_TILED_2DBC, p: int = 1, q: int = 1, sms: int = 148):
+    """(edges, kinds, ijk, stats) of the plan stf_potrf(n, nb, 'L', <kind>, p*q)
+    would execute with the current options (stf_dag_build_call), host only."""
+    st = stf_plan_stats()
+    args = (n, nb, kind, p * q, p, q, sms)
+    check(_abi.stf_dag_build_call(*args, 0, None, 0, None, None, ctypes.byref(st)), "stf_dag_build_call")
+    ntasks = st.dag_tasks
+    E = (ctypes.c_int64 * (2 * max(1, st.edges)))()
+    K = (ctypes.c_int32 * max(1, ntasks))()
+    IJK = (ctypes.c_int64 * (3 * max(1, ntasks)))()
+    check(_abi.stf_dag_build_call(*args, st.edges, E, ntasks, K, IJK, ctypes.byref(st)), "stf_dag_build_call")
+    edges = [(E[2 * e], E[2 * e + 1]) for e in range(st.edges)]
+    kinds = [_abi.KIND_NAMES[K[t]] for t in range(ntasks)]
+    ijk = [(IJK[3 * t], IJK[3 * t + 1], IJK[3 * t + 2]) for t in range(ntasks)]
+    return edges, kinds, ijk, st.as_dict()
+
+
 def dag_io(ntasks: int):
     """(buffers read, buffer written) of every task of the last dag() call, and
     the number of buffers (home tiles + replicas, or device frames out of core)."""

@@ -47,20 +47,31 @@ class stf_plan_stats(ctypes.Structure):
         ("host_loads", ctypes.c_int64),
         ("host_stores", ctypes.c_int64),
         ("frames", ctypes.c_int64),
+        ("pushed", ctypes.c_int64),
+        ("replicas_max", ctypes.c_int64),
+        ("data_plane", ctypes.c_int64),
+        ("graph_fallback", ctypes.c_int64),
+        ("graph", ctypes.c_int64),
+        ("devices", ctypes.c_int64),
+        ("slots", ctypes.c_int64),
+        ("peer_transfers", ctypes.c_int64),
     ]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
 
 
-# Every symbol include/stf_cholesky.h declares (checked by tests/test_abi.py).
+# Every symbol include/stf_cholesky.h declares (checked by tests/test_abi.py) ...
 EXPORTS = [
     "stf_cholesky_init", "stf_potrf", "stf_finalize", "stf_last_error",
-    "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_infer_edges",
-    "stf_fill_spd_tiles", "stf_fill_spd_block",
-    "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace", "stf_debug_last_trace",
-    "stf_debug_trsm_trace",
+    "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_dag_build_call", "stf_infer_edges",
     "stf_dag_tasks_io", "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
+]
+# ... and every symbol include/stf_harness.h declares (test / benchmark entry points).
+HARNESS_EXPORTS = [
+    "stf_fill_spd_tiles", "stf_fill_spd_block",
+    "stf_kernel_gemm_nt", "stf_kernel_trsm", "stf_kernel_potrf", "stf_bench_kernel", "stf_debug_potrf_trace",
+    "stf_debug_last_trace", "stf_debug_trsm_trace",
 ]
 
 if not os.path.exists(LIB_PATH):
@@ -90,6 +101,8 @@ stf_get_option = _decl("stf_get_option", _int, [ctypes.c_char_p, _P(_i64)])
 stf_last_stats = _decl("stf_last_stats", _int, [_P(stf_plan_stats)])
 stf_dag_build = _decl("stf_dag_build", _int, [_i64, _int, _int, _i64, _P(_i64), _i64, _P(_i32), _P(_i64),
                                               _P(stf_plan_stats)])
+stf_dag_build_call = _decl("stf_dag_build_call", _int, [_i64, _i64, _int, _int, _int, _int, _int, _i64, _P(_i64), _i64,
+                                                        _P(_i32), _P(_i64), _P(stf_plan_stats)])
 stf_infer_edges = _decl("stf_infer_edges", _i64, [_i64, _P(_i32), _P(_i64), _P(_i32), _i64, _P(_i64)])
 stf_fill_spd_tiles = _decl("stf_fill_spd_tiles", _int, [_i64, _i64, _P(stf_matrix_desc), _int, ctypes.c_uint64])
 stf_fill_spd_block = _decl("stf_fill_spd_block", _int, [_vp, _i64, _i64, _i64, _i64, _i64, _i64, ctypes.c_uint64])

@@ -29,7 +29,10 @@ SOURCES = [
     "kernels/trsm_panel.cu",
     "kernels/trsm_res.cu",
     "plan.cpp",
-    "runtime.cpp",
+    "api.cpp",
+    "exec.cpp",
+    "mp.cpp",
+    "harness.cpp",
 ]
 
 
@@ -42,7 +45,8 @@ def _deps_mtime() -> float:
     for dp, _, fs in os.walk(CSRC):
         for f in fs:
             m = max(m, os.path.getmtime(os.path.join(dp, f)))
-    m = max(m, os.path.getmtime(os.path.join(ROOT, "include", "stf_cholesky.h")))
+    for h in ("stf_cholesky.h", "stf_harness.h"):
+        m = max(m, os.path.getmtime(os.path.join(ROOT, "include", h)))
     return m
 
 

@@ -843,7 +843,9 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   const int T = p.Nb;
   const int par = T * (T - 1) / 2 > 0 ? T * (T - 1) / 2 : 1;  // widest update wave
   int ctas = std::min(par, std::min(ctas_override > 0 ? ctas_override : df_max_ctas(T), num_sms()));
-  if (p.crit) ctas = std::min(p.ntasks, ctas - 1) + 1;  // + the critical-chain CTA
+  // + the critical-chain CTA; at least one bulk CTA when there are bulk tasks (the
+  // chain waits on updates only bulk CTAs claim)
+  if (p.crit) ctas = std::min(p.ntasks, std::max(ctas, 2) - 1) + 1;
   p.trace = trace;
   return launch_df(stream, prio, p, ctas);
 }

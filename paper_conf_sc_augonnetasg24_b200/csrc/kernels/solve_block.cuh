@@ -50,6 +50,7 @@ __device__ __forceinline__ void solve_block(double* Xs, int c0, DA D, const doub
     double b[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) b[i] = Xs[xo(r, cb + i)];
+    __syncwarp();  // lanes 16..31 read rows 0..15 too: all reads before lanes 0..15 store
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const int c = 8 * P + i;

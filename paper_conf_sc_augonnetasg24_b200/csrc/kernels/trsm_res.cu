@@ -9,19 +9,22 @@
 // column block is never re-read through L2.  Left-looking over 64-wide column
 // blocks jb, with two warp roles running concurrently:
 //
-//   MMA warps (8):    acc = - sum_{pb<jb} X[:,pb] L[jb,pb]^T on the DMMA pipe,
-//                     A operand from the resident panel, L blocks streamed by
-//                     cp.async through a 3-slot ring; the terms pb < jb-1 do not
-//                     depend on the block being solved and run while it is
-//                     solved; X[:,jb] = (B[:,jb] + acc_even) + acc_odd -> panel.
-//   solver warps (2): X[:,jb] <- X[:,jb] L[jb,jb]^-T by substitution (4 lanes per
-//                     row, 16 columns each, the pivot quotient shuffled inside the
-//                     row's lane quad), then to global memory (+ fused-push mirrors).
+//   MMA warps (6, SM sub-partitions 0-2):  acc = - sum_{pb<jb} X[:,pb] L[jb,pb]^T
+//                     on the DMMA pipe, A operand from the resident panel, L
+//                     blocks streamed by TMA (128B-swizzled boxes) through a
+//                     4-slot mbarrier ring (tr::NST); k-groups split mod 3 and
+//                     combined in a fixed order; the terms pb < jb-1 do not depend
+//                     on the block being solved and run while it is solved.
+//   producer warp (1, sub-partition 3): issues the TMA loads of the ring.
+//   solver warp (1, sub-partition 3): X[:,jb] <- X[:,jb] L[jb,jb]^-T by
+//                     substitution in 8-column sub-blocks (register chain with
+//                     correctly rounded division, sub-block updates on DMMA),
+//                     then to global memory (+ fused-push mirrors).
 //
 // Hand-off by named barriers: READY (MMA arrive -> solver sync) when X[:,jb]
 // holds its updated right-hand side, SOLVED (solver arrive -> MMA sync) when it
-// holds the solution.  Every sum has a fixed order (k-steps split by parity
-// between two warp groups, combined in a fixed order), so results are
+// holds the solution.  Every sum has a fixed order (k-steps split mod 3
+// between the MMA k-groups, combined in a fixed order), so results are
 // bit-identical run to run; the quotient is the correctly rounded a / L_cc
 // (div_by: one IEEE reciprocal per column + Markstein correction), so
 // unit-diagonal dyadic inputs stay exact (pin P2).

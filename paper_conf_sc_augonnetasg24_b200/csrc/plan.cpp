@@ -12,6 +12,8 @@
 namespace stf {
 
 int streams_per_slot(const PlanOptions& opt) {
+  if (opt.stream_pool == 2) return 1;
+  if (opt.stream_pool == 1) return 2;
   if (opt.serial) return 1 + opt.copy_streams;
   return opt.crit_streams + opt.bulk_streams + opt.copy_streams;
 }
@@ -49,12 +51,13 @@ struct Builder {
   }
 
   int copy_stream(int dst_slot) const {
+    if (p.opt.stream_pool) return p.opt.stream_pool == 1 ? 1 : 0;
     const int base = p.opt.serial ? 1 : p.opt.crit_streams + p.opt.bulk_streams;
     return base + dst_slot % p.opt.copy_streams;
   }
 
   int compute_stream(const Task& t) const {
-    if (p.opt.serial) return 0;
+    if (p.opt.serial || p.opt.stream_pool) return 0;
     if (p.opt.priority && t.prio >= 4) return crit_stream(t, p.opt.crit_streams);
     return p.opt.crit_streams + (int)((t.i * T + t.j) % p.opt.bulk_streams);
   }
@@ -439,10 +442,12 @@ struct OocBuilder {
           free_frames.pop_back();
         } else {
           // furthest next use among residents the current task does not touch
+          // (F >= 3 guarantees one: a task touches at most 3 tiles; build_plan rejects F < 3)
           auto it = resident.end();
           do {
             --it;
-          } while (it->second == need[0] || it->second == need[1] || it->second == need[2]);
+          } while (it != resident.begin() &&
+                   (it->second == need[0] || it->second == need[1] || it->second == need[2]));
           const int64_t v = it->second;
           resident.erase(it);
           f = frame_of[(size_t)v];
@@ -663,20 +668,23 @@ void build_plan(Plan& plan, int64_t T, const PlanOptions& opt) {
   plan.nstores = 0;
   plan.replicas_per_slot.assign((size_t)opt.nslots, 0);
   const int64_t NT = T * (T + 1) / 2;
-  if (opt.frames > 0 && opt.nslots == 1 && opt.with_load && opt.with_store) {
+  if (opt.frames > 0 && opt.frames < 3) plan.opt.frames = 3;  // a GEMM holds 3 tiles (callers validate F >= 3)
+  if (plan.opt.frames > 0 && opt.nslots == 1 && opt.with_load && opt.with_store) {
     // out-of-core: datum ids = frames, then the caller's host tiles
-    plan.graph = TaskGraph(opt.frames + NT + 1);
-    const int base = plan.opt.serial ? 1 : plan.opt.crit_streams + plan.opt.bulk_streams;
-    OocBuilder b(plan, T, opt.frames);
-    b.run(plan.opt.crit_streams, plan.opt.bulk_streams, base, base + (plan.opt.copy_streams > 1 ? 1 : 0),
-          plan.opt.serial, plan.opt.priority,
+    plan.graph = TaskGraph(plan.opt.frames + NT + 1);
+    const int base = plan.opt.stream_pool ? (plan.opt.stream_pool == 1 ? 1 : 0)
+                     : plan.opt.serial ? 1 : plan.opt.crit_streams + plan.opt.bulk_streams;
+    const int store = plan.opt.stream_pool ? base : base + (plan.opt.copy_streams > 1 ? 1 : 0);
+    OocBuilder b(plan, T, plan.opt.frames);
+    b.run(plan.opt.crit_streams, plan.opt.bulk_streams, base, store, plan.opt.serial || plan.opt.stream_pool != 0,
+          plan.opt.priority,
           // auto: 2D-blocked for re-ordered plans (n = 32768, nb = 1024: F = 33..396 all
           // ahead of the tall order); in program order only while less than half the
           // tiles fit (F = 33 / 66 / 132 +58% / +42% / +2%, F = 264 -1.6%)
           plan.opt.ooc_order >= 0 ? plan.opt.ooc_order
-                                  : ((opt.order_mode == 2 && opt.ooc_reorder) || 2 * opt.frames < NT ? 1 : 0));
+                                  : ((opt.order_mode == 2 && opt.ooc_reorder) || 2 * plan.opt.frames < NT ? 1 : 0));
     if (opt.order_mode == 2 && opt.ooc_reorder)
-      reorder_list(plan, b.accs, opt.frames + NT + 1, opt.sched_width > 0 ? opt.sched_width : 2, 0);
+      reorder_list(plan, b.accs, plan.opt.frames + NT + 1, opt.sched_width > 0 ? opt.sched_width : 2, 0);
   } else {
     plan.opt.frames = 0;
     // dense datum ids: home tiles + at most one replica per (tile, slot)

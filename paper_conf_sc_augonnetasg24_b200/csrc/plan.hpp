@@ -47,7 +47,8 @@ struct PlanOptions {
   int bulk_streams = 8;
   int crit_streams = 2;
   int copy_streams = 2;
-  bool serial = false;     // all tasks of all slots on stream 0 (program order)
+  bool serial = false;     // all compute tasks of a slot on stream 0 (program order)
+  int stream_pool = 0;     // 1: one compute + one copy stream per slot; 2: one stream per slot (ablations)
   bool priority = true;
   int prio_mode = 0;       // level assignment variant (0 default; see plan.cpp)
   bool with_load = false;  // LOAD tasks first (COLMAJOR descriptors)

@@ -3,7 +3,7 @@
 This module holds NO arithmetic of the method (no factorization, no update,
 no solve): only counter-based random numbers and the closed-form test
 matrices of SURVEY.md §8(c)/(d).  Both the CPU side (this file, numpy) and the
-CUDA library (``csrc/kernels/generate.cu``) implement the same counter-based
+CUDA library (``fill_spd_kernel`` in ``csrc/kernels/panel.cu``) implement the same counter-based
 SplitMix64 spec, and a GPU test asserts the two produce identical bits.
 
 Generator spec ("Generator"):

@@ -96,3 +96,44 @@ def dyadic_spd(seed: int, n: int, m: int = 25):
     L0 = dyadic_unit_lower(seed, n, m)
     A = np.asfortranarray(L0 @ L0.T)
     return A, L0
+
+
+# ---------------------------------------------------------------- torch (device) form
+def _t_splitmix64(x):
+    """splitmix64 on int64 torch tensors (two's complement wraps like uint64;
+    logical right shifts emulated with a mask)."""
+    import torch
+
+    def shr(v, k):
+        return (v >> k) & ((1 << (64 - k)) - 1)
+
+    def c(u):  # uint64 constant as the int64 with the same bits
+        return u - (1 << 64) if u >= (1 << 63) else u
+
+    x = x + c(0x9E3779B97F4A7C15)
+    z = (x ^ shr(x, 30)) * c(0xBF58476D1CE4E5B9)
+    z = (z ^ shr(z, 27)) * c(0x94D049BB133111EB)
+    return z ^ shr(z, 31)
+
+
+def dyadic_unit_lower_block_torch(seed: int, n: int, r0: int, c0: int, rows: int, cols: int, m: int = 25,
+                                  device="cuda"):
+    """Rows r0.., columns c0.. of dyadic_unit_lower(seed, n, m) as a torch float64
+    tensor (row-major (rows, cols)) on `device`; bit-identical to the numpy form
+    (tests/test_synth.py).  For the full-size P2 pins (n up to 65536), generated
+    block by block on the GPU."""
+    import torch
+
+    p = m - max(1, math.ceil(math.log2(max(n, 2))))
+    assert p >= 1, "n too large for this m"
+    i = torch.arange(r0, r0 + rows, dtype=torch.int64, device=device)[:, None]
+    j = torch.arange(c0, c0 + cols, dtype=torch.int64, device=device)[None, :]
+    s = int(splitmix64(np.uint64(seed)))
+    s = s - (1 << 64) if s >= (1 << 63) else s
+    h = _t_splitmix64(((i << 32) | j) ^ s)
+    span = (1 << (p + 1)) - 1
+    k = ((h >> 11) & ((1 << 53) - 1)) % span
+    kf = k.to(torch.float64) - float((1 << p) - 1)
+    L0 = torch.where(i > j, kf * (2.0 ** -m), torch.zeros((), dtype=torch.float64, device=device))
+    L0 = torch.where(i == j, torch.ones((), dtype=torch.float64, device=device), L0)
+    return L0

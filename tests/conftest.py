@@ -28,3 +28,20 @@ def pytest_collection_modifyitems(config, items):
     for it in items:
         if "gpu" in it.keywords:
             it.add_marker(skip)
+
+
+@pytest.fixture
+def options():
+    """set_option(name, value) that restores every touched option afterwards."""
+    import paper_conf_sc_augonnetasg24_b200 as stf
+
+    saved = {}
+
+    def setter(name, value):
+        if name not in saved:
+            saved[name] = stf.get_option(name)
+        stf.set_option(name, value)
+
+    yield setter
+    for k, v in saved.items():
+        stf.set_option(k, v)

@@ -13,10 +13,11 @@ from paper_conf_sc_augonnetasg24_b200 import _abi
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 HEADER = os.path.join(ROOT, "include", "stf_cholesky.h")
+HARNESS = os.path.join(ROOT, "include", "stf_harness.h")
 
 
-def header_functions():
-    src = open(HEADER).read()
+def header_functions(path=HEADER):
+    src = open(path).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
     return sorted(set(re.findall(r"\b(stf_[a-z_0-9]+)\s*\(", src)))
 
@@ -30,9 +31,11 @@ def test_header_declares_the_planned_boundary():
 def test_library_exports_every_declared_symbol():
     out = subprocess.run(["nm", "-D", "--defined-only", _abi.LIB_PATH], capture_output=True, text=True).stdout
     exported = set(re.findall(r"\bT (stf_[a-z_0-9]+)", out))
-    missing = [f for f in header_functions() if f not in exported]
+    missing = [f for f in header_functions() + header_functions(HARNESS) if f not in exported]
     assert not missing, missing
     assert sorted(_abi.EXPORTS) == header_functions()
+    assert sorted(_abi.HARNESS_EXPORTS) == header_functions(HARNESS)
+    assert not set(_abi.EXPORTS) & set(_abi.HARNESS_EXPORTS)
 
 
 def test_library_has_sm100a_code():

@@ -37,7 +37,8 @@ def test_reference_arm_json_line():
     assert d["value"] > 0 and d["steps"] == 2 and d["warmup"] == 1
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
-    assert d["config"]["n"] == 32768 and d["config"]["nb"] == 1024
+    assert d["config"]["n"] == 65536 and d["config"]["nb"] == 1024
+    assert "configs[3]" in d["config"]["workload"]
 
 
 def test_reference_arm_under_torchrun_two_ranks():

@@ -132,15 +132,15 @@ def test_fused_push_replaces_panel_copies(T, p, q, known):
 
 
 @pytest.mark.parametrize("T,p,q", [(6, 1, 1), (8, 2, 2), (8, 2, 4), (5, 1, 2), (16, 1, 1)])
-@pytest.mark.parametrize("order", [("STF_ORDER_ASAP", "1"), ("STF_ORDER_MODE", "2"), ("STF_DEV_ORDER", "1")],
+@pytest.mark.parametrize("order", [("order_asap", 1), ("order_mode", 2), ("dev_order", 1)],
                          ids=["asap", "list", "left_looking"])
-def test_submission_orders_same_dag(T, p, q, order, monkeypatch):
+def test_submission_orders_same_dag(T, p, q, order, options):
     """The re-submission orders (plan.cpp reorder_asap / reorder_list, the latter
     the default for nb >= 512) are topological orders of the program-order DAG,
     and re-applying the STF rule in that order yields the same DAG (edges
     identical up to the task relabelling): only the stream-order chains change."""
     e0, k0, ijk0, st0 = stf.dag(T, p, q)
-    monkeypatch.setenv(*order)
+    options(*order)
     e1, k1, ijk1, st1 = stf.dag(T, p, q)
     keys0 = [(k, *x) for k, x in zip(k0, ijk0)]
     keys1 = [(k, *x) for k, x in zip(k1, ijk1)]
@@ -152,17 +152,17 @@ def test_submission_orders_same_dag(T, p, q, order, monkeypatch):
     assert st1["critical_path"] == st0["critical_path"] and st1["edges"] == st0["edges"]
 
 
-def test_list_order_submits_the_panel_chain_early(monkeypatch):
+def test_list_order_submits_the_panel_chain_early(options):
     """List-scheduling order (default for T <= 16 and COLMAJOR calls): POTRF(k+1)
     is submitted as soon as its chain allows, ahead of bulk updates of step k that
     are not its ancestors (in program order it comes after all of them)."""
     T = 8
-    monkeypatch.setenv("STF_ORDER_MODE", "2")
+    options("order_mode", 2)
     e, k, ijk, st = stf.dag(T, 1, 1)
     pos = {(kd, *x): t for t, (kd, x) in enumerate(zip(k, ijk))}
     for step in range(T - 2):
         assert pos[("POTRF", step + 1, step + 1, step + 1)] < pos[("GEMM", T - 1, T - 2, step)]
-    monkeypatch.setenv("STF_ORDER_MODE", "0")
+    options("order_mode", 0)
     e0, k0, ijk0, _ = stf.dag(T, 1, 1)
     pos0 = {(kd, *x): t for t, (kd, x) in enumerate(zip(k0, ijk0))}
     assert pos0[("POTRF", 1, 1, 1)] > pos0[("GEMM", T - 1, T - 2, 0)]

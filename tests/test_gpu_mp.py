@@ -14,10 +14,10 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _run(n, nb, p, q, push=0, reps=2, port=29611, graph=1):
+def _run(n, nb, p, q, push=0, reps=2, port=29611, graph=1, p2=0):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % (p * q),
            "--master-addr", "127.0.0.1", "--master-port", str(port),
-           os.path.join(ROOT, "tests", "mp_worker.py"), str(n), str(nb), str(p), str(q), str(push), str(reps), str(graph)]
+           os.path.join(ROOT, "tests", "mp_worker.py"), str(n), str(nb), str(p), str(q), str(push), str(reps), str(graph), str(p2)]
     out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
     assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-3000:]
     line = [l for l in out.stdout.splitlines() if l.startswith("MP_RESULT")]
@@ -34,6 +34,14 @@ def test_multiprocess_bit_equal_to_single_process(p, q, push, graph, port):
     if graph:  # the whole local DAG, flag waits/writes included, is one CUDA graph per process
         nodes = eval(line.split("graph_nodes=")[1].split(" ms=")[0])
         assert all(g > 0 for g in nodes), line
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("p,q,push,port", [(2, 2, 0, 29681), (2, 2, 1, 29691), (1, 2, 1, 29701)])
+def test_multiprocess_p2_exact(p, q, push, port):
+    """Against the closed form: every rank's tiles equal L0 bit for bit (P2)."""
+    line = _run(1536, 128, p, q, push=push, port=port, reps=2, p2=1)
+    assert "p2=1" in line
 
 
 @pytest.mark.gpu

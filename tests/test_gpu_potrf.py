@@ -68,7 +68,7 @@ def _reset_options(request):
     if "stf" in request.fixturenames:
         s = request.getfixturevalue("stf")
         _options(s, graph=1, serial=0, priority=1, streams=32, grid_p=0, dataflow=1, trsm=3, threads=8, lookahead=1, trsm_split=4, push=0,
-                 trsm_rows=128)
+                 trsm_rows=128, stream_pool=0, prio_mode=0, order_mode=-1, dev_order=0, order_asap=0, host_eager=0)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
@@ -112,6 +112,9 @@ def test_tiny_tiles_on_virtual_grids_bit_equal(stf, n, nb, p, q):
     got = _bits(stf, n, nb, p, q, seed=6)
     _options(stf, push=0)
     assert np.array_equal(ref, got)
+    for push in (0, 1):  # and against the closed form
+        L, L0, _ = _p2(stf, n, nb, p, q, push=push)
+        assert np.array_equal(L, L0)
 
 
 @pytest.fixture(scope="module")
@@ -198,37 +201,47 @@ def _bits(stf, n, nb, p=1, q=1, seed=3, **opts):
     return out
 
 
-def test_bit_stable_runs_and_schedules(stf):
-    n, nb = 2048, 256
-    ref = _bits(stf, n, nb)
-    assert np.array_equal(ref, _bits(stf, n, nb))
-    assert np.array_equal(ref, _bits(stf, n, nb, serial=1))
-    assert np.array_equal(ref, _bits(stf, n, nb, graph=0))
-    assert np.array_equal(ref, _bits(stf, n, nb, priority=0, streams=3))
+def _p2(stf, n, nb, p=1, q=1, **opts):
+    """Factor the P2 dyadic matrix A = L0 L0^T (exact in any summation order) with
+    the given options; every variant must return L0 bit for bit."""
+    A, L0 = synth.dyadic_spd(101, n)
+    _options(stf, **opts)
+    try:
+        L, info = _factor_dense(stf, A, nb, p, q)
+        st = stf.last_stats()
+    finally:
+        _options(stf, graph=1, serial=0, priority=1, streams=32, threads=8, lookahead=1, push=0, stream_pool=0,
+                 prio_mode=0, order_mode=-1, dev_order=0, order_asap=0)
+    assert info == 0
+    return L, L0, st
 
 
-@pytest.mark.parametrize("p,q", [(1, 2), (2, 1), (2, 2), (2, 4)])
-def test_bit_equal_across_virtual_grids(stf, p, q):
-    n, nb = 2048, 256
-    ref = _bits(stf, n, nb, 1, 1)
-    assert np.array_equal(ref, _bits(stf, n, nb, p, q))
-    assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0, threads=1))
-    assert np.array_equal(ref, _bits(stf, n, nb, p, q, graph=0, threads=p * q))  # one submission thread per slot
-    _options(stf, push=1)  # fused push: TRSM epilogues write the consumers' replicas
-    got = _bits(stf, n, nb, p, q)
-    st = stf.last_stats()
-    _options(stf, push=0)
-    assert np.array_equal(ref, got)
+@pytest.mark.parametrize("variant", [
+    {}, {"serial": 1}, {"graph": 0}, {"priority": 0, "streams": 3}, {"lookahead": 0},
+    {"stream_pool": 1}, {"stream_pool": 2}, {"stream_pool": 1, "lookahead": 0}, {"prio_mode": 2},
+    {"order_mode": 0}, {"order_mode": 2}, {"order_mode": 0, "order_asap": 1}, {"dev_order": 1}],
+    ids=lambda v: ",".join("%s=%s" % kv for kv in v.items()) or "default")
+def test_schedule_variants_p2_exact(stf, variant):
+    """Every schedule / ablation variant (NEXT-1: stream pools, single stream, 1
+    compute + 1 copy stream, per-step fences, priorities, submission orders,
+    eager vs graph) against the closed form: L == L0 exactly."""
+    L, L0, st = _p2(stf, 2048, 256, **variant)
+    assert np.array_equal(L, L0)
+    assert st["graph"] == (0 if variant.get("graph") == 0 else 1) and st["graph_fallback"] == 0
 
 
-def test_no_lookahead_fence_ablation_same_bits(stf):
-    # the per-step fence only adds ordering: same kernels, same per-tile op order
-    n, nb = 2048, 256
-    ref = _bits(stf, n, nb)
-    _options(stf, lookahead=0)
-    got = _bits(stf, n, nb)
-    _options(stf, lookahead=1)
-    assert np.array_equal(ref, got)
+@pytest.mark.parametrize("p,q", [(1, 2), (2, 1), (2, 2), (2, 4), (1, 8)])
+@pytest.mark.parametrize("variant", [{}, {"graph": 0, "threads": 1}, {"graph": 0}, {"push": 1}, {"lookahead": 0}],
+                         ids=["graph", "eager1", "eager_threads", "push", "fence"])
+def test_virtual_grids_p2_exact(stf, p, q, variant):
+    """Distributed plans (2D block-cyclic and the 1D column block-cyclic 1x8 grid
+    of cuSolverMg) with COPY tasks or fused pushes, eager or graph,
+    with or without per-step fences: L == L0 exactly."""
+    L, L0, st = _p2(stf, 2048, 256, p, q, **variant)
+    assert np.array_equal(L, L0)
+    assert st["slots"] == p * q and st["transfers"] > 0
+    assert st["data_plane"] == (1 if variant.get("push") else 0)
+    assert (st["pushed"] > 0) == bool(variant.get("push"))
 
 
 def test_same_shape_new_tiles_rebinds_graph(stf):
@@ -299,7 +312,7 @@ def test_colmajor_descriptors(stf, where, order, ngpus):
 
 
 @pytest.mark.parametrize("ngpus", [1, 2])
-def test_host_colmajor_submission_orders_same_bits(stf, ngpus, monkeypatch):
+def test_host_colmajor_submission_orders_same_bits(stf, ngpus):
     """HOST_COLMAJOR calls with nb >= 512 are re-submitted in list-scheduling
     order; that order, the earliest-start order and the eager lowering
     all keep the DAG, so the same bits as the device-resident tiles."""
@@ -308,18 +321,15 @@ def test_host_colmajor_submission_orders_same_bits(stf, ngpus, monkeypatch):
     n, nb = 4096, 1024
     ref = _bits(stf, n, nb, 1, ngpus, seed=7)
     A = synth.spd_matrix(7, n)
-    for env in ({}, {"STF_ORDER_MODE": "0", "STF_ORDER_ASAP": "1"}, {"STF_HOST_EAGER": "1"}):
-        for k, v in env.items():
-            monkeypatch.setenv(k, v)
-        stf.finalize()  # the environment is read when a plan is built: drop the memoised plans
-        stf.init(NSLOTS, [0] * NSLOTS)
+    for opts in ({}, {"order_mode": 0, "order_asap": 1}, {"host_eager": 1}):
+        _options(stf, **opts)  # options are part of the memo key: each builds its own plan
         t = torch.from_numpy(np.ascontiguousarray(A)).pin_memory().t()  # column-major view
         assert stf.potrf(t, nb, ngpus=ngpus) == 0
         st = stf.last_stats()
-        assert st["host_loads"] == 10 and (st["graph_nodes"] == 0) == ("STF_HOST_EAGER" in env)
-        assert np.array_equal(np.tril(t.numpy()), np.tril(ref)), env
-        for k in env:
-            monkeypatch.delenv(k)
+        _options(stf, order_mode=-1, order_asap=0, host_eager=0)
+        assert st["host_loads"] == 10 and (st["graph_nodes"] == 0) == ("host_eager" in opts)
+        assert st["graph"] == (0 if "host_eager" in opts else 1)
+        assert np.array_equal(np.tril(t.numpy()), np.tril(ref)), opts
 
 
 def test_n_zero(stf):
@@ -361,3 +371,26 @@ def test_bench_config_leading_block_and_residual(stf, n, nb, m):
         assert err <= 10
     del Ld
     assert T == n // nb
+
+
+def test_orders_after_callers_default_stream_work(stf):
+    """Ordering contract (include/stf_cholesky.h): a call starts after the work
+    the caller enqueued before it on the default stream -- here a long matmul
+    followed by the device-to-device copies that fill the tiles, with no host
+    synchronisation in between."""
+    import torch
+
+    n, nb = 1024, 256
+    A, L0 = synth.dyadic_spd(101, n)
+    Ad = torch.from_numpy(np.ascontiguousarray(A)).cuda()
+    M = stf.TiledMatrix(n, nb)
+    for t in M.tiles.values():
+        t.zero_()
+    big = torch.randn((6144, 6144), dtype=torch.float64, device="cuda")
+    torch.cuda.synchronize()
+    for _ in range(3):
+        big = big @ big / 6144.0  # ~40 ms of default-stream work ahead of the tile copies
+    for (i, j), t in M.tiles.items():
+        t.copy_(Ad[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb].T)
+    assert M.potrf() == 0
+    assert np.array_equal(M.to_dense().numpy(), L0)

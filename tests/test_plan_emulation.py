@@ -111,13 +111,15 @@ def test_distributed_plan_any_topological_order(T, p, q, lookahead):
 @pytest.mark.parametrize("ooc_order", [0, 1, -1])
 @pytest.mark.parametrize("T,frames", [(4, 3), (4, 5), (6, 3), (6, 4), (6, 7), (6, 12), (8, 6), (8, 20), (9, 10),
                                       (12, 9), (12, 30)])
-def test_out_of_core_plan_any_topological_order(T, frames, ooc_order, list_order, monkeypatch):
+def test_out_of_core_plan_any_topological_order(T, frames, ooc_order, list_order):
     """list_order: the plan re-submitted in simulated list-scheduling order
-    (STF_ORDER_MODE=2, what the runtime does at nb >= 512)."""
-    if list_order:
-        monkeypatch.setenv("STF_ORDER_MODE", "2")
+    (order_mode 2, what the runtime does at nb >= 512)."""
     A = synth.spd_matrix(11, T * NB)
-    edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames, ooc_order=ooc_order)
+    stf.set_option("order_mode", 2 if list_order else -1)
+    try:
+        edges, kinds, ijk, io, nbuf, st = _plan(T, 1, 1, frames=frames, ooc_order=ooc_order)
+    finally:
+        stf.set_option("order_mode", -1)
     NT = T * (T + 1) // 2
     assert st["frames"] == frames and nbuf == frames
     assert "COPY" not in kinds
@@ -185,3 +187,72 @@ def test_out_of_core_2d_order_cuts_panel_reloads():
         st1 = _plan(T, 1, 1, frames=frames, ooc_order=1)[5]
         assert NT <= st1["host_loads"] <= gain * st0["host_loads"], (frames, st0["host_loads"], st1["host_loads"])
         assert st1["host_stores"] == NT
+
+
+def _call_plan(n, nb, kind, p=1, q=1):
+    edges, kinds, ijk, st = stf.dag_call(n, nb, kind, p, q)
+    io, nbuf = stf.dag_io(len(kinds))
+    return edges, kinds, ijk, io, nbuf, st
+
+
+@pytest.mark.parametrize("n,nb,kind,p,q", [
+    (32768, 1024, stf.STF_DESC_HOST_COLMAJOR, 1, 1),   # bench e2e: host_stream plan, T = 32
+    (16384, 512, stf.STF_DESC_HOST_COLMAJOR, 1, 1),    # host_stream plan, T = 32, nb = 512
+    (16384, 1024, stf.STF_DESC_HOST_COLMAJOR, 1, 1),   # host_stream plan, T = 16 (smallest T it serves)
+    (8192, 1024, stf.STF_DESC_HOST_COLMAJOR, 1, 1),    # T = 8: right-looking plan with LOAD/STORE tasks
+    (32768, 1024, stf.STF_DESC_TILED_2DBC, 1, 1),      # bench: device tiles, list order over the last 8 steps
+    (32768, 1024, stf.STF_DESC_TILED_2DBC, 2, 4),      # the 8-GPU grid of the bench's scaling run
+    (16384, 1024, stf.STF_DESC_HOST_COLMAJOR, 2, 2),   # HOST_COLMAJOR on 4 GPUs
+])
+def test_call_plans_any_topological_order(n, nb, kind, p, q):
+    """The exact plans stf_potrf executes for the configurations bench.py and
+    the e2e measurement report (stf_dag_build_call: same code path as the call,
+    including the host_stream builder and the list-scheduling re-submission),
+    executed with the oracle's tile operations on 4 x 4 tiles in random
+    topological orders: oracle.tiled_potrf's bits in every order."""
+    T = n // nb
+    edges, kinds, ijk, io, nbuf, st = _call_plan(n, nb, kind, p, q)
+    NT = T * (T + 1) // 2
+    assert st["tasks"] == T + T * (T - 1) + T * (T - 1) * (T - 2) // 6
+    host = kind == stf.STF_DESC_HOST_COLMAJOR
+    if host and p * q == 1 and T >= 16:
+        assert st["frames"] == NT  # host_stream: one frame per tile, nothing evicted
+    if host:
+        assert st["host_loads"] == NT and st["host_stores"] == NT
+    A = synth.spd_matrix(13, T * NB)
+    ref = _reference(T, A)
+    for seed in (-1, 1, 2):
+        got = _emulate(T, A, kinds, ijk, io, nbuf, edges, seed, host_resident=host)
+        assert np.array_equal(got, ref), (seed, np.abs(got - ref).max())
+
+
+def test_call_plan_fence_and_stream_pool_ablations():
+    """lookahead=0 (fence per step) and the reduced stream pools keep the
+    right-looking builder for host calls (they implement those variants), and
+    stay exact in any order."""
+    n, nb, T = 16384, 1024, 16
+    A = synth.spd_matrix(14, T * NB)
+    ref = _reference(T, A)
+    for name, val in (("lookahead", 0), ("stream_pool", 1), ("stream_pool", 2)):
+        stf.set_option(name, val)
+        try:
+            edges, kinds, ijk, io, nbuf, st = _call_plan(n, nb, stf.STF_DESC_HOST_COLMAJOR)
+        finally:
+            stf.set_option(name, 1 if name == "lookahead" else 0)
+        assert st["frames"] == 0, name
+        assert ("FENCE" in kinds) == (name == "lookahead")
+        got = _emulate(T, A, kinds, ijk, io, nbuf, edges, 5, host_resident=True)
+        assert np.array_equal(got, ref), name
+
+
+def test_out_of_core_rejects_fence_ablation():
+    stf.set_option("mem_cap_tiles", 10)
+    stf.set_option("lookahead", 0)
+    try:
+        with pytest.raises(stf.StfError):
+            stf.dag(8, 1, 1)
+        with pytest.raises(stf.StfError):
+            stf.dag_call(8192, 1024, stf.STF_DESC_HOST_COLMAJOR)
+    finally:
+        stf.set_option("mem_cap_tiles", 0)
+        stf.set_option("lookahead", 1)
