@@ -242,12 +242,14 @@ struct Lowerer {
         return 0;
       case stf::K_COPY:
         // Push of a finished tile into a consumer slot's replica on the producer's
-        // copy stream (copy engine, no SMs).  Always the peer-copy API: virtual
-        // slots sharing a device take the same call (a same-device peer copy),
-        // so the path the multi-GPU run uses is the one the tests execute.
-        CUDA_TRY(cudaMemcpyPeerAsync(X.buf[(size_t)t.out], C.slots[(size_t)t.k].device, X.buf[(size_t)t.in[0]],
-                                     S.device, tile_bytes, s),
-                 "replica peer copy");
+        // copy stream (copy engine, no SMs).  One call for every slot pair: with
+        // unified addressing and peer access enabled (stf_cholesky_init), a
+        // cudaMemcpyDefault copy between two devices is a peer copy over NVLink,
+        // between virtual slots of one device a device-to-device copy, and in both
+        // cases a memcpy node when captured (cudaMemcpyPeerAsync is not
+        // capturable: the capture falls back to eager).
+        CUDA_TRY(cudaMemcpyAsync(X.buf[(size_t)t.out], X.buf[(size_t)t.in[0]], tile_bytes, cudaMemcpyDefault, s),
+                 "replica copy");
         return 0;
       case stf::K_FENCE:
         return 0;  // ordering only: its waits (and event record) are the whole task

@@ -35,9 +35,9 @@
 
 namespace stfk {
 
-template <int BK_, int STAGES_, int BN_ = 128, int MINB_ = 1>
+template <int BK_, int STAGES_, int BN_ = 128, int MINB_ = 1, int BM_ = 128>
 struct Cfg {
-  static constexpr int BM = 128, BN = BN_, BK = BK_, STAGES = STAGES_, MINB = MINB_;
+  static constexpr int BM = BM_, BN = BN_, BK = BK_, STAGES = STAGES_, MINB = MINB_;
   static constexpr int BOX = 16;                  // doubles per 128-byte swizzle row
   static constexpr int BOX_BYTES = BOX * BK * 8;  // 2 KB at BK = 16
   static constexpr int A_BYTES = BM * BK * 8;     // 16 KB at BK = 16
@@ -48,6 +48,10 @@ struct Cfg {
 using CfgK16 = Cfg<16, 4>;  // 4 x 32 KB stages
 using CfgK32 = Cfg<32, 3>;  // 3 x 64 KB stages
 using CfgN64 = Cfg<32, 2, 64, 2>;  // 128 x 64 CTA tile, 2 x 48 KB stages, 2 CTAs / SM (full GEMMs only)
+// 64 x 64 CTA tile, 4 warps of 32 x 32, 3 x 32 KB stages, 2 CTAs / SM: SYRK tiles of order <= 1024
+// (136 CTAs at nb = 1024, one wave on 148 SMs: the critical SYRK(k+1,k) spreads over the whole GPU
+// instead of 72 CTAs of 128 x 64).  Same per-element k order as the other tiles: same bits.
+using CfgS64 = Cfg<32, 3, 64, 2, 64>;
 
 // Exact negation as a sign-bit flip on the integer pipe (keeps the FP64/DMMA pipe free).
 __device__ __forceinline__ double neg(double x) {
@@ -269,6 +273,12 @@ static int gemm_narrow() {
   return v;
 }
 
+// SYRK (lower) tiles up to this order use the 64 x 64 CTA tile (STF_SYRK64_MAX, default 1024)
+static int syrk64_max() {
+  static int v = env_or("STF_SYRK64_MAX", 1024);
+  return v;
+}
+
 template <class G>
 static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tmA, const CUtensorMap& tmB, double* C,
                                   int64_t ldc, int M, int N, int K, int lower) {
@@ -291,15 +301,23 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   CUtensorMap tmA, tmB;
   if (!make_operand_map(&tmA, A, M, K, lda, bk) || !make_operand_map(&tmB, B, N, K, ldb, bk))
     return cudaErrorInvalidValue;
-  const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = lower ? dim3(narrow ? tM * (tM + 1) : tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
-  cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributePriority;
   attr[0].val.priority = prio;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  cfg.stream = stream;
+  if (lower && M <= syrk64_max() && bk == CfgS64::BK) {
+    const int t64 = (M + 63) / 64;
+    cfg.gridDim = dim3(t64 * (t64 + 1) / 2, 1, 1);
+    cfg.blockDim = dim3(128, 1, 1);
+    cfg.dynamicSmemBytes = CfgS64::SMEM_BYTES;
+    ++launch_count();
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgS64>, tmA, tmB, C, ldc, M, N, K, lower);
+  }
+  const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
+  cfg.gridDim = lower ? dim3(narrow ? tM * (tM + 1) : tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
   ++launch_count();
   if (narrow) {
     cfg.dynamicSmemBytes = CfgN64::SMEM_BYTES;
@@ -333,6 +351,9 @@ cudaError_t gemm_init_attrs() {
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, CfgN64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              CfgN64::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, CfgS64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             CfgS64::SMEM_BYTES);
   return e;
 }
 

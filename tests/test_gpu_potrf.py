@@ -240,6 +240,7 @@ def test_virtual_grids_p2_exact(stf, p, q, variant):
     L, L0, st = _p2(stf, 2048, 256, p, q, **variant)
     assert np.array_equal(L, L0)
     assert st["slots"] == p * q and st["transfers"] > 0
+    assert st["graph_fallback"] == 0 and st["graph"] == (0 if variant.get("graph") == 0 else 1)
     assert st["data_plane"] == (1 if variant.get("push") else 0)
     assert (st["pushed"] > 0) == bool(variant.get("push"))
 
