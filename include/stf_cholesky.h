@@ -227,6 +227,12 @@ int stf_dag_build_call(int64_t n, int64_t nb, int kind, int ngpus, int p, int q,
  * number of buffers.  Needs no GPU. */
 int stf_dag_tasks_io(int64_t cap_tasks, int64_t *io);
 
+/* Replica buffers written by the tasks of the last stf_dag_build(_call) on this
+ * thread besides their output (fused push, "push" = 1): mir[8*t] = count (<= 7),
+ * mir[8*t+1 ..] the buffer ids (-1 unused).  Returns the total number of pushed
+ * replica writes.  Needs no GPU. */
+int64_t stf_dag_tasks_mirrors(int64_t cap_tasks, int64_t *mir);
+
 /* Generic STF rule on an arbitrary access list (the Algorithm 1 example):
  * ntasks tasks, task t has nacc[t] accesses listed consecutively in data[] and
  * modes[] (1 = read, 2 = write, 3 = read-write).  Writes up to cap edges.

@@ -93,6 +93,13 @@ def dag_io(ntasks: int):
     return [((IO[3 * t], IO[3 * t + 1]), IO[3 * t + 2]) for t in range(ntasks)], nbuf
 
 
+def dag_mirrors(ntasks: int):
+    """Replica buffers each task of the last dag()/dag_call() also writes (fused push)."""
+    MI = (ctypes.c_int64 * (8 * max(1, ntasks)))()
+    check(_abi.stf_dag_tasks_mirrors(ntasks, MI), "stf_dag_tasks_mirrors")
+    return [[MI[8 * t + 1 + m] for m in range(MI[8 * t])] for t in range(ntasks)]
+
+
 def infer_edges(tasks: Sequence[Sequence[tuple]]) -> set:
     """Generic STF rule (C++ core) on [[(datum:int, mode:'r'|'w'|'rw'), ...], ...]."""
     mode_code = {"r": 1, "w": 2, "rw": 3}

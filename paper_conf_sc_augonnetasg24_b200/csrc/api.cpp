@@ -489,6 +489,21 @@ int stf_dag_tasks_io(int64_t cap_tasks, int64_t* io) {
   return (int)std::min<size_t>(plan.buffers.size(), INT_MAX);
 }
 
+int64_t stf_dag_tasks_mirrors(int64_t cap_tasks, int64_t* mir) {
+  g_err.clear();
+  const stf::Plan& plan = g_dag_plan;
+  int64_t total = 0;
+  for (size_t t = 0; t < plan.tasks.size(); ++t) {
+    const stf::Task& k = plan.tasks[t];
+    total += k.nmir;
+    if ((int64_t)t < cap_tasks && mir) {
+      mir[8 * t] = k.nmir;
+      for (int m = 0; m < 7; ++m) mir[8 * t + 1 + m] = m < k.nmir ? k.mir[m] : -1;
+    }
+  }
+  return total;
+}
+
 }  // extern "C"
 
 namespace {

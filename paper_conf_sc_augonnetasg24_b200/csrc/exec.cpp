@@ -84,6 +84,7 @@ stf::PlanOptions call_plan_options(const Options& o, int64_t n, int64_t nb, int 
   po.ooc_reorder = o.ooc_reorder != 0;
   po.dev_order = (int)o.dev_order;
   po.push = o.push != 0 && o.trsm >= 2;
+  po.push_potrf = po.push && o.dataflow != 0;  // the dataflow POTRF kernel stores into replicas
   po.ooc_order = (int)o.ooc_order;
   // Scheduling model of the submission order (plan.cpp reorder_list), in units of
   // one nb^3 GEMM task's duration while `width` of them share the GPU: a tile
@@ -169,10 +170,13 @@ struct Lowerer {
     Slot& S = C.slots[(size_t)t.slot];
     switch (t.kind) {
       case stf::K_POTRF:
-        if (X.opt.dataflow)
-          CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws),
+        if (X.opt.dataflow) {
+          stfk::Mirrors mir{};  // fused push of L_kk (NEXT-3): every final block also into the replicas
+          for (int m = 0; m < t.nmir && m < 7; ++m) mir.p[m] = X.buf[(size_t)t.mir[m]];
+          mir.n = t.nmir < 7 ? t.nmir : 7;
+          CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir),
                    "POTRF launch");
-        else
+        } else
           CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
                    "POTRF launch");
         return 0;

@@ -215,7 +215,7 @@ int64_t stf_debug_potrf_trace(int64_t n, double* A, int64_t lda, int ctas, int64
   if (e == cudaSuccess) e = cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)n, (int)n));
   if (e == cudaSuccess) e = stfk::dataflow_prepare((int)n, (int)n, true);
   if (e == cudaSuccess) e = stfk::info_reset(0, d_info);
-  if (e == cudaSuccess) e = stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws, d_tr, ctas);
+  if (e == cudaSuccess) e = stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws, nullptr, d_tr, ctas);
   if (e == cudaSuccess) e = cudaStreamSynchronize(0);
   const int64_t cnt = std::min<int64_t>(cap, slots);
   if (e == cudaSuccess && trace) e = cudaMemcpy(trace, d_tr, (size_t)cnt * 8, cudaMemcpyDeviceToHost);

@@ -70,6 +70,7 @@ struct DfParams {
   int potrf;
   int crit;  // POTRF: one CTA runs the critical chain P -> S -> U -> P (blocks kept in smem)
   unsigned long long* trace;  // debug: %globaltimer stamps (null in production)
+  Mirrors mir;                // POTRF: replicas of the tile, written with every final block (fused push)
 };
 
 __device__ __forceinline__ unsigned long long gtime() {
@@ -434,8 +435,10 @@ __device__ __forceinline__ void store_chunk(const double (&v)[16], double* G, in
   }
 }
 
-// S task: X[rows x nc] <- X L^-T with L = the nc x nc diagonal block at L (global).
-__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc) {
+// S task: X[rows x nc] <- X L^-T with L = the nc x nc diagonal block at L (global);
+// the result also goes to the mirrors at element offset `off` (fused push).
+__device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc,
+                           const Mirrors* mir = nullptr, int64_t off = 0) {
   double* Xs = sm;                    // publication buffer [r][LDB]
   double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
   double* Rc = Ls + df::W * df::LDB;
@@ -445,10 +448,14 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
   __syncthreads();
   solve_core(b, Ls, Rc, Xs, df::LDB, nc);
   store_chunk(b, X, ldx, rows, nc, false);
+  if (mir)
+    for (int m = 0; m < mir->n; ++m) store_chunk(b, mir->p[m] + off, ldx, rows, nc, false);
 }
 
-// P task: in-place lower Cholesky of the nc x nc diagonal block at X (global).
-__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info) {
+// P task: in-place lower Cholesky of the nc x nc diagonal block at X (global)
+// (+ the mirrors at element offset `off`).
+__device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t col0, unsigned long long* info,
+                          const Mirrors* mir = nullptr, int64_t off = 0) {
   double* S = sm;
   double* Lc = sm + df::W * df::LDB;
   double* Dp = Lc + 3 * df::W;
@@ -456,6 +463,8 @@ __device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t co
   load_il(a, X, ldx, nc, nc, true);
   chol_core(a, S, Lc, Dp, nc, col0, info);
   store_block_rm(S, df::LDB, X, ldx, nc, nc, true);
+  if (mir)
+    for (int m = 0; m < mir->n; ++m) store_block_rm(S, df::LDB, mir->p[m] + off, ldx, nc, nc, true);
 }
 
 // The critical path of the tile Cholesky, run by ONE CTA with its blocks kept
@@ -494,6 +503,7 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
     }
     store_block_rm(D, df::LDB, Xkk, p.ldx, nk, nk, true);
+    for (int m = 0; m < p.mir.n; ++m) store_block_rm(D, df::LDB, p.mir.p[m] + (Xkk - p.X), p.ldx, nk, nk, true);
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
@@ -530,11 +540,17 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
         XS[m * df::LDO + k] = Xp[(m >> 4) * 16 * W + sb::xo(m & 15, k)];
       }
       __syncthreads();
+      for (int mm = 0; mm < p.mir.n; ++mm)  // fused push of the finished block (solve_block wrote the home tile)
+        for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+          const int k = idx >> 6, m = idx & (W - 1);
+          if (m < rows) p.mir.p[mm][(Xik - p.X) + (int64_t)k * p.ldx + m] = XS[m * df::LDO + k];
+        }
     } else {
       double b[16];
       load_chunk(b, Xik, p.ldx, rows, nk, false);
       solve_core(b, D, Rc, XS, df::LDO, nk);
       store_chunk(b, Xik, p.ldx, rows, nk, false);
+      for (int m = 0; m < p.mir.n; ++m) store_chunk(b, p.mir.p[m] + (Xik - p.X), p.ldx, rows, nk, false);
       __syncthreads();
     }
     if (threadIdx.x == 0) {
@@ -645,9 +661,10 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
       double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
       const int nk = min(W, p.n - kb * W);
       if (type == df::T_P) {
-        task_chol(sm, Xkk, p.ldx, nk, p.col0 + (int64_t)kb * W, p.info);
+        task_chol(sm, Xkk, p.ldx, nk, p.col0 + (int64_t)kb * W, p.info, &p.mir, Xkk - p.X);
       } else if (type == df::T_S) {
-        task_solve(sm, p.X + (int64_t)kb * W * p.ldx + ib * W, p.ldx, Xkk, p.ldx, rows, nk);
+        double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
+        task_solve(sm, Xik, p.ldx, Xkk, p.ldx, rows, nk, &p.mir, Xik - p.X);
       } else {
         const int cols = min(W, p.n - jb * W);
         task_update(sm, p.X + (int64_t)jb * W * p.ldx + ib * W, p.ldx, p.X + (int64_t)kb * W * p.ldx + ib * W, p.ldx,
@@ -824,7 +841,8 @@ cudaError_t dataflow_init_attrs() {
 }
 
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
-                       unsigned long long* info, int* ws, unsigned long long* trace, int ctas_override) {
+                       unsigned long long* info, int* ws, const Mirrors* mirrors, unsigned long long* trace,
+                       int ctas_override) {
   if (n <= 0) return cudaSuccess;
   DfParams p{};
   p.X = A;
@@ -840,6 +858,7 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   p.col0 = col0;
   p.info = info;
   p.potrf = 1;
+  if (mirrors) p.mir = *mirrors;
   const int T = p.Nb;
   const int par = T * (T - 1) / 2 > 0 ? T * (T - 1) / 2 : 1;  // widest update wave
   int ctas = std::min(par, std::min(ctas_override > 0 ? ctas_override : df_max_ctas(T), num_sms()));

@@ -33,13 +33,23 @@ cudaError_t trsm_rlt(cudaStream_t stream, int prio, int M, int n, const double* 
 cudaError_t potrf_lower(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                         unsigned long long* info);
 
+// Replica destinations written by a kernel's epilogue together with the home
+// tile (same offsets and leading dimension): fused push of a finished tile.
+struct Mirrors {
+  double* p[7];
+  int n;
+};
+
 // K3/K4 as single-launch device-side dataflow kernels over 64 x 64 blocks
 // (dataflow.cu).  `ws` is a device workspace of dataflow_ws_bytes(m, n) bytes,
 // private to the launch (zeroed by the launcher with a memset on `stream`).
 // dataflow_prepare() uploads the task table for the shape; it must be called
-// once before the first launch of that shape inside a stream capture.
+// once before the first launch of that shape inside a stream capture.  POTRF:
+// every final block of L is also stored into each `mirrors` replica (fused push
+// of L_kk, NEXT-3).
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
-                       unsigned long long* info, int* ws, unsigned long long* trace = nullptr, int ctas = 0);
+                       unsigned long long* info, int* ws, const Mirrors* mirrors = nullptr,
+                       unsigned long long* trace = nullptr, int ctas = 0);
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                       int64_t ldb, int* ws);
 size_t dataflow_ws_bytes(int m, int n);
@@ -47,12 +57,6 @@ size_t dataflow_ws_bytes(int m, int n);
 // K3 row-panel form (trsm_panel.cu): one launch, ceil(M/R) CTAs each owning R
 // rows (R = 32: lower latency, 64: higher efficiency; 0 = STF_TRSM_ROWS, default
 // 64), left-looking over 64-wide column blocks (DMMA update + substitution).
-// Replica destinations written by a kernel's epilogue together with the home
-// tile (same offsets and leading dimension): fused push of a finished tile.
-struct Mirrors {
-  double* p[7];
-  int n;
-};
 cudaError_t trsm_panel(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                        int64_t ldb, int rows_per_cta = 0, const Mirrors* mirrors = nullptr);
 cudaError_t dataflow_prepare(int m, int n, bool potrf);

@@ -105,6 +105,17 @@ struct Builder {
     return s;
   }
 
+  // slots (other than the owner) whose TRSM(i,k), i > k, read the final L_kk
+  std::vector<int> consumers_of_diag_tile(int64_t k) const {
+    std::vector<int> s;
+    for (int64_t i = k + 1; i < T; ++i) {
+      const int g = p.owner(i, k);
+      if (g != p.owner(k, k) && std::find(s.begin(), s.end(), g) == s.end()) s.push_back(g);
+    }
+    std::sort(s.begin(), s.end());
+    return s;
+  }
+
   int64_t replica_buffer(int64_t i, int64_t j, int slot) {
     const int64_t d = Plan::tile_id(i, j);
     const size_t r = (size_t)(d * G + slot);
@@ -131,6 +142,7 @@ struct Builder {
     acc[n++] = {w, RW};
     std::vector<int> cons;
     if (kind == K_TRSM && p.opt.push) cons = consumers_of_panel_tile(wi, wj);
+    if (kind == K_POTRF && p.opt.push && p.opt.push_potrf) cons = consumers_of_diag_tile(wi);
     for (int g : cons) {
       const int64_t rb2 = replica_buffer(wi, wj, g);
       t.mir[t.nmir++] = rb2;

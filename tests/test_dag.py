@@ -108,20 +108,26 @@ def test_task_counts_closed_form(T):
 
 @pytest.mark.parametrize("T,p,q,known", [(8, 2, 2, None), (32, 2, 4, 1892)])
 def test_fused_push_replaces_panel_copies(T, p, q, known):
-    """NEXT-3: with push on, TRSM(i,k) writes L_ik's replicas itself: the only
-    COPY tasks left carry L_kk; total transfers are unchanged, and reachability
-    among compute tasks still equals the single-GPU STF closure."""
+    """NEXT-3: with push on, TRSM(i,k) writes L_ik's replicas and POTRF(k) writes
+    L_kk's from their epilogues: no COPY task is left, total transfers are
+    unchanged (all of them pushes), and reachability among compute tasks still
+    equals the single-GPU STF closure.  With the recursive POTRF (dataflow 0)
+    L_kk still moves by COPY."""
     stf.set_option("push", 1)
     try:
         edges, kinds, ijk, st = stf.dag(T, p, q)
+        stf.set_option("dataflow", 0)
+        _, kinds0, ijk0, st0 = stf.dag(T, p, q)
     finally:
         stf.set_option("push", 0)
-    assert st["transfers"] == _expected_transfers(T, p, q)
+        stf.set_option("dataflow", 1)
+    assert st["transfers"] == _expected_transfers(T, p, q) == st0["transfers"]
     if known:
         assert st["transfers"] == known
-    for t, k in enumerate(kinds):
+    assert "COPY" not in kinds and st["pushed"] == st["transfers"] and st["data_plane"] == 1
+    for t, k in enumerate(kinds0):
         if k == "COPY":
-            i, j, _ = ijk[t]
+            i, j, _ = ijk0[t]
             assert i == j  # only diagonal (POTRF) tiles are still copied
     comp = [t for t, k in enumerate(kinds) if k != "COPY"]
     R = oracle.transitive_closure(len(kinds), set(edges))

@@ -20,18 +20,26 @@ import synth
 NB = 4  # tile order for the emulation (values are irrelevant to the schedule)
 
 
-def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1):
+def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0):
     stf.set_option("mem_cap_tiles", frames)
     stf.set_option("lookahead", lookahead)
     stf.set_option("ooc_order", ooc_order)
+    stf.set_option("push", push)
     try:
         edges, kinds, ijk, st = stf.dag(T, p, q)
         io, nbuf = stf.dag_io(len(kinds))
+        mir = stf.dag_mirrors(len(kinds))
     finally:
         stf.set_option("mem_cap_tiles", 0)
         stf.set_option("lookahead", 1)
         stf.set_option("ooc_order", -1)
+        stf.set_option("push", 0)
+    _MIRRORS.clear()
+    _MIRRORS.extend(mir)
     return edges, kinds, ijk, io, nbuf, st
+
+
+_MIRRORS = []  # replica writes (fused push) of the tasks of the last _plan()
 
 
 def _emulate(T, A, kinds, ijk, io, nbuf, edges, order_seed, host_resident):
@@ -76,6 +84,9 @@ def _emulate(T, A, kinds, ijk, io, nbuf, edges, order_seed, host_resident):
             H[(i, j)][:, :] = buf[r0]
         else:
             assert kd == "FENCE"
+        if _MIRRORS and kd in ("POTRF", "TRSM"):  # fused push: the epilogue also writes these replicas
+            for m in _MIRRORS[t]:
+                buf[m][:, :] = buf[w]
         done += 1
         for d in succ[t]:
             indeg[d] -= 1
@@ -97,10 +108,16 @@ def _reference(T, A):
     return np.tril(L)
 
 
-@pytest.mark.parametrize("T,p,q,lookahead", [(5, 1, 1, 1), (6, 1, 2, 1), (6, 2, 2, 1), (7, 2, 4, 1), (6, 2, 2, 0)])
-def test_distributed_plan_any_topological_order(T, p, q, lookahead):
+@pytest.mark.parametrize("push", [0, 1])
+@pytest.mark.parametrize("T,p,q,lookahead", [(5, 1, 1, 1), (6, 1, 2, 1), (6, 2, 2, 1), (7, 2, 4, 1), (6, 2, 2, 0),
+                                             (9, 1, 8, 1), (9, 1, 8, 0)])
+def test_distributed_plan_any_topological_order(T, p, q, lookahead, push):
+    """2D block-cyclic grids and the 1D column block-cyclic 1 x 8 grid (cuSolverMg's
+    layout), with and without per-step fences, COPY tasks or fused pushes."""
     A = synth.spd_matrix(7, T * NB)
-    edges, kinds, ijk, io, nbuf, st = _plan(T, p, q, lookahead=lookahead)
+    edges, kinds, ijk, io, nbuf, st = _plan(T, p, q, lookahead=lookahead, push=push)
+    if push and p * q > 1:
+        assert "COPY" not in kinds and st["pushed"] == st["transfers"] > 0
     ref = _reference(T, A)
     for seed in (-1, 1, 2, 3):
         got = _emulate(T, A, kinds, ijk, io, nbuf, edges, seed, host_resident=False)
@@ -192,6 +209,8 @@ def test_out_of_core_2d_order_cuts_panel_reloads():
 def _call_plan(n, nb, kind, p=1, q=1):
     edges, kinds, ijk, st = stf.dag_call(n, nb, kind, p, q)
     io, nbuf = stf.dag_io(len(kinds))
+    _MIRRORS.clear()
+    _MIRRORS.extend(stf.dag_mirrors(len(kinds)))
     return edges, kinds, ijk, io, nbuf, st
 
 
