@@ -233,7 +233,8 @@ def run_ours(args, rank, world):
             torch.cuda.set_device(0 if args.virtual else int(os.environ.get("LOCAL_RANK", "0")))
     N = args.gpus
     n, nb = args.n, args.nb
-    P, Q = grid_for(N)
+    P, Q = grid_for(N) if not args.grid else tuple(int(x) for x in args.grid.lower().split("x"))
+    assert P * Q == N, "--grid must have P*Q == --gpus"
     mode = args.mode or ("mp" if dist_on else "single")
     if mode == "mp":
         assert dist_on and world == N, "--mode mp needs torchrun with one rank per GPU"
@@ -537,6 +538,7 @@ def main():
     ap.add_argument("--n", "--order", dest="n", type=int, default=65536)
     ap.add_argument("--nb", "--tile", dest="nb", type=int, default=1024)
     ap.add_argument("--virtual-slots", dest="virtual", type=int, default=0, help="map all slots onto cuda:0")
+    ap.add_argument("--grid", default="", help="PxQ process grid (default: P <= Q, P maximal)")
     ap.add_argument("--mode", default=None, choices=["single", "mp"],
                     help="N>1: mp = one process per GPU (default under torchrun), single = rank 0 drives all GPUs")
     ap.add_argument("--e2e-steps", type=int, default=2)
