@@ -125,8 +125,14 @@ const char *stf_last_error(void);
  *   "priority" STF_PRIO     1: critical-path tasks on high-priority streams (default 1)
  *   "prio_mode" STF_PRIO_MODE  priority level assignment variant (0 default; 1..3 ablations)
  *   "grid_p"   STF_GRID     rows P of the P x Q grid for COLMAJOR kinds (0 = auto)
- *   "push"     STF_PUSH     1: TRSM(i,k) writes L_ik into its consumers' replicas from its own
- *                           epilogue (fused push over NVLink, NEXT-3); 0: COPY tasks (default)
+ *   "push"     STF_PUSH     data plane of the finished-tile broadcast (NEXT-3):
+ *                           0 (default) COPY tasks on the producer's copy streams (copy engine);
+ *                           1 fused push: the POTRF(k) / TRSM(i,k) epilogues store L_kk / L_ik
+ *                           straight into every consumer's replica (peer stores over NVLink);
+ *                           2 the same through one NVSwitch multicast object (multimem.st: one
+ *                           store reaches every device) when the call spans >= 2 distinct
+ *                           devices that support multicast, in single-process mode; else as 1
+ *                           (stf_plan_stats.data_plane reports what ran)
  *   "threads"  STF_THREADS  eager backend: host submission threads, slots split round-robin
  *                           (default 8, capped at ngpus; the graph backend captures on one thread)
  *   "lookahead" STF_LOOKAHEAD 1: pure STF DAG (default); 0: a fence task closes every
@@ -190,7 +196,8 @@ typedef struct stf_plan_stats {
   int64_t frames;         /* device tile frames of an out-of-core plan ("mem_cap_tiles"), else 0 */
   int64_t pushed;         /* replicas written by fused epilogue pushes (part of transfers) */
   int64_t replicas_max;   /* largest number of replica tiles held by one slot */
-  int64_t data_plane;     /* 0 COPY tasks (copy engine), 1 fused epilogue push */
+  int64_t data_plane;     /* 0 COPY tasks (copy engine), 1 fused epilogue push (peer stores),
+                             2 fused push through an NVSwitch multicast object */
   int64_t graph_fallback; /* 1: the graph capture was rejected and the eager backend ran */
   int64_t graph;          /* 1: the call ran as one CUDA graph launch, 0: eager streams */
   int64_t devices;        /* distinct CUDA devices spanned by the call's slots */

@@ -33,6 +33,7 @@ SOURCES = [
     "exec.cpp",
     "mp.cpp",
     "harness.cpp",
+    "mcast.cpp",
 ]
 
 

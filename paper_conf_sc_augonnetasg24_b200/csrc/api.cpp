@@ -51,7 +51,7 @@ const std::vector<OptDesc>& option_table() {
       {"grid_p", "STF_GRID", &Options::grid_p, 0, 64, false},  // the grid itself is part of the key
       {"lookahead", "STF_LOOKAHEAD", &Options::lookahead, 0, 1, true},
       {"threads", "STF_THREADS", &Options::threads, 1, 64, false},  // eager submission only
-      {"push", "STF_PUSH", &Options::push, 0, 1, true},
+      {"push", "STF_PUSH", &Options::push, 0, 2, true},
       {"mem_cap_tiles", "STF_MEM_CAP_TILES", &Options::mem_cap_tiles, 0, INT64_MAX, true},
       {"ooc_order", "STF_OOC_ORDER", &Options::ooc_order, -1, 1, true},
       {"host_stream", "STF_HOST_STREAM", &Options::host_stream, 0, 1, true},

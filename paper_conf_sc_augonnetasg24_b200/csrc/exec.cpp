@@ -85,6 +85,7 @@ stf::PlanOptions call_plan_options(const Options& o, int64_t n, int64_t nb, int 
   po.dev_order = (int)o.dev_order;
   po.push = o.push != 0 && o.trsm >= 2;
   po.push_potrf = po.push && o.dataflow != 0;  // the dataflow POTRF kernel stores into replicas
+  po.data_plane = po.push ? (int)o.push : 0;
   po.ooc_order = (int)o.ooc_order;
   // Scheduling model of the submission order (plan.cpp reorder_list), in units of
   // one nb^3 GEMM task's duration while `width` of them share the GPU: a tile
@@ -154,6 +155,21 @@ struct Lowerer {
     return v > lo ? lo : v;
   }
 
+  // replica destinations of a pushing task: each replica, or the multicast address of the tile
+  stfk::Mirrors mirrors_of(const stf::Task& t) const {
+    stfk::Mirrors mir{};
+    if (t.nmir <= 0) return mir;
+    if (X.mcs && X.mc_off[(size_t)t.out] >= 0) {
+      mir.p[0] = reinterpret_cast<double*>(X.mcs->mcva) + X.mc_off[(size_t)t.out];
+      mir.n = 1;
+      mir.mc = 1;
+      return mir;
+    }
+    for (int m = 0; m < t.nmir && m < 7; ++m) mir.p[m] = X.buf[(size_t)t.mir[m]];
+    mir.n = t.nmir < 7 ? t.nmir : 7;
+    return mir;
+  }
+
   static cudaError_t trace_record(cudaEvent_t ev, cudaStream_t s) {
     cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
     cudaStreamIsCapturing(s, &st);
@@ -171,9 +187,7 @@ struct Lowerer {
     switch (t.kind) {
       case stf::K_POTRF:
         if (X.opt.dataflow) {
-          stfk::Mirrors mir{};  // fused push of L_kk (NEXT-3): every final block also into the replicas
-          for (int m = 0; m < t.nmir && m < 7; ++m) mir.p[m] = X.buf[(size_t)t.mir[m]];
-          mir.n = t.nmir < 7 ? t.nmir : 7;
+          stfk::Mirrors mir = mirrors_of(t);  // fused push of L_kk (NEXT-3): final blocks also into the replicas
           CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir),
                    "POTRF launch");
         } else
@@ -181,9 +195,7 @@ struct Lowerer {
                    "POTRF launch");
         return 0;
       case stf::K_TRSM: {
-        stfk::Mirrors mir{};
-        for (int m = 0; m < t.nmir && m < 7; ++m) mir.p[m] = X.buf[(size_t)t.mir[m]];
-        mir.n = t.nmir < 7 ? t.nmir : 7;
+        stfk::Mirrors mir = mirrors_of(t);
         if ((skip & (3u << 16)) && t.i != t.k + 1) {  // debug what-if: non-critical TRSM costed as a GEMM
           const int kk = (skip & (1u << 17)) ? (int)(nb / 2) : (int)nb;  // (half: triangular-GEMM flops)
           CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, kk, X.buf[(size_t)t.out], nb, X.buf[(size_t)t.in[0]],
@@ -579,12 +591,41 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
     X.peer_arena.assign((size_t)X.ngpus, nullptr);
     X.peer_flags.assign((size_t)X.ngpus, nullptr);
   }
+  // push = 2: the pushed tiles' replicas in one NVSwitch multicast slab (mcast.cpp)
+  X.data_plane = P.opt.push ? 1 : 0;
+  auto in_slab = [&](const stf::Buffer& B) {
+    return X.mcs && B.replica && X.mc_off[(size_t)stf::Plan::tile_id(B.i, B.j)] >= 0;
+  };
+  if (P.opt.push && X.opt.push == 2 && !X.mp && X.ngpus >= 2 && X.ndevices == X.ngpus) {
+    std::vector<int> devs;
+    for (int s = 0; s < X.ngpus; ++s) devs.push_back(C.slots[(size_t)s].device);
+    std::string why;
+    if (mc_supported(devs, &why)) {
+      X.mc_off.assign((size_t)P.ntiles(), -1);
+      int64_t cnt = 0;
+      for (const stf::Task& t : P.tasks)
+        if (t.nmir > 0 && X.mc_off[(size_t)t.out] < 0) X.mc_off[(size_t)t.out] = (cnt++) * X.nb * X.nb;
+      std::unique_ptr<McSlab> S(new McSlab());
+      const int r = mc_create(*S, devs, (size_t)cnt * tile_bytes, &why);
+      if (r == 0) {
+        X.mcs = std::move(S);
+        X.data_plane = 2;
+        for (size_t b = 0; b < P.buffers.size(); ++b)
+          if (in_slab(P.buffers[b]))
+            X.buf[b] = reinterpret_cast<double*>(X.mcs->uc[(size_t)P.buffers[b].slot]) +
+                       X.mc_off[(size_t)stf::Plan::tile_id(P.buffers[b].i, P.buffers[b].j)];
+      } else if (r == -103) {
+        return fail(-103, "multicast slab: %s", why.c_str());
+      }
+    }
+    if (!X.mcs && getenv("STF_DEBUG_MC")) fprintf(stderr, "stf: push=2 keeps peer stores: %s\n", why.c_str());
+  }
   // library-owned storage: per slot one arena for (COLMAJOR) home tiles + replicas
   for (int s = 0; s < X.ngpus && !X.mp; ++s) {
     size_t count = 0;
     for (size_t b = 0; b < P.buffers.size(); ++b) {
       const stf::Buffer& B = P.buffers[b];
-      if (B.slot == s && (B.replica || colmajor)) count++;
+      if (B.slot == s && (B.replica || colmajor) && !in_slab(B)) count++;
     }
     const size_t nscr = (colmajor && X.uplo == 'U') ? kCopyStreams : 0;
     if (count + nscr == 0) continue;
@@ -594,7 +635,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
     size_t used = 0;
     for (size_t b = 0; b < P.buffers.size(); ++b) {
       const stf::Buffer& B = P.buffers[b];
-      if (B.slot == s && (B.replica || colmajor)) X.buf[b] = arena + (used++) * (size_t)(X.nb * X.nb);
+      if (B.slot == s && (B.replica || colmajor) && !in_slab(B)) X.buf[b] = arena + (used++) * (size_t)(X.nb * X.nb);
     }
     if (nscr) {
       X.scratch.resize((size_t)X.ngpus * kCopyStreams, nullptr);
@@ -765,7 +806,7 @@ void fill_plan_stats(const stf::Plan& P, int64_t nb, stf_plan_stats* s) {
   int64_t mx = 0;
   for (int64_t r : P.replicas_per_slot) mx = std::max(mx, r);
   s->replicas_max = mx;
-  s->data_plane = P.opt.push ? 1 : 0;
+  s->data_plane = P.opt.data_plane;
 }
 
 void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
@@ -779,6 +820,7 @@ void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
   s->devices = X.ndevices;
   s->slots = X.ngpus;
   s->peer_transfers = X.peer_transfers;
+  s->data_plane = X.data_plane;
 }
 
 }  // namespace stfrt

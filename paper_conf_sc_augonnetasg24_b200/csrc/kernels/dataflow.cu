@@ -124,6 +124,16 @@ __device__ __forceinline__ void store_block_rm(const double* S, int ld, double* 
   }
 }
 
+// mirror (fused push) forms of the stores below: plain or multimem stores
+__device__ __forceinline__ void mirror_block_rm(const double* S, int ld, double* G, int64_t ldg, int rows, int cols,
+                                                bool lower_only, int mc) {
+  for (int idx = threadIdx.x; idx < df::W * df::W; idx += df::NT) {
+    const int r = idx & (df::W - 1), c = idx >> 6;
+    if (r < rows && c < cols && (!lower_only || r >= c)) mirror_st(G + (int64_t)c * ldg + r, S[r * ld + c], mc);
+  }
+  mirror_fence(mc);
+}
+
 __device__ __forceinline__ double negd(double x) {
   return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
 }
@@ -302,26 +312,39 @@ __device__ __forceinline__ void chol_core(double (&a)[16], double* S, double* Lc
   __syncthreads();
 }
 
+__device__ __forceinline__ void bar_sync_id(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void bar_arrive_id(int id, int n) {
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
 // P of a full 64 x 64 diagonal block held row-major in D (lower part, LDB stride),
 // in place, latency-optimised for the critical chain.  8 panels of 8 columns:
 //   (a) warp 0 factors the panel: every lane factors the 8 x 8 diagonal block
 //       redundantly in registers (no shuffles on the sqrt -> reciprocal -> divide
 //       chain) and the two rows it owns below it (lane, lane + 32);
-//   (b) six warps on the other SM sub-partitions apply the panel to the trailing
-//       lower block on DMMA (K = 8), so the chain warp's FP64 pipe stays free.
+//   (b) six warps on the other SM sub-partitions (1-3, 5-7) apply the panel to the
+//       trailing lower block on DMMA (K = 8) with a look-ahead of one panel: the
+//       next panel's columns first -- then they release warp 0 (named barrier
+//       NEXT) -- and the remaining columns while warp 0 already factors the next
+//       panel (barrier DONE hands each finished panel to them).  Each 8 x 8
+//       output tile has one owner warp for the whole block (static map), so its
+//       updates stay in increasing panel order.
 // Correctly rounded sqrt and division (div_by with y = RN(1/s)); every element
 // receives its updates in increasing column order, each a single fma or a DMMA
-// k-step pair, deterministic.  Non-positive pivot (or NaN): info = min(info,
-// col0 + col + 1), s = NaN.
+// k-step pair, deterministic (the same operations as without look-ahead).
+// Non-positive pivot (or NaN): info = min(info, col0 + col + 1), s = NaN.
 __device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
-  constexpr int LD = df::LDB;
+  constexpr int LD = df::LDB, BAR_DONE = 1, BAR_NEXT = 2;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
-  int bad = 0;
+  // warp 4 shares warp 0's sub-partition: it stays out of the FP64 pipe
+  constexpr int NPART = 6 * 32 + 32;  // barrier participants: six MMA warps + warp 0
+  if (warp == 0) {
+    int bad = 0;
 #pragma unroll 1
-  for (int p = 0; p < 8; ++p) {
-    const int c0 = 8 * p;
-    if (warp == 0) {
+    for (int p = 0; p < 8; ++p) {
+      if (p > 0) bar_sync_id(BAR_NEXT, NPART);  // columns 8p .. 8p+7 received the update from panel p-1
+      const int c0 = 8 * p;
       double dg[8][8];
 #pragma unroll
       for (int i = 0; i < 8; ++i)
@@ -367,31 +390,38 @@ __device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
         if (b1) D[r1 * LD + c0 + j] = v1[j];
         if (b2) D[r2 * LD + c0 + j] = v2[j];
       }
+      bar_arrive_id(BAR_DONE, NPART);  // panel p final
     }
-    __syncthreads();
-    if (p < 7 && warp != 0 && warp != 4) {  // trailing lower block, rows and columns >= c0 + 8
-      const int mw = warp < 4 ? warp - 1 : warp - 2;  // 0..5
-      const int nf = 7 - p, npairs = nf * (nf + 1) / 2;
-      for (int idx = mw; idx < npairs; idx += 6) {
-        int fi = 0;
-        while ((fi + 1) * (fi + 2) / 2 <= idx) ++fi;
-        const int fj = idx - fi * (fi + 1) / 2;
-        const int R0 = c0 + 8 + 8 * fi, C0 = c0 + 8 + 8 * fj;
-        double* cp = D + (R0 + g) * LD + C0 + 2 * t;
-        double acc0 = cp[0], acc1 = cp[1];
+    if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
+  } else if (warp != 4) {
+    const int mw = warp < 4 ? warp - 1 : warp - 2;  // 0..5
+    auto update = [&](int R, int Cb, int c0) {      // tile rows 8R.., columns 8Cb.. from panel columns c0..
+      double* rowp = D + (8 * R + g) * LD;
+      double* cp = rowp + 8 * Cb + 2 * t;
+      double acc0 = cp[0], acc1 = cp[1];
 #pragma unroll
-        for (int ks = 0; ks < 2; ++ks) {
-          const double a = D[(R0 + g) * LD + c0 + 4 * ks + t];
-          const double b = negd(D[(C0 + g) * LD + c0 + 4 * ks + t]);
-          dmma_8x8x4(acc0, acc1, a, b);
-        }
-        cp[0] = acc0;
-        cp[1] = acc1;
+      for (int ks = 0; ks < 2; ++ks) {
+        const double a = rowp[c0 + 4 * ks + t];
+        const double b = negd(D[(8 * Cb + g) * LD + c0 + 4 * ks + t]);
+        dmma_8x8x4(acc0, acc1, a, b);
       }
+      cp[0] = acc0;
+      cp[1] = acc1;
+    };
+#pragma unroll 1
+    for (int p = 0; p < 7; ++p) {
+      bar_sync_id(BAR_DONE, NPART);  // panel p is final
+      const int c0 = 8 * p;
+      for (int R = p + 1; R < 8; ++R)  // look-ahead: the next panel's columns
+        if ((R + 5 * (p + 1)) % 6 == mw) update(R, p + 1, c0);
+      bar_arrive_id(BAR_NEXT, NPART);
+      for (int Cb = p + 2; Cb < 8; ++Cb)  // the remaining trailing lower part
+        for (int R = Cb; R < 8; ++R)
+          if ((R + 5 * Cb) % 6 == mw) update(R, Cb, c0);
     }
-    __syncthreads();
+    bar_sync_id(BAR_DONE, NPART);  // panel 7
   }
-  if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
+  __syncthreads();
 }
 
 // interleaved-column register blocks (chol_core layout): v[m] = G(r, 4m + q)
@@ -435,6 +465,18 @@ __device__ __forceinline__ void store_chunk(const double (&v)[16], double* G, in
   }
 }
 
+__device__ __forceinline__ void store_chunk_m(const double (&v)[16], double* G, int64_t ldg, int rows, int nc, int mc) {
+  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
+  if (r < rows) {
+#pragma unroll
+    for (int c = 0; c < 16; ++c) {
+      const int col = 16 * q + c;
+      if (col < nc) mirror_st(G + (int64_t)col * ldg + r, v[c], mc);
+    }
+  }
+  mirror_fence(mc);
+}
+
 // S task: X[rows x nc] <- X L^-T with L = the nc x nc diagonal block at L (global);
 // the result also goes to the mirrors at element offset `off` (fused push).
 __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc,
@@ -449,7 +491,7 @@ __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, 
   solve_core(b, Ls, Rc, Xs, df::LDB, nc);
   store_chunk(b, X, ldx, rows, nc, false);
   if (mir)
-    for (int m = 0; m < mir->n; ++m) store_chunk(b, mir->p[m] + off, ldx, rows, nc, false);
+    for (int m = 0; m < mir->n; ++m) store_chunk_m(b, mir->p[m] + off, ldx, rows, nc, mir->mc);
 }
 
 // P task: in-place lower Cholesky of the nc x nc diagonal block at X (global)
@@ -464,7 +506,7 @@ __device__ void task_chol(double* sm, double* X, int64_t ldx, int nc, int64_t co
   chol_core(a, S, Lc, Dp, nc, col0, info);
   store_block_rm(S, df::LDB, X, ldx, nc, nc, true);
   if (mir)
-    for (int m = 0; m < mir->n; ++m) store_block_rm(S, df::LDB, mir->p[m] + off, ldx, nc, nc, true);
+    for (int m = 0; m < mir->n; ++m) mirror_block_rm(S, df::LDB, mir->p[m] + off, ldx, nc, nc, true, mir->mc);
 }
 
 // The critical path of the tile Cholesky, run by ONE CTA with its blocks kept
@@ -503,7 +545,8 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
     }
     store_block_rm(D, df::LDB, Xkk, p.ldx, nk, nk, true);
-    for (int m = 0; m < p.mir.n; ++m) store_block_rm(D, df::LDB, p.mir.p[m] + (Xkk - p.X), p.ldx, nk, nk, true);
+    for (int m = 0; m < p.mir.n; ++m)
+      mirror_block_rm(D, df::LDB, p.mir.p[m] + (Xkk - p.X), p.ldx, nk, nk, true, p.mir.mc);
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
@@ -543,14 +586,15 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       for (int mm = 0; mm < p.mir.n; ++mm)  // fused push of the finished block (solve_block wrote the home tile)
         for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
           const int k = idx >> 6, m = idx & (W - 1);
-          if (m < rows) p.mir.p[mm][(Xik - p.X) + (int64_t)k * p.ldx + m] = XS[m * df::LDO + k];
+          if (m < rows) mirror_st(p.mir.p[mm] + (Xik - p.X) + (int64_t)k * p.ldx + m, XS[m * df::LDO + k], p.mir.mc);
         }
+      if (p.mir.n) mirror_fence(p.mir.mc);
     } else {
       double b[16];
       load_chunk(b, Xik, p.ldx, rows, nk, false);
       solve_core(b, D, Rc, XS, df::LDO, nk);
       store_chunk(b, Xik, p.ldx, rows, nk, false);
-      for (int m = 0; m < p.mir.n; ++m) store_chunk(b, p.mir.p[m] + (Xik - p.X), p.ldx, rows, nk, false);
+      for (int m = 0; m < p.mir.n; ++m) store_chunk_m(b, p.mir.p[m] + (Xik - p.X), p.ldx, rows, nk, p.mir.mc);
       __syncthreads();
     }
     if (threadIdx.x == 0) {

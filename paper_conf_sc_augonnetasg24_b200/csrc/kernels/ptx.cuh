@@ -78,4 +78,19 @@ __device__ __forceinline__ double div_by(double a, double d, double y) {
   return fma(r, y, q0);
 }
 
+// Store of one replica element (fused push): a plain (possibly peer, over NVLink)
+// store, or with mc a multimem store to a multicast address, which the NVSwitch
+// delivers to every device bound to the multicast object.
+__device__ __forceinline__ void mirror_st(double* p, double v, int mc) {
+  if (mc)
+    asm volatile("multimem.st.relaxed.sys.global.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+  else
+    *p = v;
+}
+// After a thread's last multimem store: make it visible system-wide before the
+// kernel completes (the consumer's wait is an event / stream-ordered hand-off).
+__device__ __forceinline__ void mirror_fence(int mc) {
+  if (mc) asm volatile("fence.acq_rel.sys;" ::: "memory");
+}
+
 }  // namespace stfk

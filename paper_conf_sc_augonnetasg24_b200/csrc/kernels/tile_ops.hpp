@@ -35,9 +35,13 @@ cudaError_t potrf_lower(cudaStream_t stream, int prio, int n, double* A, int64_t
 
 // Replica destinations written by a kernel's epilogue together with the home
 // tile (same offsets and leading dimension): fused push of a finished tile.
+// mc != 0: p[0] is a multicast address (NVSwitch multicast object bound on every
+// consumer device, cuMulticastCreate): one multimem.st per element reaches all
+// replicas, the switch replicates (n == 1).
 struct Mirrors {
   double* p[7];
   int n;
+  int mc;
 };
 
 // K3/K4 as single-launch device-side dataflow kernels over 64 x 64 blocks

@@ -217,9 +217,10 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
             const int64_t off = (int64_t)(c0 + cc) * ldx + r0 + rr;
 #pragma unroll
             for (int m = 0; m < 7; ++m)
-              if (m < mir.n) mir.p[m][off] = v;
+              if (m < mir.n) mirror_st(mir.p[m] + off, v, mir.mc);
           }
         }
+        mirror_fence(mir.mc);
       }
     } else if constexpr (tp::BM <= 64) {
       // ragged last block: row-chunked substitution, S[r][c] = acc
@@ -274,9 +275,10 @@ __global__ void __launch_bounds__(256, 1) trsm_panel_kernel(const double* __rest
             // consumers' replicas (peer memory over NVLink / another slot's arena)
   #pragma unroll
             for (int m = 0; m < 7; ++m)
-              if (m < mir.n) mir.p[m][off] = b[c];
+              if (m < mir.n) mirror_st(mir.p[m] + off, b[c], mir.mc);
           }
         }
+        mirror_fence(mir.n > 0 ? mir.mc : 0);
       }
     }
     __threadfence();  // X[rows, jb] is re-read (cp.async.cg, L2) by the next jb iterations

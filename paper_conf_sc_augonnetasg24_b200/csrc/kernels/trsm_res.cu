@@ -298,8 +298,9 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
         for (int m = 0; m < mir.n && m < 7; ++m) {
           double* dst = mir.p[m];
 #pragma unroll 8
-          for (int j = 0; j < W; ++j) dst[(int64_t)(c0 + j) * ldx + r0 + r] = Xs[xo(r, c0 + j)];
+          for (int j = 0; j < W; ++j) mirror_st(dst + (int64_t)(c0 + j) * ldx + r0 + r, Xs[xo(r, c0 + j)], mir.mc);
         }
+        mirror_fence(mir.mc);
       }
       __syncwarp();
       if (lane == 0) tr_stamp(trace, 5 * Nb + jb);  // solve end

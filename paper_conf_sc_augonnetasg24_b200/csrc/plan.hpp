@@ -65,6 +65,7 @@ struct PlanOptions {
                            // step k+1 starts only when step k is complete (ablation, NEXT-1)
   bool push = false;       // TRSM(i,k) writes L_ik into its consumers' replicas itself (fused
                            // push, NEXT-3) instead of COPY tasks at the first remote read
+  int data_plane = 0;      // requested data plane (statistics): 0 COPY, 1 fused push, 2 multicast
   bool push_potrf = false; // with push: POTRF(k) also writes L_kk into the replicas of the
                            // slots running TRSM(i,k) (the dataflow POTRF kernel's epilogue)
   int64_t frames = 0;      // > 0 (one slot, with_load/with_store): memory-capped out-of-core

@@ -63,7 +63,7 @@ struct Options {
   int64_t grid_p = 0;          // rows P of the P x Q grid for COLMAJOR kinds (0 auto)
   int64_t lookahead = 1;       // 0: FENCE task closes each panel step (ablation)
   int64_t threads = 8;         // eager backend: host submission threads
-  int64_t push = 0;            // data plane: 0 COPY tasks, 1 fused epilogue push, 2 multicast, 3 NCCL
+  int64_t push = 0;            // data plane: 0 COPY tasks, 1 fused epilogue push, 2 fused push via NVSwitch multicast
   int64_t mem_cap_tiles = 0;   // HOST_COLMAJOR on one GPU: device tile frames (0 = no cap)
   int64_t ooc_order = -1;      // out-of-core program order: 0 tall, 1 2D-blocked, -1 auto
   int64_t host_stream = 1;     // HOST_COLMAJOR on one GPU, nb >= 512, T >= 16: frame-per-tile OOC builder
@@ -106,6 +106,20 @@ struct Slot {
   unsigned long long* d_info = nullptr;
 };
 
+// NVSwitch multicast slab (mcast.cpp): one multicast object bound on every device of a call
+struct McSlab {
+  CUmemGenericAllocationHandle mc = 0;
+  size_t size = 0;
+  std::vector<int> devs;
+  std::vector<CUmemGenericAllocationHandle> phys;  // per device: its physical copy
+  std::vector<CUdeviceptr> uc;                     // per device: its mapping of its copy
+  std::vector<char> bound;
+  CUdeviceptr mcva = 0;                            // the multicast mapping
+  ~McSlab();
+};
+bool mc_supported(const std::vector<int>& devs, std::string* why);
+int mc_create(McSlab& S, const std::vector<int>& devs, size_t bytes, std::string* why);
+
 constexpr int kCritStreams = 6;  // 0: panel chain, 1: its feeders, 2..5: other urgent tasks by row
 constexpr int kCopyStreams = 2;
 constexpr size_t kCacheMax = 4;
@@ -139,6 +153,9 @@ struct Exec {
   int64_t launches = 0;
   double build_ms = 0;
   int ndevices = 1;                  // distinct CUDA devices spanned by the slots of the call
+  int data_plane = 0;                // 0 COPY tasks, 1 fused push (peer stores), 2 fused push via multicast
+  std::unique_ptr<McSlab> mcs;       // push = 2: the multicast slab (null when not eligible)
+  std::vector<int64_t> mc_off;       // per home tile: element offset of its replicas in the slab (-1: none)
   int64_t peer_transfers = 0;        // COPY tasks / pushes whose endpoints are distinct devices
   // caller matrix for COLMAJOR kinds
   double* mat = nullptr;

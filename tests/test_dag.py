@@ -125,6 +125,12 @@ def test_fused_push_replaces_panel_copies(T, p, q, known):
     if known:
         assert st["transfers"] == known
     assert "COPY" not in kinds and st["pushed"] == st["transfers"] and st["data_plane"] == 1
+    stf.set_option("push", 2)  # multicast data plane: the same plan (pushes), lowered through one multicast object
+    try:
+        e2, k2, ijk2, st2 = stf.dag(T, p, q)
+    finally:
+        stf.set_option("push", 0)
+    assert (e2, k2, ijk2) == (edges, kinds, ijk) and st2["data_plane"] == 2
     for t, k in enumerate(kinds0):
         if k == "COPY":
             i, j, _ = ijk0[t]

@@ -231,8 +231,9 @@ def test_schedule_variants_p2_exact(stf, variant):
 
 
 @pytest.mark.parametrize("p,q", [(1, 2), (2, 1), (2, 2), (2, 4), (1, 8)])
-@pytest.mark.parametrize("variant", [{}, {"graph": 0, "threads": 1}, {"graph": 0}, {"push": 1}, {"lookahead": 0}],
-                         ids=["graph", "eager1", "eager_threads", "push", "fence"])
+@pytest.mark.parametrize("variant", [{}, {"graph": 0, "threads": 1}, {"graph": 0}, {"push": 1}, {"push": 2},
+                                     {"push": 1, "graph": 0}, {"lookahead": 0}],
+                         ids=["graph", "eager1", "eager_threads", "push", "push_mc", "push_eager", "fence"])
 def test_virtual_grids_p2_exact(stf, p, q, variant):
     """Distributed plans (2D block-cyclic and the 1D column block-cyclic 1x8 grid
     of cuSolverMg) with COPY tasks or fused pushes, eager or graph,
@@ -241,6 +242,7 @@ def test_virtual_grids_p2_exact(stf, p, q, variant):
     assert np.array_equal(L, L0)
     assert st["slots"] == p * q and st["transfers"] > 0
     assert st["graph_fallback"] == 0 and st["graph"] == (0 if variant.get("graph") == 0 else 1)
+    # push=2 (multicast) needs distinct devices: on virtual slots it keeps the peer stores of push=1
     assert st["data_plane"] == (1 if variant.get("push") else 0)
     assert (st["pushed"] > 0) == bool(variant.get("push"))
 
