@@ -57,6 +57,7 @@ const std::vector<OptDesc>& option_table() {
       {"host_stream", "STF_HOST_STREAM", &Options::host_stream, 0, 1, true},
       {"trsm_res_tail", "STF_TRSM_RES_TAIL", &Options::trsm_res_tail, 0, INT64_MAX, true},
       {"trsm_rows", "STF_TRSM_ROWS", &Options::trsm_rows, 32, 128, true},
+      {"trsm_res_split", "STF_TRSM_RES_SPLIT", &Options::trsm_res_split, 1, 2, true},
       {"order_mode", "STF_ORDER_MODE", &Options::order_mode, -1, 2, true},
       {"order_tail", "STF_ORDER_TAIL", &Options::order_tail, -1, INT64_MAX, true},
       {"order_asap", "STF_ORDER_ASAP", &Options::order_asap, 0, 1, true},

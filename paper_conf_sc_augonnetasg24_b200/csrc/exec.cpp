@@ -208,7 +208,8 @@ struct Lowerer {
           // the next panel's TRSM(k+1,k) is on the critical path, and near the end of the
           // factorisation every TRSM is latency-bound: the resident-panel kernel (16 rows per
           // CTA, 4x the CTAs of the row panel, solve overlapped with the updates)
-          CUDA_TRY(stfk::trsm_res(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, &mir),
+          CUDA_TRY(stfk::trsm_res_parts(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb,
+                                        &mir, (int)X.opt.trsm_res_split),
                    "TRSM launch");
         } else if (X.opt.trsm >= 2 && t.i == t.k + 1) {
           // the next panel's TRSM(k+1,k) is on the critical path: one low-latency launch

@@ -68,7 +68,8 @@ int stf_kernel_trsm(int64_t M, int64_t n, const double* L, int64_t ldl, double* 
   if (r) return r;
   const int64_t trsm = ctx().opt.trsm;
   if (trsm == 3 && stfk::trsm_res_supported((int)n, L, ldl)) {
-    CUDA_TRY(stfk::trsm_res(0, 0, (int)M, (int)n, L, ldl, B, ldb), "trsm (resident panel)");
+    CUDA_TRY(stfk::trsm_res_parts(0, 0, (int)M, (int)n, L, ldl, B, ldb, nullptr, (int)ctx().opt.trsm_res_split),
+             "trsm (resident panel)");
     CUDA_TRY(cudaStreamSynchronize(0), "trsm sync");
     return 0;
   }
@@ -160,7 +161,8 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
         case 0: step(stfk::gemm_nt(s, 0, (int)M, (int)N, (int)K, A, ldm, B, ldn, Cm, ldm, 0)); break;
         case 1: step(stfk::gemm_nt(s, 0, (int)M, (int)M, (int)K, A, ldm, A, ldm, Cm, ldm, 1)); break;
         case 2:
-          step(trsm == 3 && stfk::trsm_res_supported((int)N, Src, ldm) ? stfk::trsm_res(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)
+          step(trsm == 3 && stfk::trsm_res_supported((int)N, Src, ldm)
+                   ? stfk::trsm_res_parts(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm, nullptr, (int)ctx().opt.trsm_res_split)
                : trsm >= 2 ? stfk::trsm_panel(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm)
                : trsm == 1 ? stfk::trsm_tile(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm, ws)
                            : stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm));

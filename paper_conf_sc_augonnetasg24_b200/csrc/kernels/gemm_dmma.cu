@@ -293,6 +293,11 @@ static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tm
 
 cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
                     const double* B, int64_t ldb, double* C, int64_t ldc, int lower) {
+  return gemm_nt_tiles(stream, prio, M, N, K, A, lda, B, ldb, C, ldc, lower, 0);
+}
+
+cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
+                          const double* B, int64_t ldb, double* C, int64_t ldc, int lower, int small) {
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
     return cudaErrorMisalignedAddress;
@@ -308,9 +313,9 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   cfg.stream = stream;
-  if (lower && M <= syrk64_max() && bk == CfgS64::BK) {
+  if ((lower && M <= syrk64_max() && bk == CfgS64::BK) || (small && bk == CfgS64::BK)) {
     const int t64 = (M + 63) / 64;
-    cfg.gridDim = dim3(t64 * (t64 + 1) / 2, 1, 1);
+    cfg.gridDim = lower ? dim3(t64 * (t64 + 1) / 2, 1, 1) : dim3(t64, (N + 63) / 64, 1);
     cfg.blockDim = dim3(128, 1, 1);
     cfg.dynamicSmemBytes = CfgS64::SMEM_BYTES;
     ++launch_count();

@@ -18,6 +18,10 @@ namespace stfk {
 // lda, ldb even (TMA global strides are multiples of 16 bytes).
 cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
                     const double* B, int64_t ldb, double* C, int64_t ldc, int lower);
+// Same with small != 0: 64 x 64 CTA tiles (twice the CTAs of the default 128 x 64;
+// latency-critical updates; same per-element k order, same bits).
+cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
+                          const double* B, int64_t ldb, double* C, int64_t ldc, int lower, int small);
 
 // K3: B[M x n] <- B * L^-T with L[n x n] lower triangular, non-unit diagonal
 // (side = right, lower, transposed).  Recursive: base blocks of <= 64 columns
@@ -70,6 +74,8 @@ cudaError_t dataflow_prepare(int m, int n, bool potrf);
 // and solver warps (substitution) overlap.  Requires trsm_res_supported(n, L, ldl):
 // 64 <= n <= 1024, n % 64 == 0, ldl even, L 16-byte aligned.
 bool trsm_res_supported(int n, const double* L, int64_t ldl);
+cudaError_t trsm_res_parts(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                           int64_t ldb, const Mirrors* mirrors, int parts);
 cudaError_t trsm_res(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                      int64_t ldb, const Mirrors* mirrors = nullptr, unsigned long long* trace = nullptr);
 

@@ -311,6 +311,27 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
 
 bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld, int bk);
 
+// Resident-panel TRSM in `parts` (1 or 2) column parts, right-looking: X1 = B1 L11^-T;
+// B2 -= X1 L21^T (GEMM on 64 x 64 CTA tiles: the whole GPU); X2 = B2 L22^-T.  The
+// substitution runs on half-width panels and the middle quarter of the flops at
+// GEMM rate: the critical TRSM(k+1,k) at nb = 1024 spreads beyond 64 SMs.
+cudaError_t trsm_res_parts(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
+                           int64_t ldb, const Mirrors* mirrors, int parts) {
+  const int h = n / 2;
+  if (parts < 2 || n % 128 || !trsm_res_supported(h, L, ldl) || (ldb & 1) || (reinterpret_cast<uintptr_t>(B) & 15))
+    return trsm_res(stream, prio, M, n, L, ldl, B, ldb, mirrors);
+  Mirrors m1{}, m2{};
+  if (mirrors) {
+    m1 = *mirrors;
+    m2 = *mirrors;
+    for (int m = 0; m < m2.n && m < 7; ++m) m2.p[m] = mirrors->p[m] + (int64_t)h * ldb;
+  }
+  cudaError_t e = trsm_res(stream, prio, M, h, L, ldl, B, ldb, &m1);
+  if (e == cudaSuccess) e = gemm_nt_tiles(stream, prio, M, n - h, h, B, ldb, L + h, ldl, B + (int64_t)h * ldb, ldb, 0, 1);
+  if (e == cudaSuccess) e = trsm_res(stream, prio, M, n - h, L + (int64_t)h * ldl + h, ldl, B + (int64_t)h * ldb, ldb, &m2);
+  return e;
+}
+
 bool trsm_res_supported(int n, const double* L, int64_t ldl) {
   return n >= tr::W && n <= tr::NMAX && n % tr::W == 0 && (ldl & 1) == 0 &&
          (reinterpret_cast<uintptr_t>(L) & 15) == 0;
