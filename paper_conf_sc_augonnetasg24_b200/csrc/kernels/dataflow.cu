@@ -814,16 +814,18 @@ cudaError_t get_table(int mode, int Mb, int Nb, const uint32_t** out, int* count
   return cudaSuccess;
 }
 
-// CTAs of a dataflow POTRF launch: STF_DF_CTAS, else 2 per 64-block column
+// CTAs of a dataflow POTRF launch: STF_DF_CTAS, else 3 per 64-block column
 // (16 .. 96): the critical chain needs the bulk updates of the next columns
-// done in time (profiles: nb = 1024 0.69 -> 0.59 ms, nb = 2048 3.4 -> 1.3 ms).
+// done in time (profiles: nb = 1024 0.69 -> 0.59 ms, nb = 2048 3.4 -> 1.3 ms at 2
+// per column; with the look-ahead P of round 2 the chain waited for its S input
+// at 2 per column: 396 -> 375 us at 3, tools/potrf_trace.py).
 int df_max_ctas(int T = 16) {
   static int v = [] {
     const char* e = getenv("STF_DF_CTAS");
     return e ? atoi(e) : 0;
   }();
   if (v > 0) return v;
-  return std::min(96, std::max(16, 2 * T));
+  return std::min(96, std::max(16, 3 * T));
 }
 
 int num_sms() {
