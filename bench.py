@@ -260,6 +260,7 @@ def run_ours(args, rank, world):
         dist.barrier()
     clocks = ClockSampler()
     steps_ms = []
+    walls = []
     stats = None
     if rank == 0:
         clocks.start()
@@ -267,7 +268,9 @@ def run_ours(args, rank, world):
             M.fill_spd(1)  # untimed regeneration (input is overwritten by L)
             for d in set(devices):
                 torch.cuda.synchronize(d)
-            info = M.potrf()
+            t0 = time.perf_counter()
+            info = M.potrf()  # synchronous
+            walls.append(1e3 * (time.perf_counter() - t0))
             assert info == 0 or os.environ.get("STF_DEBUG_SKIP"), info
             stats = stf.last_stats()
             steps_ms.append(stats["device_ms"])
@@ -295,7 +298,7 @@ def run_ours(args, rank, world):
     del M
     torch.cuda.empty_cache()
     report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "single", args.steps * stats["kernel_launches"],
-           check)
+           check, walls)
     stf.finalize()
     if dist_on:
         dist.destroy_process_group()
@@ -318,14 +321,18 @@ def run_mp(args, rank, world, P, Q):
     dist.all_gather_object(blobs, blob)
     A.import_blobs(blobs)
 
+    walls = []
+
     def step():
         A.fill_spd(1)  # untimed regeneration of this rank's tiles
         torch.cuda.synchronize(dev)
         dist.barrier()
-        info = A.potrf()
+        t0 = time.perf_counter()
+        info = A.potrf()  # synchronous
         assert info == 0 or os.environ.get("STF_DEBUG_SKIP"), info
         ms = stf.last_stats()["device_ms"]
         dist.barrier()
+        walls.append(1e3 * (time.perf_counter() - t0))  # barrier to barrier (cross-check of the device time)
         return ms
 
     t0 = time.perf_counter()
@@ -336,7 +343,9 @@ def run_mp(args, rank, world, P, Q):
     clocks = ClockSampler()
     if rank == 0:
         clocks.start()
+    walls.clear()
     mine = [step() for _ in range(args.steps)]
+    wall_ms = [max_over_ranks(x, True) for x in walls]
     clk = clocks.stop() if rank == 0 else None
     stats = stf.last_stats()
     check = None
@@ -371,14 +380,14 @@ def run_mp(args, rank, world, P, Q):
         del A
         torch.cuda.empty_cache()
         report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, "mp", args.steps * int(launches.item()),
-               check)
+               check, wall_ms)
         stf.finalize()
     dist.barrier()
     dist.destroy_process_group()
     return 0
 
 
-def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, gpu_launches, check=None):
+def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, gpu_launches, check=None, wall_ms=None):
     import torch
 
     n, nb = args.n, args.nb
@@ -464,6 +473,7 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
         "check": check,
         "first_call_ms": round(first_ms, 1) if first_ms else None,
         "step_ms": [round(x, 3) for x in steps_ms],
+        "step_wall_ms": [round(x, 3) for x in wall_ms] if wall_ms else None,
     }
     print(json.dumps(line), flush=True)
 

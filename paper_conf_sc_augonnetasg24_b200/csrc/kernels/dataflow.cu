@@ -46,8 +46,8 @@ constexpr int W = 64;       // block order
 constexpr int LDO = 68;     // smem stride of DMMA operand blocks [k][row] (68 = 4 mod 16: conflict-free)
 constexpr int LDB = 65;     // smem stride of substitution / Cholesky blocks [row][col]
 constexpr int NT = 256;
-// critical CTA: D [W][LDB] + XS [W][LDO] + Rc [W] + 4 swizzled 16-row panels + Y [W]
-constexpr int SMEM_BYTES = (W * LDB + W * LDO + W + 4 * 16 * W + W) * 8;  // 103,168 B
+// critical CTA: D [W][LDB] + XS [W][LDO] + Rc [W] + 4 swizzled 16-row panels + 4 x Y [W] + a counter
+constexpr int SMEM_BYTES = (W * LDB + W * LDO + W + 4 * 16 * W + 4 * W) * 8 + 16;  // 104,720 B
 enum : uint32_t { T_P = 0, T_S = 1, T_U = 2 };
 
 __host__ __device__ inline uint32_t enc(uint32_t t, uint32_t i, uint32_t j, uint32_t k) {
@@ -424,6 +424,113 @@ __device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
   __syncthreads();
 }
 
+__device__ __forceinline__ int ld_volatile_s(const int* p) {
+  int v;
+  asm volatile("ld.volatile.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+
+// P of the critical chain by warps 0-3 only (group D), while warps 4-7 solve
+// S(kb+1, kb) against the panels as they become final (critical_chain).  Warp 0
+// factors each 8-column panel (as in chol_block), warps 1-3 apply it to the
+// trailing lower block on DMMA with the same one-panel look-ahead (named barriers
+// 1 / 2 over the 128 threads of the group); after panel p, *dpanel = p + 1
+// tells the S warps its columns are final.  Same operations per element as
+// chol_block: bit-identical.
+__device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info, int* dpanel) {
+  constexpr int LD = df::LDB, BAR_DONE = 1, BAR_NEXT = 2, GRP = 128;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
+  if (warp == 0) {
+    int bad = 0;
+#pragma unroll 1
+    for (int p = 0; p < 8; ++p) {
+      if (p > 0) bar_sync_id(BAR_NEXT, GRP);
+      const int c0 = 8 * p;
+      double dg[8][8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j <= i; ++j) dg[i][j] = D[(c0 + i) * LD + c0 + j];
+      const int r1 = lane, r2 = lane + 32;
+      const bool b1 = r1 >= c0 + 8, b2 = r2 >= c0 + 8;
+      double v1[8], v2[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
+        v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const double d = dg[i][i];
+        const bool ok = d > 0.0;
+        if (!ok && bad == 0) bad = c0 + i + 1;
+        const double sq = ok ? sqrt(d) : kNaN, y = 1.0 / sq;
+        dg[i][i] = sq;
+#pragma unroll
+        for (int r = i + 1; r < 8; ++r) dg[r][i] = div_by(dg[r][i], sq, y);
+#pragma unroll
+        for (int r = i + 1; r < 8; ++r)
+#pragma unroll
+          for (int c = i + 1; c <= r; ++c) dg[r][c] = fma(-dg[r][i], dg[c][i], dg[r][c]);
+        v1[i] = div_by(v1[i], sq, y);
+        v2[i] = div_by(v2[i], sq, y);
+#pragma unroll
+        for (int c = i + 1; c < 8; ++c) {
+          v1[c] = fma(-v1[i], dg[c][i], v1[c]);
+          v2[c] = fma(-v2[i], dg[c][i], v2[c]);
+        }
+      }
+      if (lane == 0) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j <= i; ++j) D[(c0 + i) * LD + c0 + j] = dg[i][j];
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        if (b1) D[r1 * LD + c0 + j] = v1[j];
+        if (b2) D[r2 * LD + c0 + j] = v2[j];
+      }
+      __syncwarp();
+      if (lane == 0) {  // panel p is final: the S warps may use it
+        __threadfence_block();
+        *reinterpret_cast<volatile int*>(dpanel) = p + 1;
+      }
+      bar_arrive_id(BAR_DONE, GRP);
+    }
+    if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
+  } else {
+    const int mw = warp - 1;  // 0..2
+    auto update = [&](int R, int Cb, int c0) {
+      double* rowp = D + (8 * R + g) * LD;
+      double* cp = rowp + 8 * Cb + 2 * t;
+      double acc0 = cp[0], acc1 = cp[1];
+#pragma unroll
+      for (int ks = 0; ks < 2; ++ks) {
+        const double a = rowp[c0 + 4 * ks + t];
+        const double b = negd(D[(8 * Cb + g) * LD + c0 + 4 * ks + t]);
+        dmma_8x8x4(acc0, acc1, a, b);
+      }
+      cp[0] = acc0;
+      cp[1] = acc1;
+    };
+#pragma unroll 1
+    for (int p = 0; p < 7; ++p) {
+      bar_sync_id(BAR_DONE, GRP);
+      const int c0 = 8 * p;
+      for (int R = p + 1; R < 8; ++R)
+        if ((R + 2 * (p + 1)) % 3 == mw) update(R, p + 1, c0);
+      bar_arrive_id(BAR_NEXT, GRP);
+      for (int Cb = p + 2; Cb < 8; ++Cb)
+        for (int R = Cb; R < 8; ++R)
+          if ((R + 2 * Cb) % 3 == mw) update(R, Cb, c0);
+    }
+    bar_sync_id(BAR_DONE, GRP);  // panel 7
+  }
+  bar_sync_id(4, GRP);  // every write of the group to D is done
+}
+
 // interleaved-column register blocks (chol_core layout): v[m] = G(r, 4m + q)
 __device__ __forceinline__ void load_il(double (&v)[16], const double* G, int64_t ldg, int rows, int nc, bool lower) {
   const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
@@ -521,6 +628,9 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
   double* Rc = XS + W * df::LDO;           // W
   double* Lc = XS;                         // 3 W: chol_core scratch (XS is dead during P)
   double* Dp = XS + 3 * W;                 // W + 2
+  double* Xp = Rc + W;                     // 4 x [16 x 64] swizzled panels of S(kb+1, kb)
+  double* Yc = Xp + 4 * 16 * W;            // 4 x W: per S-warp 1 / L_cc
+  int* dpanel = reinterpret_cast<int*>(Yc + 4 * W);  // panels of P(kb) final so far
   int* prog = p.ws + 2;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   const int wm0 = (warp & 1) * 32, wn0 = (warp >> 1) * 16;
@@ -530,78 +640,97 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
   for (int kb = 0; kb < T; ++kb) {
     const int nk = min(W, p.n - kb * W);
     double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
-    // ---- P(kb)
+    // ---- P(kb), and S(kb+1, kb) concurrently on the other four warps
     DF_STAMP(6 * kb + 0);
+    const int ib = kb + 1, rows = ib < T ? min(W, p.n - ib * W) : 0;
+    double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
     if (nk == W) {
       if (kb == 0) {  // P(0) input: nothing precedes it
         for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
           const int rr = idx & (W - 1), cc = idx >> 6;
           if (rr >= cc) D[rr * df::LDB + cc] = __ldcg(Xkk + (int64_t)cc * p.ldx + rr);
         }
-        __syncthreads();
       }
-      chol_block(D, p.col0 + (int64_t)kb * W, p.info);
-    } else {
-      chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
-    }
-    store_block_rm(D, df::LDB, Xkk, p.ldx, nk, nk, true);
-    for (int m = 0; m < p.mir.n; ++m)
-      mirror_block_rm(D, df::LDB, p.mir.p[m] + (Xkk - p.X), p.ldx, nk, nk, true, p.mir.mc);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      st_release(&prog[kb * p.Nb + kb], kb + 1);
-    }
-    DF_STAMP(6 * kb + 1);
-    if (kb + 1 == T) return;
-    // ---- S(ib, kb), ib = kb + 1, with L_kk from D
-    const int ib = kb + 1, rows = min(W, p.n - ib * W);
-    double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
-    if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + kb], kb);
-    __syncthreads();
-    DF_STAMP(6 * kb + 2);
-    if (nk == W) {
-      // four warps, one per SM sub-partition, each solve 16 rows (solve_block: 8-column
-      // sub-blocks by substitution, their updates on DMMA; the FP64 pipes of the
-      // sub-partitions work in parallel), then the result goes to XS for U
-      double* Xp = Rc + W;        // 4 x [16 x 64] swizzled panels
-      double* Yc = Xp + 4 * 16 * W;  // 1 / L_cc (IEEE)
-      for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
-        const int rr = idx & (W - 1), cc = idx >> 6;
-        Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)] = rr < rows ? __ldcg(Xik + (int64_t)cc * p.ldx + rr) : 0.0;
-      }
-      if (threadIdx.x < W) Yc[threadIdx.x] = 1.0 / D[threadIdx.x * df::LDB + threadIdx.x];
+      if (threadIdx.x == 0) *dpanel = 0;
       __syncthreads();
-      if (warp < 4) {
-        const int rr = 16 * warp + (lane & 15);
-        solve_block<0>(Xp + warp * 16 * W, 0, sb::RowMajor<df::LDB>{D}, Yc, lane, Xik, p.ldx, rr,
-                       lane < 16 && rr < rows);
+      if (warp < 4) {  // ---- group D: P(kb), then L_kk to global and published
+        chol_block_grp(D, p.col0 + (int64_t)kb * W, p.info, dpanel);
+        for (int idx = threadIdx.x; idx < W * W; idx += 128) {
+          const int rr = idx & (W - 1), cc = idx >> 6;
+          if (rr >= cc) Xkk[(int64_t)cc * p.ldx + rr] = D[rr * df::LDB + cc];
+        }
+        for (int m = 0; m < p.mir.n; ++m) {
+          for (int idx = threadIdx.x; idx < W * W; idx += 128) {
+            const int rr = idx & (W - 1), cc = idx >> 6;
+            if (rr >= cc) mirror_st(p.mir.p[m] + (Xkk - p.X) + (int64_t)cc * p.ldx + rr, D[rr * df::LDB + cc], p.mir.mc);
+          }
+          mirror_fence(p.mir.mc);
+        }
+        bar_sync_id(4, 128);
+        if (threadIdx.x == 0) {
+          __threadfence();
+          st_release(&prog[kb * p.Nb + kb], kb + 1);
+        }
+        DF_STAMP(6 * kb + 1);
+      } else if (rows > 0) {  // ---- group S: X(kb+1, kb) <- X L_kk^-T, panel by panel as P finishes them
+        const int tid = threadIdx.x - 128, sw = warp - 4;
+        if (tid == 0) {
+          wait_geq(&prog[ib * p.Nb + kb], kb);  // all updates U(kb+1, kb, k'), k' < kb, done
+          if (p.trace) p.trace[6 * kb + 2] = gtime();
+        }
+        bar_sync_id(3, 128);
+        for (int idx = tid; idx < W * W; idx += 128) {
+          const int rr = idx & (W - 1), cc = idx >> 6;
+          Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)] = rr < rows ? __ldcg(Xik + (int64_t)cc * p.ldx + rr) : 0.0;
+        }
+        bar_sync_id(3, 128);
+        double* Yw = Yc + sw * W;  // this warp's copy of 1 / L_cc (IEEE)
+        auto gate = [&](int P) {   // sub-block P needs panel P of L_kk final
+          while (ld_volatile_s(dpanel) <= P) {
+          }
+          __threadfence_block();
+          if (lane < 8) Yw[8 * P + lane] = 1.0 / D[(8 * P + lane) * df::LDB + 8 * P + lane];
+          __syncwarp();
+        };
+        const int rr = 16 * sw + (lane & 15);
+        solve_block<0>(Xp + sw * 16 * W, 0, sb::RowMajor<df::LDB>{D}, Yw, lane, Xik, p.ldx, rr, lane < 16 && rr < rows,
+                       gate);
+        __syncwarp();
+        for (int m = 0; m < p.mir.n; ++m) {  // fused push of the finished block
+          if (lane < 16 && rr < rows)
+            for (int c = 0; c < W; ++c)
+              mirror_st(p.mir.p[m] + (Xik - p.X) + (int64_t)c * p.ldx + rr, Xp[sw * 16 * W + sb::xo(lane & 15, c)],
+                        p.mir.mc);
+          mirror_fence(p.mir.mc);
+        }
+        bar_sync_id(3, 128);
+        if (tid == 0) {
+          __threadfence();
+          st_release(&prog[ib * p.Nb + kb], kb + 1);
+          if (p.trace) p.trace[6 * kb + 3] = gtime();
+        }
       }
       __syncthreads();
-      for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+      if (kb + 1 == T) return;
+      for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {  // X for U's operands
         const int m = idx >> 6, k = idx & (W - 1);
         XS[m * df::LDO + k] = Xp[(m >> 4) * 16 * W + sb::xo(m & 15, k)];
       }
       __syncthreads();
-      for (int mm = 0; mm < p.mir.n; ++mm)  // fused push of the finished block (solve_block wrote the home tile)
-        for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
-          const int k = idx >> 6, m = idx & (W - 1);
-          if (m < rows) mirror_st(p.mir.p[mm] + (Xik - p.X) + (int64_t)k * p.ldx + m, XS[m * df::LDO + k], p.mir.mc);
-        }
-      if (p.mir.n) mirror_fence(p.mir.mc);
     } else {
-      double b[16];
-      load_chunk(b, Xik, p.ldx, rows, nk, false);
-      solve_core(b, D, Rc, XS, df::LDO, nk);
-      store_chunk(b, Xik, p.ldx, rows, nk, false);
-      for (int m = 0; m < p.mir.n; ++m) store_chunk_m(b, p.mir.p[m] + (Xik - p.X), p.ldx, rows, nk, p.mir.mc);
+      // ragged last block (n % 64 != 0): the register-resident Cholesky core
+      chol_core(a, D, Lc, Dp, nk, p.col0 + (int64_t)kb * W, p.info);
+      store_block_rm(D, df::LDB, Xkk, p.ldx, nk, nk, true);
+      for (int m = 0; m < p.mir.n; ++m)
+        mirror_block_rm(D, df::LDB, p.mir.p[m] + (Xkk - p.X), p.ldx, nk, nk, true, p.mir.mc);
       __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence();
+        st_release(&prog[kb * p.Nb + kb], kb + 1);
+      }
+      DF_STAMP(6 * kb + 1);
+      return;  // a ragged block is the last one
     }
-    if (threadIdx.x == 0) {
-      __threadfence();
-      st_release(&prog[ib * p.Nb + kb], kb + 1);
-    }
-    DF_STAMP(6 * kb + 3);
     // ---- U(ib, ib, kb): D <- lower(C - X X^T), C = block (ib, ib) after all earlier updates
     if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + ib], kb);
     __syncthreads();

@@ -40,10 +40,17 @@ struct RowMajor {  // p[r * LD + c]
 // Every sum keeps a fixed order; results are deterministic.
 using sb::xo;
 
-template <int P, class DA>
+struct NoHook {
+  __device__ __forceinline__ void operator()(int) const {}
+};
+
+// hook(P) runs at the start of sub-block P (e.g. waiting until the diagonal
+// block's columns 8P..8P+7 are final and staging their reciprocals in Y)
+template <int P, class DA, class Hook = NoHook>
 __device__ __forceinline__ void solve_block(double* Xs, int c0, DA D, const double* Y, int lane,
-                                            double* X, int64_t ldx, int64_t xrow, bool wr) {
+                                            double* X, int64_t ldx, int64_t xrow, bool wr, const Hook& hook = Hook()) {
   if constexpr (P < 8) {
+    hook(P);
     const int r = lane & 15;
     const int cb = c0 + 8 * P;
     // (a) serial substitution of the 8 columns of sub-block P
@@ -103,7 +110,7 @@ __device__ __forceinline__ void solve_block(double* Xs, int c0, DA D, const doub
         }
       __syncwarp();
     }
-    solve_block<P + 1>(Xs, c0, D, Y, lane, X, ldx, xrow, wr);
+    solve_block<P + 1>(Xs, c0, D, Y, lane, X, ldx, xrow, wr, hook);
   }
 }
 

@@ -27,18 +27,17 @@ bulk = t[6 * T:].reshape(-1, 3)
 bulk = bulk[bulk[:, 0] > 0]
 t0 = min(chain[0, 0], bulk[:, 0].min() if len(bulk) else chain[0, 0])
 print("n=%d ctas=%d total %.1f us, bulk tasks %d" % (n, ctas, (max(chain.max(), bulk.max() if len(bulk) else 0) - t0) / 1e3, len(bulk)))
-print("step  P_us  S_wait_us  S_us  U_wait_us  U_us  (chain, from P start)")
+print("step  P_us  S_in_ready  S_done  U_wait_us  U_us   (chain CTA; times from the step's P start; P and S overlap)")
 for kb in range(T):
-    c = chain[kb] - t0
+    c = chain[kb]
     if c[1] <= 0:
         continue
-    pu = (chain[kb, 1] - chain[kb, 0]) / 1e3
+    f = lambda e: (c[e] - c[0]) / 1e3 if c[e] > 0 else float("nan")
     if kb + 1 < T:
-        print("%3d %6.1f %9.1f %6.1f %9.1f %6.1f" % (kb, pu, (chain[kb, 2] - chain[kb, 1]) / 1e3,
-              (chain[kb, 3] - chain[kb, 2]) / 1e3, (chain[kb, 4] - chain[kb, 3]) / 1e3,
-              (chain[kb, 5] - chain[kb, 4]) / 1e3))
+        print("%3d %6.1f %10.1f %7.1f %9.1f %6.1f" % (kb, f(1), f(2), f(3), (c[4] - max(c[1], c[3])) / 1e3,
+                                                   (c[5] - c[4]) / 1e3))
     else:
-        print("%3d %6.1f" % (kb, pu))
+        print("%3d %6.1f" % (kb, f(1)))
 if len(bulk):
     w = (bulk[:, 1] - bulk[:, 0]) / 1e3
     d = (bulk[:, 2] - bulk[:, 1]) / 1e3
