@@ -99,21 +99,37 @@ __device__ __forceinline__ void wait_geq(const int* p, int v) {
   }
 }
 
+// Block loads: all W*W/NT = 16 loads of a thread are issued before any store, so
+// the L2 latency is paid once per block, not once per element row (a loop that
+// alternates load and smem store serialises them: 6.8 -> ~3 us per U task).
+constexpr int kPerThread = df::W * df::W / df::NT;
 // smem S[c * ld + r] = G(r0 + r, c0 + c) for r < rows, c < cols; zero elsewhere (W x W)
 __device__ __forceinline__ void load_block_cm(double* S, int ld, const double* G, int64_t ldg, int rows, int cols) {
-  for (int idx = threadIdx.x; idx < df::W * df::W; idx += df::NT) {
-    const int r = idx & (df::W - 1), c = idx >> 6;
-    S[c * ld + r] = (r < rows && c < cols) ? __ldcg(G + (int64_t)c * ldg + r) : 0.0;
+  double v[kPerThread];
+#pragma unroll
+  for (int u = 0; u < kPerThread; ++u) {
+    const int idx = threadIdx.x + u * df::NT, r = idx & (df::W - 1), c = idx >> 6;
+    v[u] = (r < rows && c < cols) ? __ldcg(G + (int64_t)c * ldg + r) : 0.0;
+  }
+#pragma unroll
+  for (int u = 0; u < kPerThread; ++u) {
+    const int idx = threadIdx.x + u * df::NT, r = idx & (df::W - 1), c = idx >> 6;
+    S[c * ld + r] = v[u];
   }
 }
 // smem S[r * ld + c] = G(r, c)  (row-major in smem)
 __device__ __forceinline__ void load_block_rm(double* S, int ld, const double* G, int64_t ldg, int rows, int cols,
                                               bool lower_only) {
-  for (int idx = threadIdx.x; idx < df::W * df::W; idx += df::NT) {
-    const int r = idx & (df::W - 1), c = idx >> 6;
-    double v = 0.0;
-    if (r < rows && c < cols && (!lower_only || r >= c)) v = __ldcg(G + (int64_t)c * ldg + r);
-    S[r * ld + c] = v;
+  double v[kPerThread];
+#pragma unroll
+  for (int u = 0; u < kPerThread; ++u) {
+    const int idx = threadIdx.x + u * df::NT, r = idx & (df::W - 1), c = idx >> 6;
+    v[u] = (r < rows && c < cols && (!lower_only || r >= c)) ? __ldcg(G + (int64_t)c * ldg + r) : 0.0;
+  }
+#pragma unroll
+  for (int u = 0; u < kPerThread; ++u) {
+    const int idx = threadIdx.x + u * df::NT, r = idx & (df::W - 1), c = idx >> 6;
+    S[r * ld + c] = v[u];
   }
 }
 __device__ __forceinline__ void store_block_rm(const double* S, int ld, double* G, int64_t ldg, int rows, int cols,
@@ -645,12 +661,7 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
     const int ib = kb + 1, rows = ib < T ? min(W, p.n - ib * W) : 0;
     double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
     if (nk == W) {
-      if (kb == 0) {  // P(0) input: nothing precedes it
-        for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
-          const int rr = idx & (W - 1), cc = idx >> 6;
-          if (rr >= cc) D[rr * df::LDB + cc] = __ldcg(Xkk + (int64_t)cc * p.ldx + rr);
-        }
-      }
+      if (kb == 0) load_block_rm(D, df::LDB, Xkk, p.ldx, W, W, true);  // P(0) input: nothing precedes it
       if (threadIdx.x == 0) *dpanel = 0;
       __syncthreads();
       if (warp < 4) {  // ---- group D: P(kb), then L_kk to global and published
@@ -679,15 +690,24 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
           if (p.trace) p.trace[6 * kb + 2] = gtime();
         }
         bar_sync_id(3, 128);
-        for (int idx = tid; idx < W * W; idx += 128) {
-          const int rr = idx & (W - 1), cc = idx >> 6;
-          Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)] = rr < rows ? __ldcg(Xik + (int64_t)cc * p.ldx + rr) : 0.0;
+#pragma unroll 1
+        for (int h = 0; h < 2; ++h) {  // 2 x 16 loads in flight per thread
+          double v[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) {
+            const int idx = tid + (16 * h + u) * 128, rr = idx & (W - 1), cc = idx >> 6;
+            v[u] = rr < rows ? __ldcg(Xik + (int64_t)cc * p.ldx + rr) : 0.0;
+          }
+#pragma unroll
+          for (int u = 0; u < 16; ++u) {
+            const int idx = tid + (16 * h + u) * 128, rr = idx & (W - 1), cc = idx >> 6;
+            Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)] = v[u];
+          }
         }
         bar_sync_id(3, 128);
         double* Yw = Yc + sw * W;  // this warp's copy of 1 / L_cc (IEEE)
         auto gate = [&](int P) {   // sub-block P needs panel P of L_kk final
-          while (ld_volatile_s(dpanel) <= P) {
-          }
+          while (ld_volatile_s(dpanel) <= P) __nanosleep(40);  // keep the issue slots for the P warps
           __threadfence_block();
           if (lane < 8) Yw[8 * P + lane] = 1.0 / D[(8 * P + lane) * df::LDB + 8 * P + lane];
           __syncwarp();
@@ -890,13 +910,20 @@ std::vector<uint32_t> build_tasks(bool potrf, int Mb, int Nb, bool crit) {
     t.push_back(enc(df::T_P, 0, 0, 0));
     for (int i = 1; i < T; ++i) t.push_back(enc(df::T_S, i, 0, 0));
     for (int i = 1; i < T; ++i) t.push_back(enc(df::T_U, i, 1, 0));
+    // per step: P(kb+1) and its solves; then the column kb+2 -- the next panel's
+    // inputs -- first receives the update from column kb and then from column kb+1
+    // (the look-ahead), ahead of the bulk updates of the columns behind it; every
+    // block still sees its updates in increasing k, so a task only waits on
+    // smaller tickets (deadlock-free)
     for (int kb = 0; kb + 1 < T; ++kb) {
       t.push_back(enc(df::T_P, kb + 1, kb + 1, kb + 1));
       for (int i = kb + 2; i < T; ++i) t.push_back(enc(df::T_S, i, kb + 1, kb + 1));
-      for (int j = kb + 2; j < T; ++j)
-        for (int i = j; i < T; ++i) t.push_back(enc(df::T_U, i, j, kb));
-      if (kb + 2 < T)
+      if (kb + 2 < T) {
+        for (int i = kb + 2; i < T; ++i) t.push_back(enc(df::T_U, i, kb + 2, kb));
         for (int i = kb + 2; i < T; ++i) t.push_back(enc(df::T_U, i, kb + 2, kb + 1));
+      }
+      for (int j = kb + 3; j < T; ++j)
+        for (int i = j; i < T; ++i) t.push_back(enc(df::T_U, i, j, kb));
     }
   } else {
     for (int i = 0; i < Mb; ++i) t.push_back(enc(df::T_S, i, 0, 0));

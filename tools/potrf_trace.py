@@ -43,3 +43,35 @@ if len(bulk):
     d = (bulk[:, 2] - bulk[:, 1]) / 1e3
     print("bulk: wait mean %.1f us (max %.1f), run mean %.1f us (max %.1f), busy sum %.1f us" % (
         w.mean(), w.max(), d.mean(), d.max(), d.sum()))
+
+# ---- the bulk tasks that feed the chain's S input X(kb+1, kb): S(kb+1, kb-1) and U(kb+1, kb, kb-1)
+def tasks_order(T):  # replica of dataflow.cu build_tasks(potrf, crit) ticket order
+    t = [("P", 0, 0, 0)] + [("S", i, 0, 0) for i in range(1, T)] + [("U", i, 1, 0) for i in range(1, T)]
+    for kb in range(T - 1):
+        t.append(("P", kb + 1, kb + 1, kb + 1))
+        t += [("S", i, kb + 1, kb + 1) for i in range(kb + 2, T)]
+        if kb + 2 < T:
+            t += [("U", i, kb + 2, kb) for i in range(kb + 2, T)]
+            t += [("U", i, kb + 2, kb + 1) for i in range(kb + 2, T)]
+        t += [("U", i, j, kb) for j in range(kb + 3, T) for i in range(j, T)]
+
+    def chain(x):
+        ty, i, j, k = x
+        return ty == "P" or (ty == "S" and i == k + 1) or (ty == "U" and i == k + 1 and j == k + 1)
+    return [x for x in t if not chain(x)]
+
+
+order = tasks_order(T)
+raw = t[6 * T:].reshape(-1, 3)
+pos = {x: n for n, x in enumerate(order)}
+print("feeders of X(kb+1,kb) (us from the chain's P(kb-1) start): S(kb+1,kb-1) claim/ready/done, "
+      "U(kb+1,kb,kb-1) claim/ready/done; chain S(kb,kb-1) done")
+for kb in range(2, T - 1):
+    s0 = chain[kb - 1, 0]
+    a = pos.get(("S", kb + 1, kb - 1, kb - 1))
+    b = pos.get(("U", kb + 1, kb, kb - 1))
+    f = lambda x: "%6.1f" % ((x - s0) / 1e3) if x > 0 else "   nan"
+    if a is None or b is None or a >= len(raw) or b >= len(raw):
+        continue
+    print("%3d  S: %s %s %s   U: %s %s %s   chainS: %s" % (kb, f(raw[a, 0]), f(raw[a, 1]), f(raw[a, 2]),
+                                                       f(raw[b, 0]), f(raw[b, 1]), f(raw[b, 2]), f(chain[kb - 1, 3])))
