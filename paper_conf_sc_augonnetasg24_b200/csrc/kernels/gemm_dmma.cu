@@ -273,6 +273,11 @@ static int gemm_narrow() {
   return v;
 }
 
+// warps of the 64 x 64 CTA tile: 4 (32 x 32 each) or 8 (32 x 16; STF_S64_WARPS)
+static int s64_warps() {
+  static int v = env_or("STF_S64_WARPS", 8) == 4 ? 4 : 8;
+  return v;
+}
 // SYRK (lower) tiles up to this order use the 64 x 64 CTA tile (STF_SYRK64_MAX, default 1024)
 static int syrk64_max() {
   static int v = env_or("STF_SYRK64_MAX", 1024);
@@ -316,9 +321,13 @@ cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, co
   if ((lower && M <= syrk64_max() && bk == CfgS64::BK) || (small && bk == CfgS64::BK)) {
     const int t64 = (M + 63) / 64;
     cfg.gridDim = lower ? dim3(t64 * (t64 + 1) / 2, 1, 1) : dim3(t64, (N + 63) / 64, 1);
-    cfg.blockDim = dim3(128, 1, 1);
     cfg.dynamicSmemBytes = CfgS64::SMEM_BYTES;
     ++launch_count();
+    if (s64_warps() == 8) {  // 32 x 16 warp tiles: two warps per SM sub-partition
+      cfg.blockDim = dim3(256, 1, 1);
+      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 16, CfgS64>, tmA, tmB, C, ldc, M, N, K, lower);
+    }
+    cfg.blockDim = dim3(128, 1, 1);
     return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgS64>, tmA, tmB, C, ldc, M, N, K, lower);
   }
   const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
@@ -358,6 +367,9 @@ cudaError_t gemm_init_attrs() {
                              CfgN64::SMEM_BYTES);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 32, CfgS64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             CfgS64::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(gemm_nt_dmma_kernel<32, 16, CfgS64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              CfgS64::SMEM_BYTES);
   return e;
 }
