@@ -87,8 +87,33 @@ def test_init_without_gpu_fails_cleanly():
 
 
 OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (3, 1), "streams": (32, 3), "serial": (0, 1),
-           "priority": (1, 0), "grid_p": (0, 2), "lookahead": (1, 0), "threads": (8, 2), "trsm_split": (4, 2), "push": (0, 1),
-           "trsm_res_tail": (8192, 0), "trsm_rows": (128, 64)}
+           "priority": (1, 0), "grid_p": (0, 2), "lookahead": (1, 0), "threads": (8, 2), "trsm_split": (4, 2), "push": (0, 2),
+           "trsm_res_tail": (8192, 0), "trsm_rows": (128, 64), "trsm_res_split": (2, 1), "stream_pool": (0, 1),
+           "order_mode": (-1, 2), "order_tail": (-1, 0), "order_asap": (0, 1), "sched_width": (0, 3), "prio_mode": (0, 2),
+           "ooc_reorder": (1, 0), "dev_order": (0, 1), "ooc_budget_pct": (-1, 40), "host_stream_budget_pct": (90, 75),
+           "host_eager": (0, 1), "mem_cap_tiles": (0, 10), "ooc_order": (-1, 0), "host_stream": (1, 0), "pdl": (0, 1),
+           "debug_skip": (0, 8), "debug_trace": (0, 1)}
+
+
+@pytest.mark.parametrize("name,value", [("trsm_rows", 48), ("mem_cap_tiles", 2), ("push", 3), ("order_mode", 1),
+                                        ("stream_pool", 3), ("ooc_budget_pct", 5), ("streams", 0)])
+def test_options_reject_out_of_range(name, value):
+    before = stf.get_option(name)
+    with pytest.raises(stf.StfError):
+        stf.set_option(name, value)
+    assert stf.get_option(name) == before
+
+
+def test_environment_options_are_validated_at_init(tmp_path):
+    """An out-of-range STF_<NAME> is rejected at stf_cholesky_init (-105) before any
+    device work (in a GPU-less process the device probe fails first: -101)."""
+    import subprocess
+    import sys
+    code = ("import ctypes, sys; sys.path.insert(0, %r); from paper_conf_sc_augonnetasg24_b200 import _abi; "
+            "print(_abi.stf_cholesky_init(1, None))" % ROOT)
+    env = dict(os.environ, STF_MEM_CAP_TILES="2")
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, timeout=120)
+    assert r.stdout.strip() in ("-105", "-101"), r.stdout + r.stderr
 
 
 def test_options_roundtrip_without_gpu():

@@ -47,3 +47,25 @@ def test_multiprocess_p2_exact(p, q, push, port):
 @pytest.mark.gpu
 def test_multiprocess_large_tile():
     print(_run(2048, 512, 2, 2, push=1, reps=2, port=29651))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", ["mp", "single"])
+def test_bench_two_ranks_virtual_slots(mode):
+    """bench.py under torchrun with 2 ranks (both on cuda:0): the N > 1 line carries
+    the plan statistics and the on-box P2 check (every tile bit-exact)."""
+    import json
+
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", "29721" if mode == "mp" else "29731",
+           os.path.join(ROOT, "bench.py"), "--gpus", "2", "--virtual-slots", "1", "--mode", mode,
+           "--n", "4096", "--nb", "512", "--steps", "2", "--warmup", "1", "--no-e2e", "--no-cpu"]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT)
+    assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-3000:]
+    lines = [json.loads(l) for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    d = lines[0]
+    assert d["n_gpus"] == 2 and d["config"]["grid"] == "1x2" and d["value"] > 0
+    assert d["check"]["bit_exact"] and d["check"]["tiles_checked"] == 36
+    assert d["plan"]["slots"] == 2 and d["plan"]["transfers"] > 0
+    assert d["step_wall_ms"] and len(d["step_ms"]) == 2
