@@ -171,6 +171,8 @@ const char *stf_last_error(void);
  *                           results invalid
  *   "debug_trace" STF_DEBUG_TRACE 1: timing events around every task (one slot), see
  *                           stf_debug_last_trace in stf_harness.h
+ *   "nvtx"     STF_NVTX     1: an NVTX range per task submission ("GEMM(i,j,k)@slot", eager
+ *                           backend) and one around each call's graph launch (profiler timelines)
  * Returns 0 or -105. */
 int stf_set_option(const char *name, int64_t value);
 int stf_get_option(const char *name, int64_t *value);

@@ -85,6 +85,20 @@ def dag_call(n: int, nb: int, kind: int = STF_DESC_TILED_2DBC, p: int = 1, q: in
     return edges, kinds, ijk, st.as_dict()
 
 
+def dag_dot(edges, kinds, ijk, path: str) -> None:
+    """Write the DAG of dag()/dag_call() as a Graphviz DOT file (one node per task,
+    labelled KIND(i,j,k); COPY nodes carry the destination slot as k)."""
+    col = {"POTRF": "red", "TRSM": "orange", "SYRK": "blue", "GEMM": "gray", "COPY": "green", "LOAD": "cyan",
+           "STORE": "cyan", "FENCE": "black"}
+    with open(path, "w") as f:
+        f.write("digraph stf {\n  node [shape=box, fontsize=9];\n")
+        for t, (k, (i, j, kk)) in enumerate(zip(kinds, ijk)):
+            f.write('  t%d [label="%s(%d,%d,%d)", color=%s];\n' % (t, k, i, j, kk, col.get(k, "black")))
+        for a, b in edges:
+            f.write("  t%d -> t%d;\n" % (a, b))
+        f.write("}\n")
+
+
 def dag_io(ntasks: int):
     """(buffers read, buffer written) of every task of the last dag() call, and
     the number of buffers (home tiles + replicas, or device frames out of core)."""

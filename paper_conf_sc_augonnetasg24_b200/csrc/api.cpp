@@ -72,6 +72,7 @@ const std::vector<OptDesc>& option_table() {
       {"pdl", "STF_PDL", &Options::pdl, 0, 1, true},
       {"debug_skip", "STF_DEBUG_SKIP", &Options::debug_skip, 0, INT64_MAX, true},
       {"debug_trace", "STF_DEBUG_TRACE", &Options::debug_trace, 0, 1, true},
+      {"nvtx", "STF_NVTX", &Options::nvtx, 0, 1, false},
   };
   return t;
 }

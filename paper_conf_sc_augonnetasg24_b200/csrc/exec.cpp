@@ -9,6 +9,8 @@
 #include <cstdlib>
 #include <thread>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "runtime_internal.hpp"
 
 namespace stfrt {
@@ -396,7 +398,15 @@ struct Lowerer {
       }
       // debug timeline: timing events (external record nodes when captured), no SM work
       if (!X.trace.empty()) CUDA_TRY(trace_record(X.trace[2 * t], s), "trace");
+      const bool nv = X.opt.nvtx && !X.opt.graph;  // one NVTX range per task submission (eager)
+      if (nv) {
+        static const char* kn[] = {"POTRF", "TRSM", "SYRK", "GEMM", "COPY", "LOAD", "STORE", "FENCE"};
+        char name[64];
+        snprintf(name, sizeof name, "%s(%d,%d,%d)@%d", kn[task.kind & 7], task.i, task.j, task.k, task.slot);
+        nvtxRangePushA(name);
+      }
       int r = body(task, t, s, prio_of(task));
+      if (nv) nvtxRangePop();
       if (r) return r;
       if (!X.trace.empty()) CUDA_TRY(trace_record(X.trace[2 * t + 1], s), "trace");
       if (X.mp) {  // publish remote replicas written by this task (COPY target, fused-push mirrors)
@@ -765,10 +775,14 @@ int run(Context& C, Exec& X) {
   }
   cudaSetDevice(C.origin_dev);
   CUDA_TRY(cudaEventRecord(C.t_start, C.origin), "timing start");
+  if (X.opt.nvtx) nvtxRangePushA(X.opt.graph ? "stf_potrf graph launch" : "stf_potrf eager submission");
   if (X.opt.graph) {
-    CUDA_TRY(cudaGraphLaunch(X.gexec, C.origin), "graph launch");
+    const cudaError_t ge = cudaGraphLaunch(X.gexec, C.origin);
+    if (X.opt.nvtx) nvtxRangePop();
+    CUDA_TRY(ge, "graph launch");
   } else {
     int r = issue_all(C, X);
+    if (X.opt.nvtx) nvtxRangePop();
     if (r) return r;
   }
   cudaSetDevice(C.origin_dev);

@@ -604,6 +604,48 @@ __device__ __forceinline__ void store_chunk_m(const double (&v)[16], double* G, 
 // the result also goes to the mirrors at element offset `off` (fused push).
 __device__ void task_solve(double* sm, double* X, int64_t ldx, const double* L, int64_t ldl, int rows, int nc,
                            const Mirrors* mir = nullptr, int64_t off = 0) {
+  if (nc == df::W) {
+    // full block: four warps (one per SM sub-partition) solve 16 rows each with
+    // solve_block (8-column sub-blocks by substitution, their updates on DMMA) --
+    // the form the critical chain uses, 8.8 -> ~6 us per task
+    constexpr int W = df::W;
+    double* Xp = sm;                  // 4 x [16 x 64] swizzled panels
+    double* D = Xp + 4 * 16 * W;      // L row-major [W][LDB], lower part
+    double* Yc = D + W * df::LDB;     // 1 / L_cc (IEEE)
+    {
+      double v[kPerThread];
+#pragma unroll
+      for (int u = 0; u < kPerThread; ++u) {
+        const int idx = threadIdx.x + u * df::NT, rr = idx & (W - 1), cc = idx >> 6;
+        v[u] = rr < rows ? __ldcg(X + (int64_t)cc * ldx + rr) : 0.0;
+      }
+#pragma unroll
+      for (int u = 0; u < kPerThread; ++u) {
+        const int idx = threadIdx.x + u * df::NT, rr = idx & (W - 1), cc = idx >> 6;
+        Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)] = v[u];
+      }
+    }
+    load_block_rm(D, df::LDB, L, ldl, W, W, true);
+    __syncthreads();
+    if (threadIdx.x < W) Yc[threadIdx.x] = 1.0 / D[threadIdx.x * df::LDB + threadIdx.x];
+    __syncthreads();
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (warp < 4) {
+      const int rr = 16 * warp + (lane & 15);
+      solve_block<0>(Xp + warp * 16 * W, 0, sb::RowMajor<df::LDB>{D}, Yc, lane, X, ldx, rr, lane < 16 && rr < rows);
+    }
+    if (mir && mir->n) {
+      __syncthreads();
+      for (int m = 0; m < mir->n; ++m) {
+        for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {
+          const int rr = idx & (W - 1), cc = idx >> 6;
+          if (rr < rows) mirror_st(mir->p[m] + off + (int64_t)cc * ldx + rr, Xp[(rr >> 4) * 16 * W + sb::xo(rr & 15, cc)], mir->mc);
+        }
+        mirror_fence(mir->mc);
+      }
+    }
+    return;
+  }
   double* Xs = sm;                    // publication buffer [r][LDB]
   double* Ls = sm + df::W * df::LDB;  // Ls[c][p]
   double* Rc = Ls + df::W * df::LDB;

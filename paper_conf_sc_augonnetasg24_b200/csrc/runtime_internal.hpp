@@ -84,6 +84,7 @@ struct Options {
   int64_t pdl = 0;             // programmatic dependent launch between same-stream chain kernels
   int64_t debug_skip = 0;      // bit mask of task kinds not launched (timing what-ifs; results invalid)
   int64_t debug_trace = 0;     // timing events around every task (one slot)
+  int64_t nvtx = 0;            // NVTX range per task submission (eager backend; the graph launch is one range)
 };
 
 struct OptDesc {

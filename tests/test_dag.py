@@ -178,3 +178,16 @@ def test_list_order_submits_the_panel_chain_early(options):
     e0, k0, ijk0, _ = stf.dag(T, 1, 1)
     pos0 = {(kd, *x): t for t, (kd, x) in enumerate(zip(k0, ijk0))}
     assert pos0[("POTRF", 1, 1, 1)] > pos0[("GEMM", T - 1, T - 2, 0)]
+
+
+def test_dag_dot_export(tmp_path):
+    """DOT export of the DAG (SURVEY §5 tracing): one node per task, one edge per
+    STF dependency, COPY nodes for the replica transfers of a distributed plan."""
+    edges, kinds, ijk, st = stf.dag(4, 1, 2)
+    path = tmp_path / "chol.dot"
+    stf.dag_dot(edges, kinds, ijk, str(path))
+    txt = path.read_text()
+    assert txt.startswith("digraph stf")
+    assert txt.count("->") == st["edges"] == len(edges)
+    assert txt.count("[label=") == st["dag_tasks"]
+    assert "COPY(" in txt and 'POTRF(0,0,0)' in txt
