@@ -395,6 +395,7 @@ __device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
           v2[c] = fma(-v2[i], dg[c][i], v2[c]);
         }
       }
+      __syncwarp();  // every lane has read the diagonal block before lane 0 overwrites it
       if (lane == 0) {
 #pragma unroll
         for (int i = 0; i < 8; ++i)
@@ -440,10 +441,15 @@ __device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
   __syncthreads();
 }
 
+// progress flags in shared memory between warp groups of one CTA: release /
+// acquire at CTA scope (the writer's data stores are ordered before the flag)
 __device__ __forceinline__ int ld_volatile_s(const int* p) {
   int v;
-  asm volatile("ld.volatile.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
   return v;
+}
+__device__ __forceinline__ void st_release_s(int* p, int v) {
+  asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
 
 // P of the critical chain by warps 0-3 only (group D), while warps 4-7 solve
@@ -497,6 +503,7 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
           v2[c] = fma(-v2[i], dg[c][i], v2[c]);
         }
       }
+      __syncwarp();  // every lane has read the diagonal block before lane 0 overwrites it
       if (lane == 0) {
 #pragma unroll
         for (int i = 0; i < 8; ++i)
@@ -509,10 +516,7 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
         if (b2) D[r2 * LD + c0 + j] = v2[j];
       }
       __syncwarp();
-      if (lane == 0) {  // panel p is final: the S warps may use it
-        __threadfence_block();
-        *reinterpret_cast<volatile int*>(dpanel) = p + 1;
-      }
+      if (lane == 0) st_release_s(dpanel, p + 1);  // panel p is final: the S warps may use it
       bar_arrive_id(BAR_DONE, GRP);
     }
     if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
