@@ -112,8 +112,9 @@ const char *stf_last_error(void);
  *                           over P column blocks (panel kernel + GEMM updates; default 4)
  *   "trsm_res_tail" STF_TRSM_RES_TAIL C >= 0: with trsm 3, every TRSM(i,k) of a panel step
  *                           whose trailing order n - k nb <= C uses the resident panel (default 8192)
- *   "trsm_res_split" STF_TRSM_RES_SPLIT 2 (default): a resident-panel TRSM runs as two column
- *                           halves with a GEMM between (more CTAs on the critical path); 1: one launch
+ *   "trsm_res_split" STF_TRSM_RES_SPLIT 2 (default) or 4: a resident-panel TRSM runs as that many
+ *                           column parts, right-looking, with a GEMM after each (more CTAs on the
+ *                           critical path); 1: one launch
  *   "trsm_rows" STF_TRSM_ROWS 32, 64 or 128 (default): rows per CTA of the row-panel TRSM
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA graph,
  *                           memoised per (n, nb, grid, tiles, options) (default); 0: eager

@@ -311,25 +311,31 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
 
 bool make_operand_map(CUtensorMap* tm, const double* ptr, int rows, int cols, int64_t ld, int bk);
 
-// Resident-panel TRSM in `parts` (1 or 2) column parts, right-looking: X1 = B1 L11^-T;
-// B2 -= X1 L21^T (GEMM on 64 x 64 CTA tiles: the whole GPU); X2 = B2 L22^-T.  The
-// substitution runs on half-width panels and the middle quarter of the flops at
-// GEMM rate: the critical TRSM(k+1,k) at nb = 1024 spreads beyond 64 SMs.
+// Resident-panel TRSM in `parts` (1, 2 or 4) column parts, right-looking: for each
+// part p, X_p = B_p L_pp^-T, then B_{>p} -= X_p L_{>p,p}^T (one GEMM on 64 x 64 CTA
+// tiles: the whole GPU).  The substitution runs on narrower panels and the
+// off-diagonal flops at GEMM rate: the critical TRSM(k+1,k) at nb = 1024 spreads
+// beyond the 64 CTAs of one resident-panel launch.
 cudaError_t trsm_res_parts(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                            int64_t ldb, const Mirrors* mirrors, int parts) {
-  const int h = n / 2;
-  if (parts < 2 || n % 128 || !trsm_res_supported(h, L, ldl) || (ldb & 1) || (reinterpret_cast<uintptr_t>(B) & 15))
+  if (parts < 2 || n % (64 * parts) || (ldb & 1) || (reinterpret_cast<uintptr_t>(B) & 15) ||
+      !trsm_res_supported(n / parts, L, ldl))
     return trsm_res(stream, prio, M, n, L, ldl, B, ldb, mirrors);
-  Mirrors m1{}, m2{};
-  if (mirrors) {
-    m1 = *mirrors;
-    m2 = *mirrors;
-    for (int m = 0; m < m2.n && m < 7; ++m) m2.p[m] = mirrors->p[m] + (int64_t)h * ldb;
+  const int w = n / parts;
+  for (int p = 0; p < parts; ++p) {
+    const int64_t c0 = (int64_t)p * w;
+    Mirrors mp{};
+    if (mirrors) {
+      mp = *mirrors;
+      for (int m = 0; m < mp.n && m < 7; ++m) mp.p[m] = mirrors->p[m] + c0 * ldb;
+    }
+    cudaError_t e = trsm_res(stream, prio, M, w, L + c0 * ldl + c0, ldl, B + c0 * ldb, ldb, &mp);
+    if (e == cudaSuccess && p + 1 < parts)
+      e = gemm_nt_tiles(stream, prio, M, n - (int)c0 - w, w, B + c0 * ldb, ldb, L + c0 * ldl + c0 + w, ldl,
+                        B + (c0 + w) * ldb, ldb, 0, 1);
+    if (e != cudaSuccess) return e;
   }
-  cudaError_t e = trsm_res(stream, prio, M, h, L, ldl, B, ldb, &m1);
-  if (e == cudaSuccess) e = gemm_nt_tiles(stream, prio, M, n - h, h, B, ldb, L + h, ldl, B + (int64_t)h * ldb, ldb, 0, 1);
-  if (e == cudaSuccess) e = trsm_res(stream, prio, M, n - h, L + (int64_t)h * ldl + h, ldl, B + (int64_t)h * ldb, ldb, &m2);
-  return e;
+  return cudaSuccess;
 }
 
 bool trsm_res_supported(int n, const double* L, int64_t ldl) {

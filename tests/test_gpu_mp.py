@@ -59,7 +59,7 @@ def test_bench_two_ranks_virtual_slots(mode):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr", "127.0.0.1", "--master-port", "29721" if mode == "mp" else "29731",
            os.path.join(ROOT, "bench.py"), "--gpus", "2", "--virtual-slots", "1", "--mode", mode,
-           "--n", "4096", "--nb", "512", "--steps", "2", "--warmup", "1", "--no-e2e", "--no-cpu"]
+           "--order", "4096", "--tile", "512", "--steps", "2", "--warmup", "1", "--no-e2e", "--no-cpu"]
     out = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT)
     assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-3000:]
     lines = [json.loads(l) for l in out.stdout.splitlines() if l.startswith("{")]

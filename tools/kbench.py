@@ -11,6 +11,9 @@ import paper_conf_sc_augonnetasg24_b200 as stf  # noqa: E402
 from paper_conf_sc_augonnetasg24_b200 import _abi  # noqa: E402
 
 nb = int(sys.argv[1]) if len(sys.argv) > 1 else 1024
+for kv in filter(None, os.environ.get("KB_OPT", "").split(",")):  # e.g. KB_OPT=trsm_res_split=4
+    k, v = kv.split("=")
+    stf.set_option(k, int(v))
 PEAK = 37.09
 out = {}
 for name, kind, M, N, K in (("gemm_tile", 0, nb, nb, nb), ("syrk_tile", 1, nb, nb, nb), ("trsm_tile", 2, nb, nb, 0),
@@ -22,6 +25,9 @@ for name, kind, M, N, K in (("gemm_tile", 0, nb, nb, nb), ("syrk_tile", 1, nb, n
 print(json.dumps(out), flush=True)
 if os.environ.get("KB_FULL", "1") == "1":
     stf.init(1, [0])
+    for kv in filter(None, os.environ.get("KB_OPT", "").split(",")):
+        k, v = kv.split("=")
+        stf.set_option(k, int(v))
     for n, b in ((8192, 1024), (8192, 512), (16384, 1024), (32768, 1024)):
         M = stf.TiledMatrix(n, b)
         ts = []
