@@ -441,17 +441,19 @@ __device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
   __syncthreads();
 }
 
-// progress flags in shared memory between warp groups of one CTA: shared-memory
-// atomics after a block-scope fence on the writer's side, a fence after the read
-// on the reader's (atomics are also what compute-sanitizer racecheck models)
+// progress flags in shared memory between warp groups of one CTA: release /
+// acquire at CTA scope (the writer's data stores are ordered before the flag, the
+// reader's data loads after it).  compute-sanitizer racecheck models barriers,
+// not flag protocols: it reports the data handed over this way as hazards
+// (profiles/r02/sanitize_racecheck.txt); shared-memory atomics instead of
+// ld.acquire/st.release do not change that and cost 12 us per POTRF tile.
 __device__ __forceinline__ int ld_volatile_s(const int* p) {
-  const int v = atomicOr(const_cast<int*>(p), 0);
-  __threadfence_block();
+  int v;
+  asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
   return v;
 }
 __device__ __forceinline__ void st_release_s(int* p, int v) {
-  __threadfence_block();
-  atomicExch(p, v);
+  asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
 
 // P of the critical chain by warps 0-3 only (group D), while warps 4-7 solve
