@@ -197,9 +197,6 @@ __device__ void task_update(double* sm, double* C, int64_t ldc, const double* A,
       }
 }
 
-__device__ __forceinline__ void named_bar(int id, int nthreads) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
-}
 
 // Substitution core.  Thread (r = tid & 63, q = tid >> 6) holds X[r, 16q .. 16q+15]
 // in b[].  Ls[c * LDB + p] = L(c, p) (lower part read only).  Chunk q solves its
@@ -333,114 +330,6 @@ __device__ __forceinline__ void bar_arrive_id(int id, int n) {
   asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
-// P of a full 64 x 64 diagonal block held row-major in D (lower part, LDB stride),
-// in place, latency-optimised for the critical chain.  8 panels of 8 columns:
-//   (a) warp 0 factors the panel: every lane factors the 8 x 8 diagonal block
-//       redundantly in registers (no shuffles on the sqrt -> reciprocal -> divide
-//       chain) and the two rows it owns below it (lane, lane + 32);
-//   (b) six warps on the other SM sub-partitions (1-3, 5-7) apply the panel to the
-//       trailing lower block on DMMA (K = 8) with a look-ahead of one panel: the
-//       next panel's columns first -- then they release warp 0 (named barrier
-//       NEXT) -- and the remaining columns while warp 0 already factors the next
-//       panel (barrier DONE hands each finished panel to them).  Each 8 x 8
-//       output tile has one owner warp for the whole block (static map), so its
-//       updates stay in increasing panel order.
-// Correctly rounded sqrt and division (div_by with y = RN(1/s)); every element
-// receives its updates in increasing column order, each a single fma or a DMMA
-// k-step pair, deterministic (the same operations as without look-ahead).
-// Non-positive pivot (or NaN): info = min(info, col0 + col + 1), s = NaN.
-__device__ void chol_block(double* D, int64_t col0, unsigned long long* info) {
-  constexpr int LD = df::LDB, BAR_DONE = 1, BAR_NEXT = 2;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
-  const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
-  // warp 4 shares warp 0's sub-partition: it stays out of the FP64 pipe
-  constexpr int NPART = 6 * 32 + 32;  // barrier participants: six MMA warps + warp 0
-  if (warp == 0) {
-    int bad = 0;
-#pragma unroll 1
-    for (int p = 0; p < 8; ++p) {
-      if (p > 0) bar_sync_id(BAR_NEXT, NPART);  // columns 8p .. 8p+7 received the update from panel p-1
-      const int c0 = 8 * p;
-      double dg[8][8];
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j <= i; ++j) dg[i][j] = D[(c0 + i) * LD + c0 + j];
-      const int r1 = lane, r2 = lane + 32;
-      const bool b1 = r1 >= c0 + 8, b2 = r2 >= c0 + 8;
-      double v1[8], v2[8];
-#pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
-        v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
-      }
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const double d = dg[i][i];
-        const bool ok = d > 0.0;
-        if (!ok && bad == 0) bad = c0 + i + 1;
-        const double sq = ok ? sqrt(d) : kNaN, y = 1.0 / sq;
-        dg[i][i] = sq;
-#pragma unroll
-        for (int r = i + 1; r < 8; ++r) dg[r][i] = div_by(dg[r][i], sq, y);
-#pragma unroll
-        for (int r = i + 1; r < 8; ++r)
-#pragma unroll
-          for (int c = i + 1; c <= r; ++c) dg[r][c] = fma(-dg[r][i], dg[c][i], dg[r][c]);
-        v1[i] = div_by(v1[i], sq, y);
-        v2[i] = div_by(v2[i], sq, y);
-#pragma unroll
-        for (int c = i + 1; c < 8; ++c) {
-          v1[c] = fma(-v1[i], dg[c][i], v1[c]);
-          v2[c] = fma(-v2[i], dg[c][i], v2[c]);
-        }
-      }
-      __syncwarp();  // every lane has read the diagonal block before lane 0 overwrites it
-      if (lane == 0) {
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j <= i; ++j) D[(c0 + i) * LD + c0 + j] = dg[i][j];
-      }
-#pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        if (b1) D[r1 * LD + c0 + j] = v1[j];
-        if (b2) D[r2 * LD + c0 + j] = v2[j];
-      }
-      bar_arrive_id(BAR_DONE, NPART);  // panel p final
-    }
-    if (bad) atomicMin(info, (unsigned long long)(col0 + bad));
-  } else if (warp != 4) {
-    const int mw = warp < 4 ? warp - 1 : warp - 2;  // 0..5
-    auto update = [&](int R, int Cb, int c0) {      // tile rows 8R.., columns 8Cb.. from panel columns c0..
-      double* rowp = D + (8 * R + g) * LD;
-      double* cp = rowp + 8 * Cb + 2 * t;
-      double acc0 = cp[0], acc1 = cp[1];
-#pragma unroll
-      for (int ks = 0; ks < 2; ++ks) {
-        const double a = rowp[c0 + 4 * ks + t];
-        const double b = negd(D[(8 * Cb + g) * LD + c0 + 4 * ks + t]);
-        dmma_8x8x4(acc0, acc1, a, b);
-      }
-      cp[0] = acc0;
-      cp[1] = acc1;
-    };
-#pragma unroll 1
-    for (int p = 0; p < 7; ++p) {
-      bar_sync_id(BAR_DONE, NPART);  // panel p is final
-      const int c0 = 8 * p;
-      for (int R = p + 1; R < 8; ++R)  // look-ahead: the next panel's columns
-        if ((R + 5 * (p + 1)) % 6 == mw) update(R, p + 1, c0);
-      bar_arrive_id(BAR_NEXT, NPART);
-      for (int Cb = p + 2; Cb < 8; ++Cb)  // the remaining trailing lower part
-        for (int R = Cb; R < 8; ++R)
-          if ((R + 5 * Cb) % 6 == mw) update(R, Cb, c0);
-    }
-    bar_sync_id(BAR_DONE, NPART);  // panel 7
-  }
-  __syncthreads();
-}
-
 // progress flags in shared memory between warp groups of one CTA: release /
 // acquire at CTA scope (the writer's data stores are ordered before the flag, the
 // reader's data loads after it).  compute-sanitizer racecheck models barriers,
@@ -456,13 +345,25 @@ __device__ __forceinline__ void st_release_s(int* p, int v) {
   asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
 
-// P of the critical chain by warps 0-3 only (group D), while warps 4-7 solve
-// S(kb+1, kb) against the panels as they become final (critical_chain).  Warp 0
-// factors each 8-column panel (as in chol_block), warps 1-3 apply it to the
-// trailing lower block on DMMA with the same one-panel look-ahead (named barriers
-// 1 / 2 over the 128 threads of the group); after panel p, *dpanel = p + 1
-// tells the S warps its columns are final.  Same operations per element as
-// chol_block: bit-identical.
+// P(kb) of the critical chain: the full 64 x 64 diagonal block held row-major in
+// D (lower part, LDB stride), in place, by warps 0-3 (group D) while warps 4-7
+// solve S(kb+1, kb) against the panels as they become final (critical_chain).
+// 8 panels of 8 columns:
+//   (a) warp 0 factors the panel: every lane factors the 8 x 8 diagonal block
+//       redundantly in registers (no shuffles on the sqrt -> reciprocal -> divide
+//       chain) and the two rows it owns below it (lane, lane + 32);
+//   (b) warps 1-3 (the other SM sub-partitions) apply the panel to the trailing
+//       lower block on DMMA (K = 8) with a look-ahead of one panel: the next
+//       panel's columns first -- then they release warp 0 (named barrier NEXT) --
+//       and the remaining columns while warp 0 already factors the next panel
+//       (barrier DONE hands each finished panel to them).  Each 8 x 8 output tile
+//       has one owner warp for the whole block (static map), so its updates stay
+//       in increasing panel order.
+// After panel p, *dpanel = p + 1 tells the S warps its columns are final.
+// Correctly rounded sqrt and division (div_by with y = RN(1/s)); every element
+// receives its updates in increasing column order, each a single fma or a DMMA
+// k-step pair: the same operations as without look-ahead, deterministic.
+// Non-positive pivot (or NaN): info = min(info, col0 + col + 1), s = NaN.
 __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info, int* dpanel) {
   constexpr int LD = df::LDB, BAR_DONE = 1, BAR_NEXT = 2, GRP = 128;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
@@ -562,16 +463,6 @@ __device__ __forceinline__ void load_il(double (&v)[16], const double* G, int64_
   for (int m = 0; m < 16; ++m) {
     const int col = 4 * m + q;
     v[m] = (r < rows && col < nc && (!lower || r >= col)) ? __ldcg(G + (int64_t)col * ldg + r) : 0.0;
-  }
-}
-__device__ __forceinline__ void store_il(const double (&v)[16], double* G, int64_t ldg, int rows, int nc, bool lower) {
-  const int r = threadIdx.x & (df::W - 1), q = threadIdx.x >> 6;
-  if (r < rows) {
-#pragma unroll
-    for (int m = 0; m < 16; ++m) {
-      const int col = 4 * m + q;
-      if (col < nc && (!lower || r >= col)) G[(int64_t)col * ldg + r] = v[m];
-    }
   }
 }
 
