@@ -115,6 +115,11 @@ const char *stf_last_error(void);
  *   "trsm_res_split" STF_TRSM_RES_SPLIT 2 (default) or 4: a resident-panel TRSM runs as that many
  *                           column parts, right-looking, with a GEMM after each (more CTAs on the
  *                           critical path); 1: one launch
+ *   "gemm_merge" STF_GEMM_MERGE D >= 0: the tile updates GEMM(i,j,k) and GEMM(i,j,k+1), k even,
+ *                           of a tile at least D columns right of panel k+1 become ONE task at
+ *                           step k+1 (one k sweep of 2 nb: one C load/store and pipeline ramp
+ *                           instead of two; the same operations per element, same bits);
+ *                           0 = off.  Not with lookahead = 0.
  *   "trsm_rows" STF_TRSM_ROWS 32, 64 or 128 (default): rows per CTA of the row-panel TRSM
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA graph,
  *                           memoised per (n, nb, grid, tiles, options) (default); 0: eager
@@ -208,6 +213,7 @@ typedef struct stf_plan_stats {
   int64_t devices;        /* distinct CUDA devices spanned by the call's slots */
   int64_t slots;          /* GPU slots of the call (ngpus) */
   int64_t peer_transfers; /* transfers whose source and destination are distinct devices */
+  int64_t merged_gemms;   /* GEMM tasks that carry two consecutive tile updates ("gemm_merge") */
 } stf_plan_stats;
 
 int stf_last_stats(stf_plan_stats *out);
@@ -238,6 +244,12 @@ int stf_dag_build_call(int64_t n, int64_t nb, int kind, int ngpus, int p, int q,
  * writes a frame from the caller's tile (i, j), STORE reads one).  Returns the
  * number of buffers.  Needs no GPU. */
 int stf_dag_tasks_io(int64_t cap_tasks, int64_t *io);
+
+/* Second operand pair of merged GEMM tasks ("gemm_merge") of the last
+ * stf_dag_build(_call) on this thread: io2[2*t], io2[2*t+1] = the buffers of
+ * L_i,k+1 and L_j,k+1 of a task GEMM(i,j,k) that also applies update k+1 (-1
+ * otherwise).  Returns the number of merged tasks.  Needs no GPU. */
+int64_t stf_dag_tasks_io2(int64_t cap_tasks, int64_t *io2);
 
 /* Replica buffers written by the tasks of the last stf_dag_build(_call) on this
  * thread besides their output (fused push, "push" = 1): mir[8*t] = count (<= 7),

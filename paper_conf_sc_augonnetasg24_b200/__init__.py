@@ -107,6 +107,13 @@ def dag_io(ntasks: int):
     return [((IO[3 * t], IO[3 * t + 1]), IO[3 * t + 2]) for t in range(ntasks)], nbuf
 
 
+def dag_io2(ntasks: int):
+    """Second operand pair (L_i,k+1, L_j,k+1 buffers) of merged GEMM tasks, else (-1, -1)."""
+    IO = (ctypes.c_int64 * (2 * max(1, ntasks)))()
+    check(_abi.stf_dag_tasks_io2(ntasks, IO), "stf_dag_tasks_io2")
+    return [(IO[2 * t], IO[2 * t + 1]) for t in range(ntasks)]
+
+
 def dag_mirrors(ntasks: int):
     """Replica buffers each task of the last dag()/dag_call() also writes (fused push)."""
     MI = (ctypes.c_int64 * (8 * max(1, ntasks)))()

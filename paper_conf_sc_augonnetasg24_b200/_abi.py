@@ -55,6 +55,7 @@ class stf_plan_stats(ctypes.Structure):
         ("devices", ctypes.c_int64),
         ("slots", ctypes.c_int64),
         ("peer_transfers", ctypes.c_int64),
+        ("merged_gemms", ctypes.c_int64),
     ]
 
     def as_dict(self):
@@ -65,7 +66,7 @@ class stf_plan_stats(ctypes.Structure):
 EXPORTS = [
     "stf_cholesky_init", "stf_potrf", "stf_finalize", "stf_last_error",
     "stf_set_option", "stf_get_option", "stf_last_stats", "stf_dag_build", "stf_dag_build_call", "stf_infer_edges",
-    "stf_dag_tasks_io", "stf_dag_tasks_mirrors", "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
+    "stf_dag_tasks_io", "stf_dag_tasks_io2", "stf_dag_tasks_mirrors", "stf_mp_init", "stf_mp_blob_size", "stf_mp_prepare", "stf_mp_import", "stf_mp_potrf",
 ]
 # ... and every symbol include/stf_harness.h declares (test / benchmark entry points).
 HARNESS_EXPORTS = [
@@ -112,6 +113,7 @@ stf_kernel_potrf = _decl("stf_kernel_potrf", _int, [_i64, _vp, _i64, _P(_i64)])
 stf_bench_kernel = _decl("stf_bench_kernel", _int, [_int, _i64, _i64, _i64, _int, _P(_dbl)])
 stf_dag_tasks_io = _decl("stf_dag_tasks_io", _int, [_i64, _P(_i64)])
 stf_dag_tasks_mirrors = _decl("stf_dag_tasks_mirrors", _i64, [_i64, _P(_i64)])
+stf_dag_tasks_io2 = _decl("stf_dag_tasks_io2", _i64, [_i64, _P(_i64)])
 stf_mp_init = _decl("stf_mp_init", _int, [_int, _int, _int])
 stf_mp_blob_size = _decl("stf_mp_blob_size", _i64, [])
 stf_mp_prepare = _decl("stf_mp_prepare", _int, [_i64, _i64, _P(stf_matrix_desc), _vp])

@@ -88,6 +88,8 @@ stf::PlanOptions call_plan_options(const Options& o, int64_t n, int64_t nb, int 
   po.push = o.push != 0 && o.trsm >= 2;
   po.push_potrf = po.push && o.dataflow != 0;  // the dataflow POTRF kernel stores into replicas
   po.data_plane = po.push ? (int)o.push : 0;
+  // merged tile updates need whole k tiles of 32 for the second pair (gemm_nt2)
+  po.gemm_merge = (nb % 32 == 0) ? (int)o.gemm_merge : 0;
   po.ooc_order = (int)o.ooc_order;
   // Scheduling model of the submission order (plan.cpp reorder_list), in units of
   // one nb^3 GEMM task's duration while `width` of them share the GPU: a tile
@@ -255,9 +257,15 @@ struct Lowerer {
                  "SYRK launch");
         return 0;
       case stf::K_GEMM:
-        CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[1]],
-                               nb, X.buf[(size_t)t.out], nb, 0),
-                 "GEMM launch");
+        if (t.in2[0] >= 0)  // merged GEMM(i,j,k) + GEMM(i,j,k+1): one k sweep of 2 nb
+          CUDA_TRY(stfk::gemm_nt2(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[1]],
+                                  nb, (int)nb, X.buf[(size_t)t.in2[0]], nb, X.buf[(size_t)t.in2[1]], nb,
+                                  X.buf[(size_t)t.out], nb, 0, 0),
+                   "GEMM launch");
+        else
+          CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[1]],
+                                 nb, X.buf[(size_t)t.out], nb, 0),
+                   "GEMM launch");
         return 0;
       case stf::K_COPY:
         // Push of a finished tile into a consumer slot's replica on the producer's
@@ -822,6 +830,7 @@ void fill_plan_stats(const stf::Plan& P, int64_t nb, stf_plan_stats* s) {
   for (int64_t r : P.replicas_per_slot) mx = std::max(mx, r);
   s->replicas_max = mx;
   s->data_plane = P.opt.data_plane;
+  s->merged_gemms = P.nmerged;
 }
 
 void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {

@@ -65,16 +65,23 @@ __device__ __forceinline__ uint32_t swz_off(int r, int k) {
   return box * g::BOX_BYTES + k * 128 + ((((mi >> 1) ^ (k & 7)) << 4) | ((mi & 1) << 3));
 }
 
+// k-tile kt of the operand pair: kt < KT1 from (tmA, tmB), else tile kt - KT1 of the
+// second pair (tmA2, tmB2): a merged update C -= A B^T + A2 B2^T in one k sweep
 template <class g>
 __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                                           int m0, int n0, int kt, uint64_t* full) {
+                                           const CUtensorMap* tmA2, const CUtensorMap* tmB2, int KT1, int m0, int n0,
+                                           int kt, uint64_t* full) {
   mbar_arrive_expect_tx(&full[s], g::STAGE_BYTES);
   uint8_t* sa = smem + s * g::STAGE_BYTES;
   uint8_t* sb = sa + g::A_BYTES;
+  const bool second = kt >= KT1;
+  const CUtensorMap* ma = second ? tmA2 : tmA;
+  const CUtensorMap* mb = second ? tmB2 : tmB;
+  const int kk = second ? kt - KT1 : kt;
 #pragma unroll
-  for (int b = 0; b < g::BM / g::BOX; ++b) tma_load_2d(sa + b * g::BOX_BYTES, tmA, m0 + b * g::BOX, kt * g::BK, &full[s]);
+  for (int b = 0; b < g::BM / g::BOX; ++b) tma_load_2d(sa + b * g::BOX_BYTES, ma, m0 + b * g::BOX, kk * g::BK, &full[s]);
 #pragma unroll
-  for (int b = 0; b < g::BN / g::BOX; ++b) tma_load_2d(sb + b * g::BOX_BYTES, tmB, n0 + b * g::BOX, kt * g::BK, &full[s]);
+  for (int b = 0; b < g::BN / g::BOX; ++b) tma_load_2d(sb + b * g::BOX_BYTES, mb, n0 + b * g::BOX, kk * g::BK, &full[s]);
 }
 
 // All warps are consumers (a dedicated producer warp would lower the register cap:
@@ -85,7 +92,8 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
 template <int WM, int WN, class g>
 __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                        double* __restrict__ C, int64_t ldc, int M, int N, int K, int lower) {
+                        const __grid_constant__ CUtensorMap tmA2, const __grid_constant__ CUtensorMap tmB2,
+                        double* __restrict__ C, int64_t ldc, int M, int N, int K, int K2, int lower) {
   constexpr int NCW = (g::BM / WM) * (g::BN / WN);
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // keep the pointer derived from the __shared__ array (integer offset only) so
@@ -117,18 +125,23 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
     tn = blockIdx.y;
   }
   const int m0 = tm * g::BM, n0 = tn * g::BN;
-  const int KT = (K + g::BK - 1) / g::BK;
+  const int KT1 = (K + g::BK - 1) / g::BK;
+  const int KT = KT1 + (K2 + g::BK - 1) / g::BK;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
+    if (K2 > 0) {
+      tma_prefetch_desc(&tmA2);
+      tma_prefetch_desc(&tmB2);
+    }
     for (int s = 0; s < g::STAGES; ++s) {
       mbar_init(&full[s], 1);
       released[s] = 0;
     }
     fence_barrier_init();
-    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, m0, n0, kt, full);
+    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, &tmA2, &tmB2, KT1, m0, n0, kt, full);
   }
   __syncthreads();
 
@@ -200,7 +213,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
         released[s] = 0;
         __threadfence_block();
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        load_stage<g>(smem, s, &tmA, &tmB, m0, n0, kt + g::STAGES, full);
+        load_stage<g>(smem, s, &tmA, &tmB, &tmA2, &tmB2, KT1, m0, n0, kt + g::STAGES, full);
       }
     }
   }
@@ -285,15 +298,16 @@ static int syrk64_max() {
 }
 
 template <class G>
-static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tmA, const CUtensorMap& tmB, double* C,
-                                  int64_t ldc, int M, int N, int K, int lower) {
+static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tmA, const CUtensorMap& tmB,
+                                  const CUtensorMap& tmA2, const CUtensorMap& tmB2, double* C, int64_t ldc, int M, int N,
+                                  int K, int K2, int lower) {
   cfg.dynamicSmemBytes = G::SMEM_BYTES;
   if (gemm_warps() == 16) {
     cfg.blockDim = dim3(512, 1, 1);
-    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, G>, tmA, tmB, C, ldc, M, N, K, lower);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, G>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
   }
   cfg.blockDim = dim3(256, 1, 1);
-  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, G>, tmA, tmB, C, ldc, M, N, K, lower);
+  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, G>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
 }
 
 cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
@@ -303,14 +317,32 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
 
 cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
                           const double* B, int64_t ldb, double* C, int64_t ldc, int lower, int small) {
+  return gemm_nt2(stream, prio, M, N, K, A, lda, B, ldb, 0, nullptr, 0, nullptr, 0, C, ldc, lower, small);
+}
+
+cudaError_t gemm_nt2(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda, const double* B,
+                     int64_t ldb, int K2, const double* A2, int64_t lda2, const double* B2, int64_t ldb2, double* C,
+                     int64_t ldc, int lower, int small) {
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
     return cudaErrorMisalignedAddress;
+  if (K2 > 0 && ((reinterpret_cast<uintptr_t>(A2) & 15) || (reinterpret_cast<uintptr_t>(B2) & 15) || (lda2 & 1) ||
+                 (ldb2 & 1)))
+    return cudaErrorMisalignedAddress;
   const bool narrow = gemm_narrow() != 0;
   const int bk = narrow ? 32 : gemm_bk();
-  CUtensorMap tmA, tmB;
+  // the second pair starts on a fresh k tile: the first pair's K must fill whole tiles
+  if (K2 > 0 && K % bk) return cudaErrorInvalidValue;
+  CUtensorMap tmA, tmB, tmA2, tmB2;
   if (!make_operand_map(&tmA, A, M, K, lda, bk) || !make_operand_map(&tmB, B, N, K, ldb, bk))
     return cudaErrorInvalidValue;
+  if (K2 > 0) {
+    if (!make_operand_map(&tmA2, A2, M, K2, lda2, bk) || !make_operand_map(&tmB2, B2, N, K2, ldb2, bk))
+      return cudaErrorInvalidValue;
+  } else {
+    tmA2 = tmA;
+    tmB2 = tmB;
+  }
   cudaLaunchConfig_t cfg = {};
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributePriority;
@@ -325,10 +357,10 @@ cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, co
     ++launch_count();
     if (s64_warps() == 8) {  // 32 x 16 warp tiles: two warps per SM sub-partition
       cfg.blockDim = dim3(256, 1, 1);
-      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 16, CfgS64>, tmA, tmB, C, ldc, M, N, K, lower);
+      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 16, CfgS64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
     }
     cfg.blockDim = dim3(128, 1, 1);
-    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgS64>, tmA, tmB, C, ldc, M, N, K, lower);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgS64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
   }
   const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
   cfg.gridDim = lower ? dim3(narrow ? tM * (tM + 1) : tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
@@ -337,13 +369,13 @@ cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, co
     cfg.dynamicSmemBytes = CfgN64::SMEM_BYTES;
     if (gemm_narrow() == 2) {  // 8 warps of 32 x 32, 2 CTAs (16 warps) per SM
       cfg.blockDim = dim3(256, 1, 1);
-      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64>, tmA, tmB, C, ldc, M, N, K, lower);
+      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
     }
     cfg.blockDim = dim3(128, 1, 1);  // 4 warps of 64 x 32
-    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, CfgN64>, tmA, tmB, C, ldc, M, N, K, lower);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, CfgN64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
   }
-  if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
-  return launch_variant<CfgK16>(cfg, tmA, tmB, C, ldc, M, N, K, lower);
+  if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+  return launch_variant<CfgK16>(cfg, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
 }
 
 template <class G>

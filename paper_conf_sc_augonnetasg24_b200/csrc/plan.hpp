@@ -39,6 +39,8 @@ struct Task {
   int64_t out;       // buffer id written
   int32_t nmir;      // fused push (NEXT-3): replica buffers written by the same kernel
   int64_t mir[7];
+  int64_t in2[2] = {-1, -1};  // merged GEMM: the second update's operands (GEMM(i,j,k) and GEMM(i,j,k+1)
+                              // in one task: in = L_ik, L_jk; in2 = L_i,k+1, L_j,k+1), else -1
 };
 
 struct PlanOptions {
@@ -66,6 +68,8 @@ struct PlanOptions {
   bool push = false;       // TRSM(i,k) writes L_ik into its consumers' replicas itself (fused
                            // push, NEXT-3) instead of COPY tasks at the first remote read
   int data_plane = 0;      // requested data plane (statistics): 0 COPY, 1 fused push, 2 multicast
+  int gemm_merge = 0;      // > 0: GEMM(i,j,k) and GEMM(i,j,k+1) (k even) of a tile at least this many
+                           // columns right of panel k+1 become one task at step k+1 (one K = 2 nb sweep)
   bool push_potrf = false; // with push: POTRF(k) also writes L_kk into the replicas of the
                            // slots running TRSM(i,k) (the dataflow POTRF kernel's epilogue)
   int64_t frames = 0;      // > 0 (one slot, with_load/with_store): memory-capped out-of-core
@@ -95,6 +99,7 @@ struct Plan {
   TaskGraph graph;
   int64_t ntransfers = 0;     // COPY tasks
   int64_t npushed = 0;        // replicas written by fused push
+  int64_t nmerged = 0;        // merged GEMM tasks (two tile updates each)
   int64_t nloads = 0;         // LOAD tasks (caller matrix -> device tile)
   int64_t nstores = 0;        // STORE tasks (device tile -> caller matrix)
   int64_t critical_path = 0;  // longest chain counted in compute tasks

@@ -20,26 +20,34 @@ import synth
 NB = 4  # tile order for the emulation (values are irrelevant to the schedule)
 
 
-def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0):
+def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0):
     stf.set_option("mem_cap_tiles", frames)
     stf.set_option("lookahead", lookahead)
     stf.set_option("ooc_order", ooc_order)
     stf.set_option("push", push)
+    stf.set_option("gemm_merge", merge)
     try:
         edges, kinds, ijk, st = stf.dag(T, p, q)
         io, nbuf = stf.dag_io(len(kinds))
-        mir = stf.dag_mirrors(len(kinds))
+        _extras(len(kinds))
     finally:
         stf.set_option("mem_cap_tiles", 0)
         stf.set_option("lookahead", 1)
         stf.set_option("ooc_order", -1)
         stf.set_option("push", 0)
-    _MIRRORS.clear()
-    _MIRRORS.extend(mir)
+        stf.set_option("gemm_merge", 0)
     return edges, kinds, ijk, io, nbuf, st
 
 
 _MIRRORS = []  # replica writes (fused push) of the tasks of the last _plan()
+_IO2 = []      # second operand pair of merged GEMM tasks of the last _plan()
+
+
+def _extras(ntasks):
+    _MIRRORS.clear()
+    _MIRRORS.extend(stf.dag_mirrors(ntasks))
+    _IO2.clear()
+    _IO2.extend(stf.dag_io2(ntasks))
 
 
 def _emulate(T, A, kinds, ijk, io, nbuf, edges, order_seed, host_resident):
@@ -76,6 +84,8 @@ def _emulate(T, A, kinds, ijk, io, nbuf, edges, order_seed, host_resident):
             buf[w][:, :] = oracle.tile_syrk(buf[w], buf[r0])
         elif kd == "GEMM":
             buf[w][:, :] = oracle.tile_gemm(buf[w], buf[r0], buf[r1])
+            if _IO2 and _IO2[t][0] >= 0:  # merged task: update k+1 right after update k
+                buf[w][:, :] = oracle.tile_gemm(buf[w], buf[_IO2[t][0]], buf[_IO2[t][1]])
         elif kd == "COPY":
             buf[w][:, :] = buf[r0]
         elif kd == "LOAD":
@@ -209,8 +219,7 @@ def test_out_of_core_2d_order_cuts_panel_reloads():
 def _call_plan(n, nb, kind, p=1, q=1):
     edges, kinds, ijk, st = stf.dag_call(n, nb, kind, p, q)
     io, nbuf = stf.dag_io(len(kinds))
-    _MIRRORS.clear()
-    _MIRRORS.extend(stf.dag_mirrors(len(kinds)))
+    _extras(len(kinds))
     return edges, kinds, ijk, io, nbuf, st
 
 
@@ -275,3 +284,31 @@ def test_out_of_core_rejects_fence_ablation():
     finally:
         stf.set_option("mem_cap_tiles", 0)
         stf.set_option("lookahead", 1)
+
+
+@pytest.mark.parametrize("T,p,q,merge,push", [(8, 1, 1, 1, 0), (9, 1, 1, 3, 0), (12, 2, 2, 2, 0), (12, 2, 4, 3, 1),
+                                             (10, 1, 8, 1, 0), (16, 1, 1, 3, 0)])
+def test_merged_gemm_plans_any_topological_order(T, p, q, merge, push):
+    """gemm_merge: GEMM(i,j,k) and GEMM(i,j,k+1) of far tiles as one task (two
+    consecutive updates in one k sweep): the plan stays a correct STF DAG -- the
+    oracle's bits in random orders -- with fewer GEMM tasks."""
+    A = synth.spd_matrix(17, T * NB)
+    e0, k0, _, _, _, st0 = _plan(T, p, q, push=push)
+    edges, kinds, ijk, io, nbuf, st = _plan(T, p, q, push=push, merge=merge)
+    assert st["merged_gemms"] > 0 and st0["merged_gemms"] == 0
+    assert st["tasks"] == st0["tasks"] - st["merged_gemms"]
+    assert kinds.count("GEMM") == k0.count("GEMM") - st["merged_gemms"]
+    ref = _reference(T, A)
+    for seed in (-1, 1, 2):
+        got = _emulate(T, A, kinds, ijk, io, nbuf, edges, seed, host_resident=False)
+        assert np.array_equal(got, ref), (seed, np.abs(got - ref).max())
+
+
+def test_merged_gemm_call_plan_bench_config():
+    """The bench's plan (n = 65536, nb = 1024, T = 64) with the default merge
+    distance, executed in a random topological order on 4 x 4 tiles."""
+    n, nb, T = 65536, 1024, 64
+    edges, kinds, ijk, io, nbuf, st = _call_plan(n, nb, stf.STF_DESC_TILED_2DBC)
+    A = synth.spd_matrix(18, T * NB)
+    got = _emulate(T, A, kinds, ijk, io, nbuf, edges, 3, host_resident=False)
+    assert np.array_equal(got, _reference(T, A))
