@@ -471,7 +471,7 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
         "e2e": e2e,
         "plan": {k: stats[k] for k in ("tasks", "dag_tasks", "edges", "critical_path", "graph_nodes", "kernel_launches",
                                        "transfers", "transfer_bytes", "pushed", "replicas_max", "data_plane",
-                                       "devices", "slots", "peer_transfers", "build_ms")},
+                                       "devices", "slots", "peer_transfers", "merged_gemms", "build_ms")},
         "check": check,
         "first_call_ms": round(first_ms, 1) if first_ms else None,
         "step_ms": [round(x, 3) for x in steps_ms],
