@@ -10,6 +10,14 @@ import paper_conf_sc_augonnetasg24_b200 as stf
 KIND = {"POTRF": "POTRF", "TRSM": "TRSM", "SYRK": "SYRK", "GEMM": "GEMM"}
 
 
+
+@pytest.fixture(autouse=True)
+def _paper_granularity():
+    """These tests check the paper's DAG: one task per tile update (no merged GEMMs)."""
+    stf.set_option("gemm_merge", 0)
+    yield
+    stf.set_option("gemm_merge", 2)
+
 def test_alg1_worked_example_cpp_core():
     # PAPER.md:31-40 (Algorithm 1) -> Fig. 1: {O1->O2, O1->O3, O2->O4, O3->O4}
     X, Y, Z = 0, 1, 2

@@ -21,6 +21,7 @@ NB = 4  # tile order for the emulation (values are irrelevant to the schedule)
 
 
 def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0):
+    """Plan of stf_dag_build with these options (gemm_merge restored to its default 2 after)."""
     stf.set_option("mem_cap_tiles", frames)
     stf.set_option("lookahead", lookahead)
     stf.set_option("ooc_order", ooc_order)
@@ -35,7 +36,7 @@ def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0):
         stf.set_option("lookahead", 1)
         stf.set_option("ooc_order", -1)
         stf.set_option("push", 0)
-        stf.set_option("gemm_merge", 0)
+        stf.set_option("gemm_merge", 2)
     return edges, kinds, ijk, io, nbuf, st
 
 
@@ -241,7 +242,8 @@ def test_call_plans_any_topological_order(n, nb, kind, p, q):
     T = n // nb
     edges, kinds, ijk, io, nbuf, st = _call_plan(n, nb, kind, p, q)
     NT = T * (T + 1) // 2
-    assert st["tasks"] == T + T * (T - 1) + T * (T - 1) * (T - 2) // 6
+    # merged GEMM tasks (gemm_merge, device-resident plans) carry two tile updates each
+    assert st["tasks"] + st["merged_gemms"] == T + T * (T - 1) + T * (T - 1) * (T - 2) // 6
     host = kind == stf.STF_DESC_HOST_COLMAJOR
     if host and p * q == 1 and T >= 16:
         assert st["frames"] == NT  # host_stream: one frame per tile, nothing evicted
@@ -309,6 +311,7 @@ def test_merged_gemm_call_plan_bench_config():
     distance, executed in a random topological order on 4 x 4 tiles."""
     n, nb, T = 65536, 1024, 64
     edges, kinds, ijk, io, nbuf, st = _call_plan(n, nb, stf.STF_DESC_TILED_2DBC)
+    assert st["merged_gemms"] > 0
     A = synth.spd_matrix(18, T * NB)
     got = _emulate(T, A, kinds, ijk, io, nbuf, edges, 3, host_resident=False)
     assert np.array_equal(got, _reference(T, A))
