@@ -115,11 +115,12 @@ const char *stf_last_error(void);
  *   "trsm_res_split" STF_TRSM_RES_SPLIT 2 (default) or 4: a resident-panel TRSM runs as that many
  *                           column parts, right-looking, with a GEMM after each (more CTAs on the
  *                           critical path); 1: one launch
- *   "gemm_merge" STF_GEMM_MERGE D >= 0: the tile updates GEMM(i,j,k) and GEMM(i,j,k+1), k even,
- *                           of a tile at least D columns right of panel k+1 become ONE task at
- *                           step k+1 (one k sweep of 2 nb: one C load/store and pipeline ramp
- *                           instead of two; the same operations per element, same bits);
- *                           0 = off.  Not with lookahead = 0.
+ *   "gemm_merge" STF_GEMM_MERGE D >= 0 (default 2): the tile updates GEMM(i,j,k) of a group of
+ *                           G consecutive panels k = gG .. gG+G-1 ("gemm_group" G = 2..4, default
+ *                           2) become ONE task at step gG+G-1 when the tile is at least D columns
+ *                           right of that panel (one k sweep of G nb: one C load/store and
+ *                           pipeline ramp instead of G; the same operations per element, same
+ *                           bits); 0 = off.  Not with lookahead = 0.
  *   "trsm_rows" STF_TRSM_ROWS 32, 64 or 128 (default): rows per CTA of the row-panel TRSM
  *   "graph"    STF_GRAPH    1: capture the whole task DAG of a call into one CUDA graph,
  *                           memoised per (n, nb, grid, tiles, options) (default); 0: eager
@@ -245,10 +246,11 @@ int stf_dag_build_call(int64_t n, int64_t nb, int kind, int ngpus, int p, int q,
  * number of buffers.  Needs no GPU. */
 int stf_dag_tasks_io(int64_t cap_tasks, int64_t *io);
 
-/* Second operand pair of merged GEMM tasks ("gemm_merge") of the last
- * stf_dag_build(_call) on this thread: io2[2*t], io2[2*t+1] = the buffers of
- * L_i,k+1 and L_j,k+1 of a task GEMM(i,j,k) that also applies update k+1 (-1
- * otherwise).  Returns the number of merged tasks.  Needs no GPU. */
+/* Further operand pairs of merged GEMM tasks ("gemm_merge") of the last
+ * stf_dag_build(_call) on this thread: io2[6*t + 2(u-1)], io2[6*t + 2(u-1) + 1] =
+ * the buffers of L_i,k+u and L_j,k+u (u = 1..3) of a task GEMM(i,j,k) that also
+ * applies updates k+1, .. (-1 where unused).  Returns the number of merged tasks.
+ * Needs no GPU. */
 int64_t stf_dag_tasks_io2(int64_t cap_tasks, int64_t *io2);
 
 /* Replica buffers written by the tasks of the last stf_dag_build(_call) on this

@@ -108,10 +108,12 @@ def dag_io(ntasks: int):
 
 
 def dag_io2(ntasks: int):
-    """Second operand pair (L_i,k+1, L_j,k+1 buffers) of merged GEMM tasks, else (-1, -1)."""
-    IO = (ctypes.c_int64 * (2 * max(1, ntasks)))()
+    """Further operand pairs of merged GEMM tasks: per task a list of (L_i,k+u, L_j,k+u)
+    buffer pairs, u = 1.. (empty for a single update)."""
+    IO = (ctypes.c_int64 * (6 * max(1, ntasks)))()
     check(_abi.stf_dag_tasks_io2(ntasks, IO), "stf_dag_tasks_io2")
-    return [(IO[2 * t], IO[2 * t + 1]) for t in range(ntasks)]
+    return [[(IO[6 * t + 2 * u], IO[6 * t + 2 * u + 1]) for u in range(3) if IO[6 * t + 2 * u] >= 0]
+            for t in range(ntasks)]
 
 
 def dag_mirrors(ntasks: int):

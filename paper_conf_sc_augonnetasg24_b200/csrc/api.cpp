@@ -59,6 +59,7 @@ const std::vector<OptDesc>& option_table() {
       {"trsm_rows", "STF_TRSM_ROWS", &Options::trsm_rows, 32, 128, true},
       {"trsm_res_split", "STF_TRSM_RES_SPLIT", &Options::trsm_res_split, 1, 4, true},
       {"gemm_merge", "STF_GEMM_MERGE", &Options::gemm_merge, 0, 64, true},
+      {"gemm_group", "STF_GEMM_GROUP", &Options::gemm_group, 2, 4, true},
       {"order_mode", "STF_ORDER_MODE", &Options::order_mode, -1, 2, true},
       {"order_tail", "STF_ORDER_TAIL", &Options::order_tail, -1, INT64_MAX, true},
       {"order_asap", "STF_ORDER_ASAP", &Options::order_asap, 0, 1, true},
@@ -496,10 +497,8 @@ int stf_dag_tasks_io(int64_t cap_tasks, int64_t* io) {
 int64_t stf_dag_tasks_io2(int64_t cap_tasks, int64_t* io2) {
   g_err.clear();
   const stf::Plan& plan = g_dag_plan;
-  for (size_t t = 0; t < plan.tasks.size() && (int64_t)t < cap_tasks; ++t) {
-    io2[2 * t] = plan.tasks[t].in2[0];
-    io2[2 * t + 1] = plan.tasks[t].in2[1];
-  }
+  for (size_t t = 0; t < plan.tasks.size() && (int64_t)t < cap_tasks; ++t)
+    for (int u = 0; u < 6; ++u) io2[6 * t + u] = plan.tasks[t].xin[u];
   return plan.nmerged;
 }
 

@@ -88,8 +88,9 @@ stf::PlanOptions call_plan_options(const Options& o, int64_t n, int64_t nb, int 
   po.push = o.push != 0 && o.trsm >= 2;
   po.push_potrf = po.push && o.dataflow != 0;  // the dataflow POTRF kernel stores into replicas
   po.data_plane = po.push ? (int)o.push : 0;
-  // merged tile updates need whole k tiles of 32 for the second pair (gemm_nt2)
+  // merged tile updates need whole k tiles of 32 per operand pair (gemm_nt_multi)
   po.gemm_merge = (nb % 32 == 0) ? (int)o.gemm_merge : 0;
+  po.gemm_group = (int)o.gemm_group;
   po.ooc_order = (int)o.ooc_order;
   // Scheduling model of the submission order (plan.cpp reorder_list), in units of
   // one nb^3 GEMM task's duration while `width` of them share the GPU: a tile
@@ -257,11 +258,19 @@ struct Lowerer {
                  "SYRK launch");
         return 0;
       case stf::K_GEMM:
-        if (t.in2[0] >= 0)  // merged GEMM(i,j,k) + GEMM(i,j,k+1): one k sweep of 2 nb
-          CUDA_TRY(stfk::gemm_nt2(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[1]],
-                                  nb, (int)nb, X.buf[(size_t)t.in2[0]], nb, X.buf[(size_t)t.in2[1]], nb,
-                                  X.buf[(size_t)t.out], nb, 0, 0),
+        if (t.nupd > 1) {  // merged GEMM(i,j,k) .. GEMM(i,j,k+nupd-1): one k sweep of nupd nb
+          const double* As[4];
+          const double* Bs[4];
+          As[0] = X.buf[(size_t)t.in[0]];
+          Bs[0] = X.buf[(size_t)t.in[1]];
+          for (int u = 1; u < t.nupd; ++u) {
+            As[u] = X.buf[(size_t)t.xin[2 * (u - 1)]];
+            Bs[u] = X.buf[(size_t)t.xin[2 * (u - 1) + 1]];
+          }
+          CUDA_TRY(stfk::gemm_nt_multi(s, prio, (int)nb, (int)nb, (int)nb, t.nupd, As, nb, Bs, nb, X.buf[(size_t)t.out], nb,
+                                       0, 0),
                    "GEMM launch");
+        }
         else
           CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[1]],
                                  nb, X.buf[(size_t)t.out], nb, 0),

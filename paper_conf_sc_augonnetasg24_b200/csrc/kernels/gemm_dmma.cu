@@ -28,6 +28,7 @@
 
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 #include <mutex>
 
 #include "ptx.cuh"
@@ -65,19 +66,24 @@ __device__ __forceinline__ uint32_t swz_off(int r, int k) {
   return box * g::BOX_BYTES + k * 128 + ((((mi >> 1) ^ (k & 7)) << 4) | ((mi & 1) << 3));
 }
 
-// k-tile kt of the operand pair: kt < KT1 from (tmA, tmB), else tile kt - KT1 of the
-// second pair (tmA2, tmB2): a merged update C -= A B^T + A2 B2^T in one k sweep
+// Further operand pairs of a merged update C -= A B^T + A2 B2^T + ... (up to 4
+// pairs, each K deep): consecutive tile updates in one k sweep.
+struct ExtraPairs {
+  CUtensorMap a[3], b[3];
+  int npairs;  // total pairs including (tmA, tmB): 1..4
+};
+
+// k-tile kt: pair p = kt / KT1 (p = 0: tmA, tmB), tile kt - p KT1 of that pair
 template <class g>
 __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                                           const CUtensorMap* tmA2, const CUtensorMap* tmB2, int KT1, int m0, int n0,
-                                           int kt, uint64_t* full) {
+                                           const ExtraPairs* ex, int KT1, int m0, int n0, int kt, uint64_t* full) {
   mbar_arrive_expect_tx(&full[s], g::STAGE_BYTES);
   uint8_t* sa = smem + s * g::STAGE_BYTES;
   uint8_t* sb = sa + g::A_BYTES;
-  const bool second = kt >= KT1;
-  const CUtensorMap* ma = second ? tmA2 : tmA;
-  const CUtensorMap* mb = second ? tmB2 : tmB;
-  const int kk = second ? kt - KT1 : kt;
+  const int pr = kt / KT1;
+  const CUtensorMap* ma = pr == 0 ? tmA : &ex->a[pr - 1];
+  const CUtensorMap* mb = pr == 0 ? tmB : &ex->b[pr - 1];
+  const int kk = kt - pr * KT1;
 #pragma unroll
   for (int b = 0; b < g::BM / g::BOX; ++b) tma_load_2d(sa + b * g::BOX_BYTES, ma, m0 + b * g::BOX, kk * g::BK, &full[s]);
 #pragma unroll
@@ -92,8 +98,8 @@ __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorM
 template <int WM, int WN, class g>
 __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
     gemm_nt_dmma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                        const __grid_constant__ CUtensorMap tmA2, const __grid_constant__ CUtensorMap tmB2,
-                        double* __restrict__ C, int64_t ldc, int M, int N, int K, int K2, int lower) {
+                        const __grid_constant__ ExtraPairs ex, double* __restrict__ C, int64_t ldc, int M, int N,
+                        int K, int lower) {
   constexpr int NCW = (g::BM / WM) * (g::BN / WN);
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // keep the pointer derived from the __shared__ array (integer offset only) so
@@ -126,22 +132,22 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
   }
   const int m0 = tm * g::BM, n0 = tn * g::BN;
   const int KT1 = (K + g::BK - 1) / g::BK;
-  const int KT = KT1 + (K2 + g::BK - 1) / g::BK;
+  const int KT = KT1 * ex.npairs;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
-    if (K2 > 0) {
-      tma_prefetch_desc(&tmA2);
-      tma_prefetch_desc(&tmB2);
+    for (int pr = 1; pr < ex.npairs; ++pr) {
+      tma_prefetch_desc(&ex.a[pr - 1]);
+      tma_prefetch_desc(&ex.b[pr - 1]);
     }
     for (int s = 0; s < g::STAGES; ++s) {
       mbar_init(&full[s], 1);
       released[s] = 0;
     }
     fence_barrier_init();
-    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, &tmA2, &tmB2, KT1, m0, n0, kt, full);
+    for (int kt = 0; kt < g::STAGES && kt < KT; ++kt) load_stage<g>(smem, kt, &tmA, &tmB, &ex, KT1, m0, n0, kt, full);
   }
   __syncthreads();
 
@@ -213,7 +219,7 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
         released[s] = 0;
         __threadfence_block();
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        load_stage<g>(smem, s, &tmA, &tmB, &tmA2, &tmB2, KT1, m0, n0, kt + g::STAGES, full);
+        load_stage<g>(smem, s, &tmA, &tmB, &ex, KT1, m0, n0, kt + g::STAGES, full);
       }
     }
   }
@@ -299,15 +305,14 @@ static int syrk64_max() {
 
 template <class G>
 static cudaError_t launch_variant(cudaLaunchConfig_t& cfg, const CUtensorMap& tmA, const CUtensorMap& tmB,
-                                  const CUtensorMap& tmA2, const CUtensorMap& tmB2, double* C, int64_t ldc, int M, int N,
-                                  int K, int K2, int lower) {
+                                  const ExtraPairs& ex, double* C, int64_t ldc, int M, int N, int K, int lower) {
   cfg.dynamicSmemBytes = G::SMEM_BYTES;
   if (gemm_warps() == 16) {
     cfg.blockDim = dim3(512, 1, 1);
-    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, G>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, G>, tmA, tmB, ex, C, ldc, M, N, K, lower);
   }
   cfg.blockDim = dim3(256, 1, 1);
-  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, G>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+  return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, G>, tmA, tmB, ex, C, ldc, M, N, K, lower);
 }
 
 cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
@@ -317,31 +322,38 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
 
 cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
                           const double* B, int64_t ldb, double* C, int64_t ldc, int lower, int small) {
-  return gemm_nt2(stream, prio, M, N, K, A, lda, B, ldb, 0, nullptr, 0, nullptr, 0, C, ldc, lower, small);
+  const double* As[1] = {A};
+  const double* Bs[1] = {B};
+  return gemm_nt_multi(stream, prio, M, N, K, 1, As, lda, Bs, ldb, C, ldc, lower, small);
 }
 
-cudaError_t gemm_nt2(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda, const double* B,
-                     int64_t ldb, int K2, const double* A2, int64_t lda2, const double* B2, int64_t ldb2, double* C,
-                     int64_t ldc, int lower, int small) {
+cudaError_t gemm_nt_multi(cudaStream_t stream, int prio, int M, int N, int K, int npairs, const double* const* As,
+                          int64_t lda, const double* const* Bs, int64_t ldb, double* C, int64_t ldc, int lower,
+                          int small) {
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
-  if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15) || (lda & 1) || (ldb & 1))
-    return cudaErrorMisalignedAddress;
-  if (K2 > 0 && ((reinterpret_cast<uintptr_t>(A2) & 15) || (reinterpret_cast<uintptr_t>(B2) & 15) || (lda2 & 1) ||
-                 (ldb2 & 1)))
-    return cudaErrorMisalignedAddress;
+  if (npairs < 1 || npairs > 4) return cudaErrorInvalidValue;
+  if ((lda & 1) || (ldb & 1)) return cudaErrorMisalignedAddress;
+  for (int p = 0; p < npairs; ++p)
+    if ((reinterpret_cast<uintptr_t>(As[p]) & 15) || (reinterpret_cast<uintptr_t>(Bs[p]) & 15))
+      return cudaErrorMisalignedAddress;
   const bool narrow = gemm_narrow() != 0;
   const int bk = narrow ? 32 : gemm_bk();
-  // the second pair starts on a fresh k tile: the first pair's K must fill whole tiles
-  if (K2 > 0 && K % bk) return cudaErrorInvalidValue;
-  CUtensorMap tmA, tmB, tmA2, tmB2;
-  if (!make_operand_map(&tmA, A, M, K, lda, bk) || !make_operand_map(&tmB, B, N, K, ldb, bk))
+  // every pair after the first starts on a fresh k tile: K must fill whole tiles
+  if (npairs > 1 && K % bk) return cudaErrorInvalidValue;
+  CUtensorMap tmA, tmB;
+  if (!make_operand_map(&tmA, As[0], M, K, lda, bk) || !make_operand_map(&tmB, Bs[0], N, K, ldb, bk))
     return cudaErrorInvalidValue;
-  if (K2 > 0) {
-    if (!make_operand_map(&tmA2, A2, M, K2, lda2, bk) || !make_operand_map(&tmB2, B2, N, K2, ldb2, bk))
-      return cudaErrorInvalidValue;
-  } else {
-    tmA2 = tmA;
-    tmB2 = tmB;
+  ExtraPairs ex;
+  memset(&ex, 0, sizeof ex);
+  ex.npairs = npairs;
+  for (int p = 1; p < 4; ++p) {
+    if (p < npairs) {
+      if (!make_operand_map(&ex.a[p - 1], As[p], M, K, lda, bk) || !make_operand_map(&ex.b[p - 1], Bs[p], N, K, ldb, bk))
+        return cudaErrorInvalidValue;
+    } else {
+      ex.a[p - 1] = tmA;
+      ex.b[p - 1] = tmB;
+    }
   }
   cudaLaunchConfig_t cfg = {};
   cudaLaunchAttribute attr[1];
@@ -357,10 +369,10 @@ cudaError_t gemm_nt2(cudaStream_t stream, int prio, int M, int N, int K, const d
     ++launch_count();
     if (s64_warps() == 8) {  // 32 x 16 warp tiles: two warps per SM sub-partition
       cfg.blockDim = dim3(256, 1, 1);
-      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 16, CfgS64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 16, CfgS64>, tmA, tmB, ex, C, ldc, M, N, K, lower);
     }
     cfg.blockDim = dim3(128, 1, 1);
-    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgS64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgS64>, tmA, tmB, ex, C, ldc, M, N, K, lower);
   }
   const int tM = (M + 127) / 128, tN = narrow ? (N + 63) / 64 : (N + 127) / 128;
   cfg.gridDim = lower ? dim3(narrow ? tM * (tM + 1) : tM * (tM + 1) / 2, 1, 1) : dim3(tM, tN, 1);
@@ -369,13 +381,13 @@ cudaError_t gemm_nt2(cudaStream_t stream, int prio, int M, int N, int K, const d
     cfg.dynamicSmemBytes = CfgN64::SMEM_BYTES;
     if (gemm_narrow() == 2) {  // 8 warps of 32 x 32, 2 CTAs (16 warps) per SM
       cfg.blockDim = dim3(256, 1, 1);
-      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+      return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<32, 32, CfgN64>, tmA, tmB, ex, C, ldc, M, N, K, lower);
     }
     cfg.blockDim = dim3(128, 1, 1);  // 4 warps of 64 x 32
-    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, CfgN64>, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+    return cudaLaunchKernelEx(&cfg, gemm_nt_dmma_kernel<64, 32, CfgN64>, tmA, tmB, ex, C, ldc, M, N, K, lower);
   }
-  if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
-  return launch_variant<CfgK16>(cfg, tmA, tmB, tmA2, tmB2, C, ldc, M, N, K, K2, lower);
+  if (bk == 32) return launch_variant<CfgK32>(cfg, tmA, tmB, ex, C, ldc, M, N, K, lower);
+  return launch_variant<CfgK16>(cfg, tmA, tmB, ex, C, ldc, M, N, K, lower);
 }
 
 template <class G>

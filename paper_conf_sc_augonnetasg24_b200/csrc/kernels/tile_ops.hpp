@@ -22,13 +22,14 @@ cudaError_t gemm_nt(cudaStream_t stream, int prio, int M, int N, int K, const do
 // latency-critical updates; same per-element k order, same bits).
 cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda,
                           const double* B, int64_t ldb, double* C, int64_t ldc, int lower, int small);
-// Merged update C -= A B^T + A2 B2^T in ONE sweep over k (K, then K2; K a multiple
-// of the k tile): the accumulators carry across the two pairs, so the result is
-// bit-identical to two gemm_nt calls in that order, with one C load/store and one
-// pipeline ramp instead of two (two consecutive tile updates GEMM(i,j,k), GEMM(i,j,k+1)).
-cudaError_t gemm_nt2(cudaStream_t stream, int prio, int M, int N, int K, const double* A, int64_t lda, const double* B,
-                     int64_t ldb, int K2, const double* A2, int64_t lda2, const double* B2, int64_t ldb2, double* C,
-                     int64_t ldc, int lower, int small);
+// Merged update C -= A_0 B_0^T + ... + A_{p-1} B_{p-1}^T (npairs <= 4, each pair K
+// deep, K a multiple of the k tile) in ONE sweep over k: the accumulators carry
+// across the pairs, so the result is bit-identical to npairs gemm_nt calls in that
+// order, with one C load/store and one pipeline ramp instead of npairs
+// (consecutive tile updates GEMM(i,j,k), GEMM(i,j,k+1), ... of one task).
+cudaError_t gemm_nt_multi(cudaStream_t stream, int prio, int M, int N, int K, int npairs, const double* const* As,
+                          int64_t lda, const double* const* Bs, int64_t ldb, double* C, int64_t ldc, int lower,
+                          int small);
 
 // K3: B[M x n] <- B * L^-T with L[n x n] lower triangular, non-unit diagonal
 // (side = right, lower, transposed).  Recursive: base blocks of <= 64 columns

@@ -128,24 +128,23 @@ struct Builder {
   }
 
   void compute(int32_t kind, int64_t i, int64_t j, int64_t k, int prio, int64_t ra, int64_t rb, int64_t wi,
-               int64_t wj, int64_t ra2 = -1, int64_t rb2 = -1) {
+               int64_t wj, int nupd = 1, const int64_t* xk = nullptr) {
     const int slot = p.owner(wi, wj);
     const int64_t w = Plan::tile_id(wi, wj);
     int64_t in0 = ra >= 0 ? read_buffer(ra / T, ra % T, slot) : -1;
     int64_t in1 = rb >= 0 ? read_buffer(rb / T, rb % T, slot) : -1;
     Task t{kind, (int32_t)i, (int32_t)j, (int32_t)k, slot, prio, 0, {in0, in1}, w};
-    if (ra2 >= 0) {  // merged GEMM: the second update's operands
-      t.in2[0] = read_buffer(ra2 / T, ra2 % T, slot);
-      t.in2[1] = read_buffer(rb2 / T, rb2 % T, slot);
+    if (nupd > 1) {  // merged GEMM: the operands of updates k+1 .. k+nupd-1
+      t.nupd = nupd;
+      for (int u = 0; u < 2 * (nupd - 1); ++u) t.xin[u] = read_buffer(xk[u] / T, xk[u] % T, slot);
       p.nmerged++;
     }
     t.stream = compute_stream(t);
-    Access acc[5 + 7];
+    Access acc[3 + 6 + 7];
     int n = 0;
     if (in0 >= 0) acc[n++] = {in0, READ};
     if (in1 >= 0) acc[n++] = {in1, READ};
-    if (t.in2[0] >= 0) acc[n++] = {t.in2[0], READ};
-    if (t.in2[1] >= 0) acc[n++] = {t.in2[1], READ};
+    for (int u = 0; u < 2 * (t.nupd - 1); ++u) acc[n++] = {t.xin[u], READ};
     acc[n++] = {w, RW};
     std::vector<int> cons;
     if (kind == K_TRSM && p.opt.push) cons = consumers_of_panel_tile(wi, wj);
@@ -196,10 +195,13 @@ struct Builder {
       return d <= 1 ? 4 : d == 2 ? 3 : d <= 4 ? 2 : d <= 8 ? 1 : 0;
     };
     auto P = [&](int lv) { return prio ? lv : 0; };
-    // merged GEMMs: a tile (i, j) at least D columns right of panel k+1 (k even)
-    // receives its updates k and k+1 as one task at step k+1
-    const int64_t D = p.opt.lookahead ? p.opt.gemm_merge : 0;
-    auto deferred = [&](int64_t j, int64_t k) { return D > 0 && (k % 2) == 0 && k + 1 < T && j >= k + 1 + D; };
+    // merged GEMMs: the updates of tile (i, j) from panels gG .. gG+G-1 become one
+    // task at step gG+G-1 when the tile is at least D columns right of that panel
+    const int64_t D = p.opt.lookahead ? p.opt.gemm_merge : 0, G = std::max(1, std::min(4, p.opt.gemm_group));
+    auto merged = [&](int64_t j, int64_t k) {  // update k of column j belongs to a merged group
+      const int64_t last = k / G * G + G - 1;
+      return D > 0 && G > 1 && last < j && j >= last + D;
+    };
     for (int64_t k = 0; k < T; ++k) {
       compute(K_POTRF, k, k, k, P(5), -1, -1, k, k);
       for (int64_t i = k + 1; i < T; ++i)
@@ -207,13 +209,18 @@ struct Builder {
       for (int64_t i = k + 1; i < T; ++i) {
         compute(K_SYRK, i, i, k, P(i == k + 1 ? 5 : level(i - k)), key(i, k), -1, i, i);
         for (int64_t j = k + 1; j < i; ++j) {
-          if (deferred(j, k)) continue;  // update k goes with update k+1 (next step)
-          if (k >= 1 && deferred(j, k - 1))
-            compute(K_GEMM, i, j, k - 1, P(level(j - k)), key(i, k - 1), key(j, k - 1), i, j, key(i, k), key(j, k));
-          else
+          if (!merged(j, k)) {
             compute(K_GEMM, i, j, k, P(level(j - k)), key(i, k), key(j, k), i, j);
-        }
-      }
+          } else if (k % G == G - 1) {  // the group's last panel: all G updates now
+            const int64_t f = k - G + 1;
+            int64_t x[6];
+            for (int64_t u = 1; u < G; ++u) {
+              x[2 * (u - 1)] = key(i, f + u);
+              x[2 * (u - 1) + 1] = key(j, f + u);
+            }
+            compute(K_GEMM, i, j, f, P(level(j - k)), key(i, f), key(j, f), i, j, (int)G, x);
+          }
+        }      }
       if (!p.opt.lookahead && k + 1 < T) {
         std::vector<Access> acc;
         for (int64_t d = 0; d < p.ntiles(); ++d) acc.push_back({d, RW});

@@ -39,8 +39,8 @@ struct Task {
   int64_t out;       // buffer id written
   int32_t nmir;      // fused push (NEXT-3): replica buffers written by the same kernel
   int64_t mir[7];
-  int64_t in2[2] = {-1, -1};  // merged GEMM: the second update's operands (GEMM(i,j,k) and GEMM(i,j,k+1)
-                              // in one task: in = L_ik, L_jk; in2 = L_i,k+1, L_j,k+1), else -1
+  int32_t nupd = 1;           // merged GEMM: tile updates k, k+1, .., k+nupd-1 in one task
+  int64_t xin[6] = {-1, -1, -1, -1, -1, -1};  // their operands after the first: (L_i,k+u, L_j,k+u), u = 1..3
 };
 
 struct PlanOptions {
@@ -68,8 +68,9 @@ struct PlanOptions {
   bool push = false;       // TRSM(i,k) writes L_ik into its consumers' replicas itself (fused
                            // push, NEXT-3) instead of COPY tasks at the first remote read
   int data_plane = 0;      // requested data plane (statistics): 0 COPY, 1 fused push, 2 multicast
-  int gemm_merge = 0;      // > 0: GEMM(i,j,k) and GEMM(i,j,k+1) (k even) of a tile at least this many
-                           // columns right of panel k+1 become one task at step k+1 (one K = 2 nb sweep)
+  int gemm_merge = 0;      // D > 0: the updates of a tile from a group of gemm_group consecutive panels
+  int gemm_group = 2;      // g G .. g G + G - 1 become one task at step g G + G - 1 when the tile is at
+                           // least D columns right of that panel (one K = G nb sweep)
   bool push_potrf = false; // with push: POTRF(k) also writes L_kk into the replicas of the
                            // slots running TRSM(i,k) (the dataflow POTRF kernel's epilogue)
   int64_t frames = 0;      // > 0 (one slot, with_load/with_store): memory-capped out-of-core

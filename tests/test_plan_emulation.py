@@ -20,13 +20,14 @@ import synth
 NB = 4  # tile order for the emulation (values are irrelevant to the schedule)
 
 
-def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0):
+def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0, group=2):
     """Plan of stf_dag_build with these options (gemm_merge restored to its default 2 after)."""
     stf.set_option("mem_cap_tiles", frames)
     stf.set_option("lookahead", lookahead)
     stf.set_option("ooc_order", ooc_order)
     stf.set_option("push", push)
     stf.set_option("gemm_merge", merge)
+    stf.set_option("gemm_group", group)
     try:
         edges, kinds, ijk, st = stf.dag(T, p, q)
         io, nbuf = stf.dag_io(len(kinds))
@@ -37,6 +38,7 @@ def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0):
         stf.set_option("ooc_order", -1)
         stf.set_option("push", 0)
         stf.set_option("gemm_merge", 2)
+        stf.set_option("gemm_group", 2)
     return edges, kinds, ijk, io, nbuf, st
 
 
@@ -85,8 +87,8 @@ def _emulate(T, A, kinds, ijk, io, nbuf, edges, order_seed, host_resident):
             buf[w][:, :] = oracle.tile_syrk(buf[w], buf[r0])
         elif kd == "GEMM":
             buf[w][:, :] = oracle.tile_gemm(buf[w], buf[r0], buf[r1])
-            if _IO2 and _IO2[t][0] >= 0:  # merged task: update k+1 right after update k
-                buf[w][:, :] = oracle.tile_gemm(buf[w], buf[_IO2[t][0]], buf[_IO2[t][1]])
+            for a2, b2 in (_IO2[t] if _IO2 else []):  # merged task: updates k+1, .. right after update k
+                buf[w][:, :] = oracle.tile_gemm(buf[w], buf[a2], buf[b2])
         elif kd == "COPY":
             buf[w][:, :] = buf[r0]
         elif kd == "LOAD":
@@ -242,8 +244,8 @@ def test_call_plans_any_topological_order(n, nb, kind, p, q):
     T = n // nb
     edges, kinds, ijk, io, nbuf, st = _call_plan(n, nb, kind, p, q)
     NT = T * (T + 1) // 2
-    # merged GEMM tasks (gemm_merge, device-resident plans) carry two tile updates each
-    assert st["tasks"] + st["merged_gemms"] == T + T * (T - 1) + T * (T - 1) * (T - 2) // 6
+    # merged GEMM tasks (gemm_merge, device-resident plans) carry several tile updates each
+    assert st["tasks"] + sum(len(x) for x in _IO2) == T + T * (T - 1) + T * (T - 1) * (T - 2) // 6
     host = kind == stf.STF_DESC_HOST_COLMAJOR
     if host and p * q == 1 and T >= 16:
         assert st["frames"] == NT  # host_stream: one frame per tile, nothing evicted
@@ -288,18 +290,20 @@ def test_out_of_core_rejects_fence_ablation():
         stf.set_option("lookahead", 1)
 
 
-@pytest.mark.parametrize("T,p,q,merge,push", [(8, 1, 1, 1, 0), (9, 1, 1, 3, 0), (12, 2, 2, 2, 0), (12, 2, 4, 3, 1),
-                                             (10, 1, 8, 1, 0), (16, 1, 1, 3, 0)])
-def test_merged_gemm_plans_any_topological_order(T, p, q, merge, push):
+@pytest.mark.parametrize("T,p,q,merge,push,group", [(8, 1, 1, 1, 0, 2), (9, 1, 1, 3, 0, 2), (12, 2, 2, 2, 0, 2),
+                                                   (12, 2, 4, 3, 1, 2), (10, 1, 8, 1, 0, 2), (16, 1, 1, 3, 0, 2),
+                                                   (16, 1, 1, 1, 0, 3), (17, 2, 2, 2, 1, 4), (13, 1, 1, 1, 0, 4)])
+def test_merged_gemm_plans_any_topological_order(T, p, q, merge, push, group):
     """gemm_merge: GEMM(i,j,k) and GEMM(i,j,k+1) of far tiles as one task (two
     consecutive updates in one k sweep): the plan stays a correct STF DAG -- the
     oracle's bits in random orders -- with fewer GEMM tasks."""
     A = synth.spd_matrix(17, T * NB)
     e0, k0, _, _, _, st0 = _plan(T, p, q, push=push)
-    edges, kinds, ijk, io, nbuf, st = _plan(T, p, q, push=push, merge=merge)
+    edges, kinds, ijk, io, nbuf, st = _plan(T, p, q, push=push, merge=merge, group=group)
     assert st["merged_gemms"] > 0 and st0["merged_gemms"] == 0
-    assert st["tasks"] == st0["tasks"] - st["merged_gemms"]
-    assert kinds.count("GEMM") == k0.count("GEMM") - st["merged_gemms"]
+    extra = sum(len(x) for x in _IO2)  # updates carried by merged tasks beyond their first
+    assert kinds.count("GEMM") + extra == k0.count("GEMM")
+    assert st["tasks"] + extra == st0["tasks"]
     ref = _reference(T, A)
     for seed in (-1, 1, 2):
         got = _emulate(T, A, kinds, ijk, io, nbuf, edges, seed, host_resident=False)
