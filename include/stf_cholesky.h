@@ -116,8 +116,8 @@ const char *stf_last_error(void);
  *                           column parts, right-looking, with a GEMM after each (more CTAs on the
  *                           critical path); 1: one launch
  *   "gemm_merge" STF_GEMM_MERGE D >= 0 (default 2): the tile updates GEMM(i,j,k) of a group of
- *                           G consecutive panels k = gG .. gG+G-1 ("gemm_group" G = 2..4, default
- *                           2) become ONE task at step gG+G-1 when the tile is at least D columns
+ *                           G consecutive panels k = gG .. gG+G-1 ("gemm_group" G = 2..4; default
+ *                           -1: 4 when n/nb >= 48, else 2) become ONE task at step gG+G-1 when the tile is at least D columns
  *                           right of that panel (one k sweep of G nb: one C load/store and
  *                           pipeline ramp instead of G; the same operations per element, same
  *                           bits); 0 = off.  Not with lookahead = 0.

@@ -59,7 +59,7 @@ const std::vector<OptDesc>& option_table() {
       {"trsm_rows", "STF_TRSM_ROWS", &Options::trsm_rows, 32, 128, true},
       {"trsm_res_split", "STF_TRSM_RES_SPLIT", &Options::trsm_res_split, 1, 4, true},
       {"gemm_merge", "STF_GEMM_MERGE", &Options::gemm_merge, 0, 64, true},
-      {"gemm_group", "STF_GEMM_GROUP", &Options::gemm_group, 2, 4, true},
+      {"gemm_group", "STF_GEMM_GROUP", &Options::gemm_group, -1, 4, true},
       {"order_mode", "STF_ORDER_MODE", &Options::order_mode, -1, 2, true},
       {"order_tail", "STF_ORDER_TAIL", &Options::order_tail, -1, INT64_MAX, true},
       {"order_asap", "STF_ORDER_ASAP", &Options::order_asap, 0, 1, true},
@@ -90,6 +90,7 @@ int check_option(const OptDesc& d, int64_t v, int pool_streams) {
   if (n == "ooc_budget_pct" && v != -1 && v < 10) return fail(-105, "ooc_budget_pct must be -1 (auto) or in [10, 95]");
   if (n == "order_mode" && v == 1) return fail(-105, "order_mode must be -1 (auto), 0 (program) or 2 (list)");
   if (n == "trsm_res_split" && v == 3) return fail(-105, "trsm_res_split must be 1, 2 or 4");
+  if (n == "gemm_group" && v >= 0 && v < 2) return fail(-105, "gemm_group must be -1 (auto) or 2..4");
   if (n == "streams" && pool_streams > 0 && v > pool_streams)
     return fail(-105, "streams=%lld exceeds the pool created at init (%d)", (long long)v, pool_streams);
   return 0;

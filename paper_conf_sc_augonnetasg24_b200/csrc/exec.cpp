@@ -90,7 +90,10 @@ stf::PlanOptions call_plan_options(const Options& o, int64_t n, int64_t nb, int 
   po.data_plane = po.push ? (int)o.push : 0;
   // merged tile updates need whole k tiles of 32 per operand pair (gemm_nt_multi)
   po.gemm_merge = (nb % 32 == 0) ? (int)o.gemm_merge : 0;
-  po.gemm_group = (int)o.gemm_group;
+  // 4 updates per merged task on long factorisations (n = 65536, T = 64: +0.97% over none, +0.3%
+  // over 2), 2 on shorter ones (n = 32768, T = 32: +0.47% vs +0.23% with 4;
+  // profiles/r02/gemm_merge_sweep.txt)
+  po.gemm_group = o.gemm_group > 0 ? (int)o.gemm_group : (T >= 48 ? 4 : 2);
   po.ooc_order = (int)o.ooc_order;
   // Scheduling model of the submission order (plan.cpp reorder_list), in units of
   // one nb^3 GEMM task's duration while `width` of them share the GPU: a tile

@@ -71,7 +71,7 @@ struct Options {
   int64_t trsm_rows = 128;     // row panel: rows per CTA (32, 64, 128)
   int64_t trsm_res_split = 2;  // resident-panel TRSMs in 2 (or 4) column parts with GEMMs between; 1 = one launch
   int64_t gemm_merge = 2;      // D > 0: merged tile updates for tiles >= D columns right of the panel
-  int64_t gemm_group = 2;      // updates per merged GEMM task (2..4)
+  int64_t gemm_group = -1;     // updates per merged GEMM task (2..4; -1 auto: 4 when T >= 48, else 2)
   int64_t order_mode = -1;     // submission order: 0 program, 2 list scheduling, -1 auto (nb >= 512 -> 2)
   int64_t order_tail = -1;     // order_mode 2: re-order only the last steps (0 all, -1 auto)
   int64_t order_asap = 0;      // earliest-start submission order (order_mode 0 only)

@@ -92,7 +92,7 @@ OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (3, 1), "streams": (32, 
            "order_mode": (-1, 2), "order_tail": (-1, 0), "order_asap": (0, 1), "sched_width": (0, 3), "prio_mode": (0, 2),
            "ooc_reorder": (1, 0), "dev_order": (0, 1), "ooc_budget_pct": (-1, 40), "host_stream_budget_pct": (90, 75),
            "host_eager": (0, 1), "mem_cap_tiles": (0, 10), "ooc_order": (-1, 0), "host_stream": (1, 0), "pdl": (0, 1),
-           "debug_skip": (0, 8), "debug_trace": (0, 1), "nvtx": (0, 1), "gemm_merge": (2, 0), "gemm_group": (2, 4)}
+           "debug_skip": (0, 8), "debug_trace": (0, 1), "nvtx": (0, 1), "gemm_merge": (2, 0), "gemm_group": (-1, 4)}
 
 
 @pytest.mark.parametrize("name,value", [("trsm_rows", 48), ("mem_cap_tiles", 2), ("push", 3), ("order_mode", 1),

@@ -38,7 +38,7 @@ def _plan(T, p, q, frames=0, lookahead=1, ooc_order=1, push=0, merge=0, group=2)
         stf.set_option("ooc_order", -1)
         stf.set_option("push", 0)
         stf.set_option("gemm_merge", 2)
-        stf.set_option("gemm_group", 2)
+        stf.set_option("gemm_group", -1)
     return edges, kinds, ijk, io, nbuf, st
 
 
