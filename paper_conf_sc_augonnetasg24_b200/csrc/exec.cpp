@@ -399,8 +399,9 @@ struct Lowerer {
       if (X.mp) {
         // inputs that are replicas here were written by another process: wait
         // (on the device, no host round trip) for the producer's flag
-        for (int a = 0; a < 2; ++a) {
-          const int64_t b = task.in[a];
+        // (every operand: in[] and, for a merged GEMM, the further pairs xin[])
+        for (int a = 0; a < 2 + 2 * (task.nupd - 1); ++a) {
+          const int64_t b = a < 2 ? task.in[a] : task.xin[a - 2];
           if (b >= 0 && P.buffers[(size_t)b].replica && task.kind != stf::K_COPY) {
             const CUresult cr = g_wait_value32((CUstream)s, (CUdeviceptr)(X.local_flags + X.flag_idx[(size_t)b]),
                                                X.epoch, CU_STREAM_WAIT_VALUE_GEQ);
