@@ -111,7 +111,7 @@ const char *stf_last_error(void);
  *   "trsm_split" STF_TRSM_SPLIT P in [1,16]: non-critical row-panel TRSMs run right-looking
  *                           over P column blocks (panel kernel + GEMM updates; default 4)
  *   "trsm_res_tail" STF_TRSM_RES_TAIL C >= 0: with trsm 3, every TRSM(i,k) of a panel step
- *                           whose trailing order n - k nb <= C uses the resident panel (default 8192)
+ *                           whose trailing order n - k nb <= C uses the resident panel (default 4096: n = 8192 +7%, profiles/r02/pdl_and_tail.txt)
  *   "trsm_res_split" STF_TRSM_RES_SPLIT 2 (default) or 4: a resident-panel TRSM runs as that many
  *                           column parts, right-looking, with a GEMM after each (more CTAs on the
  *                           critical path); 1: one launch
@@ -172,7 +172,18 @@ const char *stf_last_error(void);
  *                           right-looking plan with its LOAD/STORE tasks.  Same bits
  *   "host_stream_budget_pct" STF_HOST_STREAM_BUDGET_PCT block budget of that plan (default 90)
  *   "host_eager" STF_HOST_EAGER 1: HOST_COLMAJOR calls on pinned memory lowered eagerly
- *   "pdl"      STF_PDL      1: programmatic dependent launch between same-stream chain kernels
+ *   "pdl"      STF_PDL      1 (default): the panel chain POTRF(k) -> TRSM(k+1,k) -> SYRK(k+1,k)
+ *                           overlaps through programmatic dependent launch when the three
+ *                           share a slot and stream (graph backend, dataflow POTRF,
+ *                           trsm = 3, nb % 64 == 0, nb <= 1024): the TRSM reads L_kk block by
+ *                           block as the POTRF publishes it, the SYRK reads L_{k+1,k} column
+ *                           block by column block as the TRSM's CTAs finish them (device
+ *                           flags, acquire/release).  The TRSM(k+1,k) is then one
+ *                           resident-panel launch (trsm_res_split does not apply to it) in
+ *                           every grid, so the bits do not depend on where it runs.  Same
+ *                           bits with 0 (no overlap)
+ *   "pdl_lead" STF_PDL_LEAD 64-block steps before its end at which a chain kernel lets its
+ *                           dependent launch (default 8; >= nb/64: at its start)
  *   "debug_skip" STF_DEBUG_SKIP bit mask (or names potrf,trsm,syrk,gemm,copy,trsm_as_gemm,
  *                           trsm_as_half_gemm) of task kinds NOT launched: timing what-ifs only,
  *                           results invalid

@@ -49,7 +49,11 @@ int stf_kernel_potrf(int64_t n, double *A, int64_t lda, int64_t *info);
  * recorded on that same stream; *avg_ms = mean launch duration.  Inputs are
  * generated on the device (SPD generator) and restored (untimed) before each
  * TRSM / POTRF launch.  kind: 0 GEMM C[MxN] -= A[MxK] B[NxK]^T, 1 SYRK (N = M),
- * 2 TRSM B[MxN] <- B L^-T (K ignored), 3 POTRF of an M x M tile.
+ * 2 TRSM B[MxN] <- B L^-T (K ignored), 3 POTRF of an M x M tile, 4 one step of the
+ * critical chain POTRF(k) -> TRSM(k+1,k) -> SYRK(k+1,k) on M x M tiles (M a
+ * multiple of 64, <= 1024; N, K ignored) lowered as in a factorisation: one
+ * stream, captured into a graph, TRSM overlapping the POTRF when option pdl = 1;
+ * the time is taken by event nodes of that graph around the three kernels.
  * Returns 0 / -4 / -101 / -103. */
 int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double *avg_ms);
 

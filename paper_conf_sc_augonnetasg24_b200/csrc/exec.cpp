@@ -139,6 +139,46 @@ stf::PlanOptions call_plan_options(const Options& o, int64_t n, int64_t nb, int 
   return po;
 }
 
+// the node the capture of stream s would hang the next launch on (null when not capturing
+// or when that is not exactly one node)
+cudaGraphNode_t capture_last_node(cudaStream_t s) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  const cudaGraphNode_t* deps = nullptr;
+  size_t nd = 0;
+  if (cudaStreamGetCaptureInfo_v3(s, &st, nullptr, nullptr, &deps, nullptr, &nd) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return (st == cudaStreamCaptureStatusActive && nd == 1) ? deps[0] : nullptr;
+}
+// Turn the capture edge from kernel node `from` (a current dependency of stream s)
+// into a programmatic one: the next kernel captured on s may launch once every CTA
+// of `from` has executed griddepcontrol.launch_dependents (or exited).  The other
+// dependencies keep full-completion edges.  No-op when `from` is not a dependency.
+int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  const cudaGraphNode_t* deps = nullptr;
+  const cudaGraphEdgeData* ed = nullptr;
+  size_t nd = 0;
+  CUDA_TRY(cudaStreamGetCaptureInfo_v3(s, &st, nullptr, nullptr, &deps, &ed, &nd), "capture info");
+  if (st != cudaStreamCaptureStatusActive) return 0;
+  std::vector<cudaGraphNode_t> d(deps, deps + nd);
+  std::vector<cudaGraphEdgeData> e(nd);
+  bool found = false;
+  for (size_t i = 0; i < nd; ++i) {
+    e[i] = ed ? ed[i] : cudaGraphEdgeData{};
+    if (d[i] == from) {
+      e[i].from_port = cudaGraphKernelNodePortProgrammatic;
+      e[i].type = cudaGraphDependencyTypeProgrammatic;
+      found = true;
+    }
+  }
+  if (!found) return 0;
+  CUDA_TRY(cudaStreamUpdateCaptureDependencies_v2(s, d.data(), e.data(), nd, cudaStreamSetCaptureDependencies),
+           "programmatic capture edge");
+  return 0;
+}
+
 // ------------------------------------------------------------------ lowering
 namespace {
 
@@ -196,8 +236,13 @@ struct Lowerer {
       case stf::K_POTRF:
         if (X.opt.dataflow) {
           stfk::Mirrors mir = mirrors_of(t);  // fused push of L_kk (NEXT-3): final blocks also into the replicas
-          CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir),
+          // pdl: the chain CTA releases the dependent TRSM(k+1,k) pdl_lead 64-block steps before its end
+          const int nbk = (int)((nb + 63) / 64);
+          const int trig = X.opt.pdl ? (int)std::max<int64_t>(0, nbk - X.opt.pdl_lead) : -1;
+          CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir,
+                                    nullptr, 0, trig),
                    "POTRF launch");
+          if (!X.cap_node.empty()) X.cap_node[tidx] = capture_last_node(s);
         } else
           CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
                    "POTRF launch");
@@ -211,8 +256,29 @@ struct Lowerer {
                    "TRSM what-if");
           return 0;
         }
-        if (X.opt.trsm == 3 && (t.i == t.k + 1 || X.n - t.k * nb <= X.opt.trsm_res_tail) &&
+        if (X.opt.pdl && X.opt.trsm == 3 && t.i == t.k + 1 &&
             stfk::trsm_res_supported((int)nb, X.buf[(size_t)t.in[0]], nb)) {
+          // pdl: TRSM(k+1,k) in one resident-panel launch that reads the blocks of L_kk as
+          // the dataflow POTRF(k) publishes them; captured behind POTRF(k) on the same
+          // stream, the edge between the two becomes programmatic (the TRSM launches when
+          // the POTRF triggers).  Without a same-stream POTRF(k) (another slot, eager
+          // backend) L_kk is complete at launch and the flags are already final.
+          const int64_t src = X.pdl_src.empty() ? -1 : X.pdl_src[tidx];
+          const int nbk = (int)(nb / 64);
+          const int* pflag = src >= 0 && X.task_ws[(size_t)src] ? X.task_ws[(size_t)src] + 2 : nullptr;
+          if (pflag && !X.cap_node.empty() && X.cap_node[(size_t)src]) {
+            int r = capture_make_programmatic(s, X.cap_node[(size_t)src]);
+            if (r) return r;
+          }
+          // column-block counters for a SYRK(k+1,k) that overlaps this TRSM in turn
+          int* kflag = pflag ? X.task_ws[(size_t)src] + 2 + nbk * nbk : nullptr;
+          const int trig = kflag ? std::max(0, nbk - (int)X.opt.pdl_lead) : -1;
+          CUDA_TRY(stfk::trsm_res(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, &mir,
+                                  nullptr, pflag, nbk, kflag, trig),
+                   "TRSM launch");
+          if (!X.cap_node.empty()) X.cap_node[tidx] = capture_last_node(s);
+        } else if (X.opt.trsm == 3 && (t.i == t.k + 1 || X.n - t.k * nb <= X.opt.trsm_res_tail) &&
+                   stfk::trsm_res_supported((int)nb, X.buf[(size_t)t.in[0]], nb)) {
           // the next panel's TRSM(k+1,k) is on the critical path, and near the end of the
           // factorisation every TRSM is latency-bound: the resident-panel kernel (16 rows per
           // CTA, 4x the CTAs of the row panel, solve overlapped with the updates)
@@ -255,11 +321,25 @@ struct Lowerer {
                    "TRSM launch");
         return 0;
       }
-      case stf::K_SYRK:
-        CUDA_TRY(stfk::gemm_nt(s, prio, (int)nb, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.in[0]],
-                               nb, X.buf[(size_t)t.out], nb, 1),
+      case stf::K_SYRK: {
+        // pdl: SYRK(k+1,k) behind its overlapping TRSM(k+1,k) on the same stream reads
+        // the k columns of L_{k+1,k} as the TRSM's CTAs publish them (programmatic edge)
+        const int64_t src = X.pdl_src.empty() ? -1 : X.pdl_src[tidx];
+        const int* kflag = nullptr;
+        if (src >= 0) {
+          const int nbk = (int)(nb / 64);
+          kflag = X.task_ws[(size_t)X.pdl_src[(size_t)src]] + 2 + nbk * nbk;
+          if (!X.cap_node.empty() && X.cap_node[(size_t)src]) {
+            int r = capture_make_programmatic(s, X.cap_node[(size_t)src]);
+            if (r) return r;
+          }
+        }
+        const double* A = X.buf[(size_t)t.in[0]];
+        CUDA_TRY(stfk::gemm_nt_multi(s, prio, (int)nb, (int)nb, (int)nb, 1, &A, nb, &A, nb, X.buf[(size_t)t.out], nb, 1,
+                                     0, kflag, kflag ? (int)((nb + stfk::kTrsmResRows - 1) / stfk::kTrsmResRows) : 0),
                  "SYRK launch");
         return 0;
+      }
       case stf::K_GEMM:
         if (t.nupd > 1) {  // merged GEMM(i,j,k) .. GEMM(i,j,k+nupd-1): one k sweep of nupd nb
           const double* As[4];
@@ -696,6 +776,33 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
       cudaSetDevice(C.slots[(size_t)s].device);
       CUDA_TRY(stfk::dataflow_prepare((int)X.nb, (int)X.nb, true), "dataflow tables");
       CUDA_TRY(stfk::dataflow_prepare((int)X.nb, (int)X.nb, false), "dataflow tables");
+    }
+  }
+  // pdl: TRSM(k+1,k) that follows its POTRF(k) on the same slot and stream
+  X.pdl_src.assign(P.tasks.size(), -1);
+  X.cap_node.assign(X.opt.graph && X.opt.pdl ? P.tasks.size() : 0, nullptr);
+  if (X.opt.pdl && X.opt.dataflow && X.opt.trsm == 3) {
+    std::vector<int64_t> potrf_of((size_t)T, -1);
+    for (size_t t = 0; t < P.tasks.size(); ++t)
+      if (P.tasks[t].kind == stf::K_POTRF) potrf_of[(size_t)P.tasks[t].k] = (int64_t)t;
+    std::vector<int64_t> trsm_of((size_t)T, -1);
+    for (size_t t = 0; t < P.tasks.size(); ++t) {
+      const stf::Task& a = P.tasks[t];
+      if (a.kind != stf::K_TRSM || a.i != a.k + 1) continue;
+      const int64_t src = potrf_of[(size_t)a.k];
+      if (src >= 0 && P.tasks[(size_t)src].slot == a.slot && P.tasks[(size_t)src].stream == a.stream &&
+          X.nb % 64 == 0 && X.nb <= 1024) {
+        X.pdl_src[t] = src;
+        trsm_of[(size_t)a.k] = (int64_t)t;
+      }
+    }
+    // SYRK(k+1,k) that follows such a TRSM(k+1,k) on the same slot and stream
+    for (size_t t = 0; t < P.tasks.size(); ++t) {
+      const stf::Task& a = P.tasks[t];
+      if (a.kind != stf::K_SYRK || a.i != a.k + 1) continue;
+      const int64_t src = trsm_of[(size_t)a.k];
+      if (src >= 0 && P.tasks[(size_t)src].slot == a.slot && P.tasks[(size_t)src].stream == a.stream)
+        X.pdl_src[t] = src;
     }
   }
   if (X.opt.debug_trace && X.ngpus == 1 && !X.mp) {

@@ -115,8 +115,100 @@ int stf_kernel_potrf(int64_t n, double* A, int64_t lda, int64_t* info) {
   return 0;
 }
 
+// kind 4: one panel step of the critical chain, POTRF(k) -> TRSM(k+1,k) -> SYRK(k+1,k)
+// on nb = M tiles, lowered as in a factorisation (one stream; with the pdl option
+// the TRSM overlaps the POTRF through a programmatic capture edge), captured into a
+// graph with the input restores in front and timing events around the chain.
+static int bench_chain(int64_t M, int reps, double* avg_ms) {
+  if (M % 64 || M > 1024) return fail(-4, "chain bench: M must be a multiple of 64, <= 1024");
+  const Options& o = ctx().opt;
+  const size_t bytes = (size_t)(M * M) * 8;
+  double *A0 = nullptr, *B0 = nullptr, *C0 = nullptr, *A = nullptr, *B = nullptr, *Cm = nullptr;
+  unsigned long long* info = nullptr;
+  int* ws = nullptr;
+  cudaStream_t s = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  cudaError_t e = cudaSuccess;
+  int r = 0;
+  auto step = [&](cudaError_t x) {
+    if (e == cudaSuccess) e = x;
+  };
+  step(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  step(cudaEventCreate(&e0));
+  step(cudaEventCreate(&e1));
+  for (double** p : {&A0, &B0, &C0, &A, &B, &Cm}) step(cudaMalloc(p, bytes));
+  step(cudaMalloc(&info, sizeof *info));
+  step(cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)M, (int)M)));
+  if (e == cudaSuccess) {
+    // A_kk, A_{k+1,k}, A_{k+1,k+1}: blocks of one SPD matrix of order 2M
+    step(stfk::fill_spd(s, A0, M, 2 * M, 0, 0, (int)M, (int)M, 21));
+    step(stfk::fill_spd(s, B0, M, 2 * M, M, 0, (int)M, (int)M, 21));
+    step(stfk::fill_spd(s, C0, M, 2 * M, M, M, (int)M, (int)M, 21));
+    step(stfk::dataflow_prepare((int)M, (int)M, true));
+    step(cudaStreamSynchronize(s));
+  }
+  const bool pdl = o.pdl && o.dataflow && o.trsm == 3;
+  if (e == cudaSuccess) step(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+  if (e == cudaSuccess) {
+    step(cudaMemcpyAsync(A, A0, bytes, cudaMemcpyDeviceToDevice, s));
+    step(cudaMemcpyAsync(B, B0, bytes, cudaMemcpyDeviceToDevice, s));
+    step(cudaMemcpyAsync(Cm, C0, bytes, cudaMemcpyDeviceToDevice, s));
+    step(stfk::info_reset(s, info));
+    step(cudaEventRecordWithFlags(e0, s, cudaEventRecordExternal));
+    const int nbk = (int)(M / 64);
+    const int trig = pdl ? (int)std::max<int64_t>(0, nbk - o.pdl_lead) : -1;
+    step(stfk::potrf_tile(s, 0, (int)M, A, M, 0, info, ws, nullptr, nullptr, 0, trig));
+    if (pdl) {
+      cudaGraphNode_t pn = capture_last_node(s);
+      if (pn && !r) r = capture_make_programmatic(s, pn);
+      int* kflag = ws + 2 + nbk * nbk;
+      step(stfk::trsm_res(s, 0, (int)M, (int)M, A, M, B, M, nullptr, nullptr, ws + 2, nbk, kflag, trig));
+      cudaGraphNode_t tn = capture_last_node(s);
+      if (tn && !r) r = capture_make_programmatic(s, tn);
+      const double* Bp = B;
+      step(stfk::gemm_nt_multi(s, 0, (int)M, (int)M, (int)M, 1, &Bp, M, &Bp, M, Cm, M, 1, 0, kflag,
+                               (int)(M / stfk::kTrsmResRows)));
+    } else {
+      step(stfk::trsm_res_parts(s, 0, (int)M, (int)M, A, M, B, M, nullptr, (int)o.trsm_res_split));
+      step(stfk::gemm_nt(s, 0, (int)M, (int)M, (int)M, B, M, B, M, Cm, M, 1));
+    }
+    step(cudaEventRecordWithFlags(e1, s, cudaEventRecordExternal));
+    cudaError_t ec = cudaStreamEndCapture(s, &g);
+    step(ec);
+  }
+  if (e == cudaSuccess && !r) step(cudaGraphInstantiate(&ge, g, 0));
+  double total = 0;
+  for (int it = 0; it < reps + 1 && e == cudaSuccess && !r; ++it) {
+    step(cudaGraphLaunch(ge, s));
+    step(cudaStreamSynchronize(s));
+    float ms = 0;
+    step(cudaEventElapsedTime(&ms, e0, e1));
+    if (it > 0) total += ms;
+  }
+  if (ge) cudaGraphExecDestroy(ge);
+  if (g) cudaGraphDestroy(g);
+  for (double* p : {A0, B0, C0, A, B, Cm}) cudaFree(p);
+  cudaFree(info);
+  cudaFree(ws);
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (s) cudaStreamDestroy(s);
+  if (r) return r;
+  if (e != cudaSuccess) return cuda_fail(e, "chain bench");
+  *avg_ms = total / reps;
+  return 0;
+}
+
 int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double* avg_ms) {
   g_err.clear();
+  if (kind == 4 && M >= 1 && reps >= 1 && avg_ms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int r = ensure_kernel_attrs(dev);
+    return r ? r : bench_chain(M, reps, avg_ms);
+  }
   if (kind < 0 || kind > 3 || M < 1 || reps < 1 || !avg_ms) return fail(-4, "bad stf_bench_kernel arguments");
   if (kind == 1 || kind == 3) N = M;
   if (kind == 2) K = N;

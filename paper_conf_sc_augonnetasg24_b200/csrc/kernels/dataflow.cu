@@ -33,6 +33,7 @@
 #include <map>
 #include <mutex>
 #include <tuple>
+#include <type_traits>
 #include <vector>
 
 #include "ptx.cuh"
@@ -71,6 +72,8 @@ struct DfParams {
   int crit;  // POTRF: one CTA runs the critical chain P -> S -> U -> P (blocks kept in smem)
   unsigned long long* trace;  // debug: %globaltimer stamps (null in production)
   Mirrors mir;                // POTRF: replicas of the tile, written with every final block (fused push)
+  int trig;  // programmatic dependent launch: the chain CTA triggers at step `trig`, the others at their
+             // start (-1: no trigger, dependents launch at completion)
 };
 
 __device__ __forceinline__ unsigned long long gtime() {
@@ -363,16 +366,23 @@ __device__ __forceinline__ void st_release_s(int* p, int v) {
 // Correctly rounded sqrt and division (div_by with y = RN(1/s)); every element
 // receives its updates in increasing column order, each a single fma or a DMMA
 // k-step pair: the same operations as without look-ahead, deterministic.
+// (An rsqrt issued next to the sqrt plus one Newton step against the rounded s
+// gives the same y = RN(1/s) -- tools/check_rcp.cu, 0 mismatches in 3 x 2^32
+// pivots -- but P(kb) measured 7% slower with it: warp 0 is issue-bound as much as
+// latency-bound, tools/p_lab.cu, profiles/r02/potrf_chain.txt.)
 // Non-positive pivot (or NaN): info = min(info, col0 + col + 1), s = NaN.
+template <bool kRsq = false>
 __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info, int* dpanel) {
   constexpr int LD = df::LDB, BAR_DONE = 1, BAR_NEXT = 2, GRP = 128;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
   if (warp == 0) {
     int bad = 0;
-#pragma unroll 1
-    for (int p = 0; p < 8; ++p) {
-      if (p > 0) bar_sync_id(BAR_NEXT, GRP);
+    // one panel; the rows below it live in v1 (rows lane) and v2 (rows lane + 32), each
+    // stream only while some of its rows lie below the panel (v1: p <= 2, v2: p <= 6),
+    // so the warp issues no FP64 work for rows that are all above it
+    auto panel = [&](int p, auto V1, auto V2) {
+      constexpr bool kV1 = decltype(V1)::value, kV2 = decltype(V2)::value;
       const int c0 = 8 * p;
       double dg[8][8];
 #pragma unroll
@@ -380,19 +390,27 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
 #pragma unroll
         for (int j = 0; j <= i; ++j) dg[i][j] = D[(c0 + i) * LD + c0 + j];
       const int r1 = lane, r2 = lane + 32;
-      const bool b1 = r1 >= c0 + 8, b2 = r2 >= c0 + 8;
+      const bool b1 = kV1 && r1 >= c0 + 8, b2 = kV2 && r2 >= c0 + 8;
       double v1[8], v2[8];
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
-        v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
-        v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
+        if (kV1) v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
+        if (kV2) v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
       }
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         const double d = dg[i][i];
         const bool ok = d > 0.0;
         if (!ok && bad == 0) bad = c0 + i + 1;
-        const double sq = ok ? sqrt(d) : kNaN, y = 1.0 / sq;
+        double sq, y;
+        if (kRsq) {
+          const double rs = rsqrt(d);
+          sq = ok ? sqrt(d) : kNaN;
+          y = fma(rs, fma(-sq, rs, 1.0), rs);
+        } else {
+          sq = ok ? sqrt(d) : kNaN;
+          y = 1.0 / sq;
+        }
         dg[i][i] = sq;
 #pragma unroll
         for (int r = i + 1; r < 8; ++r) dg[r][i] = div_by(dg[r][i], sq, y);
@@ -400,12 +418,12 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
         for (int r = i + 1; r < 8; ++r)
 #pragma unroll
           for (int c = i + 1; c <= r; ++c) dg[r][c] = fma(-dg[r][i], dg[c][i], dg[r][c]);
-        v1[i] = div_by(v1[i], sq, y);
-        v2[i] = div_by(v2[i], sq, y);
+        if (kV1) v1[i] = div_by(v1[i], sq, y);
+        if (kV2) v2[i] = div_by(v2[i], sq, y);
 #pragma unroll
         for (int c = i + 1; c < 8; ++c) {
-          v1[c] = fma(-v1[i], dg[c][i], v1[c]);
-          v2[c] = fma(-v2[i], dg[c][i], v2[c]);
+          if (kV1) v1[c] = fma(-v1[i], dg[c][i], v1[c]);
+          if (kV2) v2[c] = fma(-v2[i], dg[c][i], v2[c]);
         }
       }
       __syncwarp();  // every lane has read the diagonal block before lane 0 overwrites it
@@ -417,9 +435,19 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
       }
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
-        if (b1) D[r1 * LD + c0 + j] = v1[j];
-        if (b2) D[r2 * LD + c0 + j] = v2[j];
+        if (kV1 && b1) D[r1 * LD + c0 + j] = v1[j];
+        if (kV2 && b2) D[r2 * LD + c0 + j] = v2[j];
       }
+    };
+#pragma unroll 1
+    for (int p = 0; p < 8; ++p) {
+      if (p > 0) bar_sync_id(BAR_NEXT, GRP);
+      if (p <= 2)
+        panel(p, std::true_type{}, std::true_type{});
+      else if (p <= 6)
+        panel(p, std::false_type{}, std::true_type{});
+      else
+        panel(p, std::false_type{}, std::false_type{});
       __syncwarp();
       if (lane == 0) st_release_s(dpanel, p + 1);  // panel p is final: the S warps may use it
       bar_arrive_id(BAR_DONE, GRP);
@@ -595,12 +623,20 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
   double a[16];
   load_il(a, p.X, p.ldx, min(W, p.n), min(W, p.n), true);  // P(0) input: nothing precedes it
   for (int kb = 0; kb < T; ++kb) {
+    if (kb == p.trig) griddep_launch_dependents();  // the dependent TRSM(k+1,k) may start (it polls prog[])
     const int nk = min(W, p.n - kb * W);
     double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
     // ---- P(kb), and S(kb+1, kb) concurrently on the other four warps
     DF_STAMP(6 * kb + 0);
     const int ib = kb + 1, rows = ib < T ? min(W, p.n - ib * W) : 0;
     double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
+    // fast U(ib, ib, kb) (full blocks): warps 0-3 own the 36 lower 8 x 8 tiles, warp w
+    // the rows Ia = 7 - w (Ia + 1 tiles) and Ib = w (Ib + 1 tiles), 9 tiles each (one
+    // SM sub-partition each: the DMMA pipe is split evenly); C is prefetched into the
+    // accumulators right after P, the operands come straight from the S panels
+    const bool fastU = nk == W && rows == W;
+    const int Ia = 7 - (warp & 3), Ib = warp & 3;
+    double uA[8][2], uB[4][2];
     if (nk == W) {
       if (kb == 0) load_block_rm(D, df::LDB, Xkk, p.ldx, W, W, true);  // P(0) input: nothing precedes it
       if (threadIdx.x == 0) *dpanel = 0;
@@ -624,6 +660,19 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
           st_release(&prog[kb * p.Nb + kb], kb + 1);
         }
         DF_STAMP(6 * kb + 1);
+        if (fastU) {  // C = block (ib, ib) after its earlier updates, into the U accumulators
+          if (threadIdx.x == 0) wait_geq(&prog[ib * p.Nb + ib], kb);
+          bar_sync_id(4, 128);
+          const double* Cii = p.X + (int64_t)ib * W * p.ldx + ib * W;
+#pragma unroll
+          for (int J = 0; J < 8; ++J)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int rA = 8 * Ia + g, rB = 8 * Ib + g, c = 8 * J + 2 * t + h;
+              uA[J][h] = (J <= Ia && rA >= c) ? __ldcg(Cii + (int64_t)c * p.ldx + rA) : 0.0;
+              if (J < 4) uB[J][h] = (J <= Ib && rB >= c) ? __ldcg(Cii + (int64_t)c * p.ldx + rB) : 0.0;
+            }
+        }
       } else if (rows > 0) {  // ---- group S: X(kb+1, kb) <- X L_kk^-T, panel by panel as P finishes them
         const int tid = threadIdx.x - 128, sw = warp - 4;
         if (tid == 0) {
@@ -673,6 +722,49 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       }
       __syncthreads();
       if (kb + 1 == T) return;
+      if (fastU) {
+        // ---- U(ib, ib, kb): D <- lower(C - X X^T) on warps 0-3, X(m, k) from the S panels
+        if (warp < 4) {
+          DF_STAMP(6 * kb + 4);
+          // X(m, k) = Xp[(m >> 4) 16 W + xo(m & 15, k)]: for the fragment rows m = 8 R + g and
+          // k = k0 + t the offset is off[R][(k0 >> 2) & 1] + 16 k0 (the swizzle depends on k & 7)
+          int off[8][2];
+#pragma unroll
+          for (int R = 0; R < 8; ++R)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int m = 8 * R + g;
+              off[R][h] = (m >> 4) * 16 * W + sb::xo(m & 15, 4 * h + t) - 16 * 4 * h;
+            }
+          const int oA0 = Ia == 7 ? off[7][0] : Ia == 6 ? off[6][0] : Ia == 5 ? off[5][0] : off[4][0];
+          const int oA1 = Ia == 7 ? off[7][1] : Ia == 6 ? off[6][1] : Ia == 5 ? off[5][1] : off[4][1];
+          const int oB0 = Ib == 0 ? off[0][0] : Ib == 1 ? off[1][0] : Ib == 2 ? off[2][0] : off[3][0];
+          const int oB1 = Ib == 0 ? off[0][1] : Ib == 1 ? off[1][1] : Ib == 2 ? off[2][1] : off[3][1];
+#pragma unroll 2
+          for (int k0 = 0; k0 < W; k0 += 4) {
+            const int h = (k0 >> 2) & 1, kk = 16 * k0;
+            const double aA = Xp[(h ? oA1 : oA0) + kk], aB = Xp[(h ? oB1 : oB0) + kk];
+#pragma unroll
+            for (int J = 0; J < 8; ++J) {
+              if (J <= Ia) {  // warp-uniform
+                const double b = negd(Xp[off[J][h] + kk]);
+                dmma_8x8x4(uA[J][0], uA[J][1], aA, b);
+                if (J < 4 && J <= Ib) dmma_8x8x4(uB[J][0], uB[J][1], aB, b);
+              }
+            }
+          }
+#pragma unroll
+          for (int J = 0; J < 8; ++J)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int c = 8 * J + 2 * t + h;
+              if (J <= Ia) D[(8 * Ia + g) * df::LDB + c] = uA[J][h];
+              if (J < 4 && J <= Ib) D[(8 * Ib + g) * df::LDB + c] = uB[J][h];
+            }
+          DF_STAMP(6 * kb + 5);
+        }
+        continue;  // the next step's first __syncthreads orders D and Xp
+      }
       for (int idx = threadIdx.x; idx < W * W; idx += df::NT) {  // X for U's operands
         const int m = idx >> 6, k = idx & (W - 1);
         XS[m * df::LDO + k] = Xp[(m >> 4) * 16 * W + sb::xo(m & 15, k)];
@@ -758,6 +850,7 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
     }
     __syncthreads();
   }
+  if (p.trig >= 0) griddep_launch_dependents();
   for (;;) {
     if (threadIdx.x == 0) s_task = atomicAdd(&p.ws[0], 1);
     __syncthreads();
@@ -958,7 +1051,9 @@ cudaError_t launch_df(cudaStream_t s, int prio, DfParams& p, int max_ctas) {
 
 size_t dataflow_ws_bytes(int m, int n) {
   const int Mb = (m + df::W - 1) / df::W, Nb = (n + df::W - 1) / df::W;
-  return ((size_t)(2 + Mb * Nb) * sizeof(int) + 255) / 256 * 256;
+  // ticket, chain role, per-block progress, then Nb counters of the chain TRSM(k+1,k)
+  // that follows a POTRF with programmatic launch (zeroed with the rest)
+  return ((size_t)(2 + Mb * Nb + Nb) * sizeof(int) + 255) / 256 * 256;
 }
 
 cudaError_t dataflow_prepare(int m, int n, bool potrf) {
@@ -985,7 +1080,7 @@ cudaError_t dataflow_init_attrs() {
 
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                        unsigned long long* info, int* ws, const Mirrors* mirrors, unsigned long long* trace,
-                       int ctas_override) {
+                       int ctas_override, int pdl_trig) {
   if (n <= 0) return cudaSuccess;
   DfParams p{};
   p.X = A;
@@ -1009,6 +1104,7 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   // chain waits on updates only bulk CTAs claim)
   if (p.crit) ctas = std::min(p.ntasks, std::max(ctas, 2) - 1) + 1;
   p.trace = trace;
+  p.trig = pdl_trig;
   return launch_df(stream, prio, p, ctas);
 }
 
@@ -1032,6 +1128,7 @@ cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double*
   p.potrf = 0;
   p.crit = 0;
   p.trace = nullptr;
+  p.trig = -1;
   const int par = p.Mb * (p.Nb > 1 ? p.Nb - 1 : 1);
   return launch_df(stream, prio, p, std::min(par, std::min(4 * df_max_ctas(16), num_sms())));
 }

@@ -71,12 +71,28 @@ __device__ __forceinline__ uint32_t swz_off(int r, int k) {
 struct ExtraPairs {
   CUtensorMap a[3], b[3];
   int npairs;  // total pairs including (tmA, tmB): 1..4
+  // Overlap with the producing TRSM (programmatic dependent launch, SYRK(k+1,k) of
+  // the panel chain): k columns [64 c, 64 c + 64) of the operands are final once
+  // kflag[c] >= kcount (the TRSM's CTAs count their finished column blocks);
+  // null: operands complete at launch.
+  const int* kflag;
+  int kcount;
 };
 
 // k-tile kt: pair p = kt / KT1 (p = 0: tmA, tmB), tile kt - p KT1 of that pair
 template <class g>
 __device__ __forceinline__ void load_stage(uint8_t* smem, int s, const CUtensorMap* tmA, const CUtensorMap* tmB,
                                            const ExtraPairs* ex, int KT1, int m0, int n0, int kt, uint64_t* full) {
+  if (ex->kflag) {  // k columns of this tile published by the TRSM (acquire), then visible to TMA
+    const int* f = ex->kflag + (kt * g::BK) / 64;
+    for (;;) {
+      int v;
+      asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+      if (v >= ex->kcount) break;
+      __nanosleep(64);
+    }
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+  }
   mbar_arrive_expect_tx(&full[s], g::STAGE_BYTES);
   uint8_t* sa = smem + s * g::STAGE_BYTES;
   uint8_t* sb = sa + g::A_BYTES;
@@ -329,7 +345,7 @@ cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, co
 
 cudaError_t gemm_nt_multi(cudaStream_t stream, int prio, int M, int N, int K, int npairs, const double* const* As,
                           int64_t lda, const double* const* Bs, int64_t ldb, double* C, int64_t ldc, int lower,
-                          int small) {
+                          int small, const int* kflag, int kcount) {
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   if (npairs < 1 || npairs > 4) return cudaErrorInvalidValue;
   if ((lda & 1) || (ldb & 1)) return cudaErrorMisalignedAddress;
@@ -346,6 +362,9 @@ cudaError_t gemm_nt_multi(cudaStream_t stream, int prio, int M, int N, int K, in
   ExtraPairs ex;
   memset(&ex, 0, sizeof ex);
   ex.npairs = npairs;
+  ex.kflag = kflag;
+  ex.kcount = kcount;
+  if (kflag && (npairs != 1 || K % 64)) return cudaErrorInvalidValue;
   for (int p = 1; p < 4; ++p) {
     if (p < npairs) {
       if (!make_operand_map(&ex.a[p - 1], As[p], M, K, lda, bk) || !make_operand_map(&ex.b[p - 1], Bs[p], N, K, ldb, bk))

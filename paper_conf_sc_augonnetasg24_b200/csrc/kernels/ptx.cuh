@@ -59,6 +59,10 @@ __device__ __forceinline__ void tma_load_2d(void* smem_dst, const CUtensorMap* t
       : "memory");
 }
 
+// Programmatic dependent launch: this CTA no longer holds back the dependent grid
+// (it launches once every CTA has executed this or exited).
+__device__ __forceinline__ void griddep_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // D(8x8) += A(8x4) * B(4x8), FP64 tensor core (SASS DMMA.8x8x4).
 // Fragments (verified on the box by tools/calib_fp64.cu): lane l, g = l>>2, t = l&3:
 //   a = A[g][t], b = B[t][g], d0 = D[g][2t], d1 = D[g][2t+1].

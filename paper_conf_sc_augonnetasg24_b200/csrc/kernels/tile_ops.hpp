@@ -27,9 +27,12 @@ cudaError_t gemm_nt_tiles(cudaStream_t stream, int prio, int M, int N, int K, co
 // across the pairs, so the result is bit-identical to npairs gemm_nt calls in that
 // order, with one C load/store and one pipeline ramp instead of npairs
 // (consecutive tile updates GEMM(i,j,k), GEMM(i,j,k+1), ... of one task).
+// kflag (optional, npairs == 1, K % 64 == 0): the k columns [64 c, 64 c + 64) of A and B
+// are waited for until kflag[c] >= kcount (counters of the TRSM producing them), so
+// the launch may overlap that TRSM (programmatic dependent launch).
 cudaError_t gemm_nt_multi(cudaStream_t stream, int prio, int M, int N, int K, int npairs, const double* const* As,
                           int64_t lda, const double* const* Bs, int64_t ldb, double* C, int64_t ldc, int lower,
-                          int small);
+                          int small, const int* kflag = nullptr, int kcount = 0);
 
 // K3: B[M x n] <- B * L^-T with L[n x n] lower triangular, non-unit diagonal
 // (side = right, lower, transposed).  Recursive: base blocks of <= 64 columns
@@ -65,7 +68,7 @@ struct Mirrors {
 // of L_kk, NEXT-3).
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                        unsigned long long* info, int* ws, const Mirrors* mirrors = nullptr,
-                       unsigned long long* trace = nullptr, int ctas = 0);
+                       unsigned long long* trace = nullptr, int ctas = 0, int pdl_trig = -1);
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                       int64_t ldb, int* ws);
 size_t dataflow_ws_bytes(int m, int n);
@@ -84,8 +87,16 @@ cudaError_t dataflow_prepare(int m, int n, bool potrf);
 bool trsm_res_supported(int n, const double* L, int64_t ldl);
 cudaError_t trsm_res_parts(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
                            int64_t ldb, const Mirrors* mirrors, int parts);
+// pflag (optional): progress array of the dataflow POTRF producing L (its ws + 2,
+// block grid pNb = n / 64): blocks of L are waited for as the solve reaches them,
+// so the launch may overlap that POTRF (programmatic dependent launch).
+// kflag (optional): per-64-column-block counters; each CTA adds 1 to kflag[jb] once its
+// rows of column block jb are stored (a consumer waits for ceil(M / 16)), and the CTAs
+// trigger their programmatic dependents at column block `trig` (-1: at exit).
 cudaError_t trsm_res(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
-                     int64_t ldb, const Mirrors* mirrors = nullptr, unsigned long long* trace = nullptr);
+                     int64_t ldb, const Mirrors* mirrors = nullptr, unsigned long long* trace = nullptr,
+                     const int* pflag = nullptr, int pNb = 0, int* kflag = nullptr, int trig = -1);
+constexpr int kTrsmResRows = 16;  // rows per CTA of trsm_res
 
 // K8: fill rows r0.., cols c0.. (global indices) of the seeded SPD metric matrix
 // of order n into dst[rows x cols] (ld).  Same SplitMix64 spec as synth/spd.py.

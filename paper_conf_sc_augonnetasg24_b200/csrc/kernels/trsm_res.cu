@@ -21,6 +21,16 @@
 //                     correctly rounded division, sub-block updates on DMMA),
 //                     then to global memory (+ fused-push mirrors).
 //
+// Overlap with the producing POTRF (programmatic dependent launch, TRSM(k+1,k)
+// of the panel chain): with `pflag` the kernel may start while the dataflow
+// POTRF of L is still running.  pflag is that kernel's per-64-block progress
+// array (prog[ib * pNb + jb] == jb + 1 once block (ib, jb) of L is final and
+// stored, published with st.release.gpu): the TMA producer acquires block
+// (jb, pb) before loading it (then a generic -> async proxy fence), the MMA
+// warps acquire the diagonal block before staging it.  Column block jb of X
+// therefore follows row block jb of L by one solve.  Without pflag the inputs
+// are complete at launch (ordinary stream / graph dependency).
+//
 // Hand-off by named barriers: READY (MMA arrive -> solver sync) when X[:,jb]
 // holds its updated right-hand side, SOLVED (solver arrive -> MMA sync) when it
 // holds the solution.  Every sum has a fixed order (k-steps split mod 3
@@ -52,7 +62,7 @@ __device__ __forceinline__ void tr_stamp(unsigned long long* trace, int idx) {
 namespace tr {
 using sb::xo;
 using sb::poff;
-constexpr int R = 16;        // rows per CTA (one 128-byte line per column of the panel)
+constexpr int R = kTrsmResRows;  // rows per CTA (one 128-byte line per column of the panel)
 constexpr int W = 64;        // column block
 constexpr int NMAX = 1024;   // resident panel limit (NMAX * 128 B = 128 KB)
 constexpr int BK = 32;       // k of L per pipeline stage
@@ -87,6 +97,14 @@ template <int N>
 __device__ __forceinline__ void cpa_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
+__device__ __forceinline__ void wait_final(const int* p, int v) {  // acquire: L block published by the POTRF
+  int x;
+  for (;;) {
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(x) : "l"(p) : "memory");
+    if (x >= v) break;
+    __nanosleep(64);
+  }
+}
 __device__ __forceinline__ double ld_cg_early(const double* p) {  // volatile: issued where written
   double v;
   asm volatile("ld.global.cg.f64 %0, [%1];" : "=d"(v) : "l"(p));
@@ -105,7 +123,8 @@ __device__ __forceinline__ double ld_cg_early(const double* p) {  // volatile: i
 // are combined in a fixed order at the end of the step.
 __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_constant__ CUtensorMap tmL, const double* __restrict__ L,
                                                               int64_t ldl, int n, double* __restrict__ X, int64_t ldx,
-                                                              int M, const Mirrors mir, unsigned long long* trace, int dbg) {
+                                                              int M, const Mirrors mir, unsigned long long* trace, int dbg,
+                                                              const int* pflag, int pNb, int* kflag, int trig) {
   using namespace tr;
   extern __shared__ __align__(1024) uint8_t smraw[];
   double* sm = reinterpret_cast<double*>(smraw + ((1024u - (smem_u32(smraw) & 1023u)) & 1023u));
@@ -138,6 +157,10 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
       for (int q = 0; q < total; ++q) {
         const int s = q % NST;
         if (q >= NST) mbar_wait(&empty[s], (q / NST - 1) & 1);
+        if (pflag && h == 0) {  // block (jb, pb) of L final
+          wait_final(pflag + jb * pNb + pb, pb + 1);
+          asm volatile("fence.proxy.async.global;" ::: "memory");
+        }
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_arrive_expect_tx(&full[s], STAGE * 8);
 #pragma unroll
@@ -163,6 +186,7 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
         double* dst = Ld + (jb & 1) * DP;
         const double* src = L + (int64_t)c0 * ldl + c0;
         const int tm = mw * 32 + lane;  // 0..191
+        if (pflag) wait_final(pflag + jb * pNb + jb, jb + 1);  // L(jb, jb) final
         for (int idx = tm; idx < W * W; idx += MMA_THREADS) {
           const int rr = idx & (W - 1), cc = idx >> 6;
           if (rr >= cc) cpa8(dst + sb::poff(rr, cc), src + (int64_t)cc * ldl + rr);
@@ -302,6 +326,12 @@ __global__ void __launch_bounds__(tr::NT, 1) trsm_res_kernel(const __grid_consta
         }
         mirror_fence(mir.mc);
       }
+      if (kflag) {  // this CTA's rows of column block jb are stored: count them for the SYRK
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) atomicAdd(kflag + jb, 1);
+      }
+      if (jb == trig) griddep_launch_dependents();  // the dependent SYRK(k+1,k) may start
       __syncwarp();
       if (lane == 0) tr_stamp(trace, 5 * Nb + jb);  // solve end
       if (more) bar_arrive_n(BAR_SOLVED, MMA_THREADS + SOLVE_THREADS);
@@ -349,7 +379,8 @@ cudaError_t trsm_res_init_attrs() {
 }
 
 cudaError_t trsm_res(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,
-                     int64_t ldb, const Mirrors* mirrors, unsigned long long* trace) {
+                     int64_t ldb, const Mirrors* mirrors, unsigned long long* trace, const int* pflag, int pNb,
+                     int* kflag, int trig) {
   Mirrors mir{};
   if (mirrors) mir = *mirrors;
   if (M <= 0 || n <= 0) return cudaSuccess;
@@ -371,7 +402,7 @@ cudaError_t trsm_res(cudaStream_t stream, int prio, int M, int n, const double* 
     const char* e = getenv("STF_TRSM_DBG");
     return e ? atoi(e) : 0;
   }();
-  return cudaLaunchKernelEx(&cfg, trsm_res_kernel, tmL, L, ldl, n, B, ldb, M, mir, trace, dbg);
+  return cudaLaunchKernelEx(&cfg, trsm_res_kernel, tmL, L, ldl, n, B, ldb, M, mir, trace, dbg, pflag, pNb, kflag, trig);
 }
 
 }  // namespace stfk

@@ -67,7 +67,7 @@ struct Options {
   int64_t mem_cap_tiles = 0;   // HOST_COLMAJOR on one GPU: device tile frames (0 = no cap)
   int64_t ooc_order = -1;      // out-of-core program order: 0 tall, 1 2D-blocked, -1 auto
   int64_t host_stream = 1;     // HOST_COLMAJOR on one GPU, nb >= 512, T >= 16: frame-per-tile OOC builder
-  int64_t trsm_res_tail = 8192;  // trsm 3: resident panel for every TRSM once n - k nb <= this
+  int64_t trsm_res_tail = 4096;  // trsm 3: resident panel for every TRSM once n - k nb <= this
   int64_t trsm_rows = 128;     // row panel: rows per CTA (32, 64, 128)
   int64_t trsm_res_split = 2;  // resident-panel TRSMs in 2 (or 4) column parts with GEMMs between; 1 = one launch
   int64_t gemm_merge = 2;      // D > 0: merged tile updates for tiles >= D columns right of the panel
@@ -83,7 +83,8 @@ struct Options {
   int64_t host_stream_budget_pct = 90;  // host_stream block budget
   int64_t host_eager = 0;      // 1: HOST_COLMAJOR calls on pinned memory lowered eagerly
   int64_t stream_pool = 0;     // 0 default pool; 1 one compute + one copy stream per slot; 2 one stream (ablations)
-  int64_t pdl = 0;             // programmatic dependent launch between same-stream chain kernels
+  int64_t pdl = 1;             // programmatic dependent launch: TRSM(k+1,k) overlaps POTRF(k) (graph backend)
+  int64_t pdl_lead = 8;        // pdl: the POTRF lets its TRSM start this many 64-block steps before its end
   int64_t debug_skip = 0;      // bit mask of task kinds not launched (timing what-ifs; results invalid)
   int64_t debug_trace = 0;     // timing events around every task (one slot)
   int64_t nvtx = 0;            // NVTX range per task submission (eager backend; the graph launch is one range)
@@ -129,6 +130,12 @@ constexpr int kCopyStreams = 2;
 constexpr size_t kCacheMax = 4;
 
 // A plan bound to physical buffers, plus its lowering artefacts.
+// Stream-capture helpers for programmatic dependent launch (exec.cpp): the single
+// node a capturing stream's next launch would depend on (else null), and turning
+// the capture edge from kernel node `from` into a programmatic one.
+cudaGraphNode_t capture_last_node(cudaStream_t s);
+int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from);
+
 struct Exec {
   // key
   int64_t n = 0, nb = 0;
@@ -145,6 +152,8 @@ struct Exec {
   std::vector<std::pair<int, void*>> allocs;  // (device, ptr) library-owned
   std::vector<double*> scratch;               // per (slot, copy stream): staging tile for 'U'
   std::vector<int*> task_ws;                  // per task: dataflow-kernel workspace (POTRF/TRSM), else null
+  std::vector<int64_t> pdl_src;               // per task: TRSM(k+1,k) -> index of POTRF(k) it may overlap, else -1
+  std::vector<cudaGraphNode_t> cap_node;      // per task: its last captured node (POTRFs with a pdl consumer)
   std::vector<cudaEvent_t> events;            // per task, null if not needed
   std::vector<int> events_dev;
   cudaGraph_t graph = nullptr;

@@ -66,7 +66,9 @@ if n // nb <= 32:
         p_ = find(0, k, k, k)
         t_ = find(1, k + 1, k, k)
         s_ = find(2, k + 1, k + 1, k)
-        print("k=%2d POTRF %.3f-%.3f  TRSM(k+1) %.3f-%.3f  SYRK(k+1) %.3f-%.3f" % (k, *p_, *t_, *s_))
+        g_ = find(3, k + 1, k, k - 1)
+        print("k=%2d POTRF %.3f-%.3f  TRSM(k+1) %.3f-%.3f  SYRK(k+1) %.3f-%.3f  GEMM(k+1,k,k-1) %.3f-%.3f" % (
+            k, *p_, *t_, *s_, *g_))
 # flop-weighted activity profile: GEMM/SYRK/TRSM flops completed per bin (task flops spread over its span)
 span = R[:, 6].max()
 edges = np.linspace(0, span, bins + 1)
