@@ -180,8 +180,8 @@ const char *stf_last_error(void);
  *                           block by column block as the TRSM's CTAs finish them (device
  *                           flags, acquire/release).  The TRSM(k+1,k) is then one
  *                           resident-panel launch (trsm_res_split does not apply to it) in
- *                           every grid, so the bits do not depend on where it runs.  Same
- *                           bits with 0 (no overlap)
+ *                           every grid, so the bits do not depend on where it runs; they
+ *                           equal pdl = 0 with trsm_res_split = 1 (tested)
  *   "pdl_lead" STF_PDL_LEAD 64-block steps before its end at which a chain kernel lets its
  *                           dependent launch (default 8; >= nb/64: at its start)
  *   "debug_skip" STF_DEBUG_SKIP bit mask (or names potrf,trsm,syrk,gemm,copy,trsm_as_gemm,

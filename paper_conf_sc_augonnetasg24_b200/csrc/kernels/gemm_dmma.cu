@@ -143,8 +143,16 @@ __global__ void __launch_bounds__((g::BM / WM) * (g::BN / WN) * 32, g::MINB)
       tn = b - t * (t + 1);
     }
   } else {
-    tm = blockIdx.x;
-    tn = blockIdx.y;
+    // L2-aware order: CTAs are dispatched in linear block order; walk the M tiles in
+    // groups of 16 rows before moving along N, so the CTAs resident at once (2 per
+    // SM) share ~16 A row panels and ~18 B column panels instead of sweeping all of A
+    // per B panel (a 1024-tile update, 8 x 16 CTAs, is one group: unchanged)
+    constexpr int G = 16;
+    const int tMg = gridDim.x, tNg = gridDim.y;
+    const int bid = blockIdx.x + blockIdx.y * tMg, per = G * tNg;
+    const int grp = bid / per, first = grp * G, gs = min(tMg - first, G), rr = bid - grp * per;
+    tm = first + rr % gs;
+    tn = rr / gs;
   }
   const int m0 = tm * g::BM, n0 = tn * g::BN;
   const int KT1 = (K + g::BK - 1) / g::BK;
