@@ -111,7 +111,9 @@ const char *stf_last_error(void);
  *   "trsm_split" STF_TRSM_SPLIT P in [1,16]: non-critical row-panel TRSMs run right-looking
  *                           over P column blocks (panel kernel + GEMM updates; default 4)
  *   "trsm_res_tail" STF_TRSM_RES_TAIL C >= 0: with trsm 3, every TRSM(i,k) of a panel step
- *                           whose trailing order n - k nb <= C uses the resident panel (default 4096: n = 8192 +7%, profiles/r02/pdl_and_tail.txt)
+ *                           whose trailing order n - k nb <= C uses the resident panel
+ *                           (-1 default: 4096 at nb >= 1024, n = 8192 +7%; 8192 below, nb = 512
+ *                           +6%; profiles/r02/pdl_and_tail.txt, split_potrf.txt)
  *   "trsm_res_split" STF_TRSM_RES_SPLIT 2 (default) or 4: a resident-panel TRSM runs as that many
  *                           column parts, right-looking, with a GEMM after each (more CTAs on the
  *                           critical path); 1: one launch

@@ -55,7 +55,7 @@ const std::vector<OptDesc>& option_table() {
       {"mem_cap_tiles", "STF_MEM_CAP_TILES", &Options::mem_cap_tiles, 0, INT64_MAX, true},
       {"ooc_order", "STF_OOC_ORDER", &Options::ooc_order, -1, 1, true},
       {"host_stream", "STF_HOST_STREAM", &Options::host_stream, 0, 1, true},
-      {"trsm_res_tail", "STF_TRSM_RES_TAIL", &Options::trsm_res_tail, 0, INT64_MAX, true},
+      {"trsm_res_tail", "STF_TRSM_RES_TAIL", &Options::trsm_res_tail, -1, INT64_MAX, true},
       {"trsm_rows", "STF_TRSM_ROWS", &Options::trsm_rows, 32, 128, true},
       {"trsm_res_split", "STF_TRSM_RES_SPLIT", &Options::trsm_res_split, 1, 4, true},
       {"gemm_merge", "STF_GEMM_MERGE", &Options::gemm_merge, 0, 64, true},

@@ -179,6 +179,27 @@ int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from) {
   return 0;
 }
 
+// Remove node `from` from the current capture dependencies of stream s (no-op when absent).
+int capture_drop_dependency(cudaStream_t s, cudaGraphNode_t from) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  const cudaGraphNode_t* deps = nullptr;
+  const cudaGraphEdgeData* ed = nullptr;
+  size_t nd = 0;
+  CUDA_TRY(cudaStreamGetCaptureInfo_v3(s, &st, nullptr, nullptr, &deps, &ed, &nd), "capture info");
+  if (st != cudaStreamCaptureStatusActive) return 0;
+  std::vector<cudaGraphNode_t> d;
+  std::vector<cudaGraphEdgeData> e;
+  for (size_t i = 0; i < nd; ++i)
+    if (deps[i] != from) {
+      d.push_back(deps[i]);
+      e.push_back(ed ? ed[i] : cudaGraphEdgeData{});
+    }
+  if (d.size() == nd) return 0;
+  CUDA_TRY(cudaStreamUpdateCaptureDependencies_v2(s, d.data(), e.data(), d.size(), cudaStreamSetCaptureDependencies),
+           "capture drop edge");
+  return 0;
+}
+
 // ------------------------------------------------------------------ lowering
 namespace {
 
@@ -239,10 +260,18 @@ struct Lowerer {
           // pdl: the chain CTA releases the dependent TRSM(k+1,k) pdl_lead 64-block steps before its end
           const int nbk = (int)((nb + 63) / 64);
           const int trig = X.opt.pdl ? (int)std::max<int64_t>(0, nbk - X.opt.pdl_lead) : -1;
+          cudaGraphNode_t chain = nullptr;
           CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir,
-                                    nullptr, 0, trig),
+                                    nullptr, 0, trig, &chain),
                    "POTRF launch");
-          if (!X.cap_node.empty()) X.cap_node[tidx] = capture_last_node(s);
+          if (!X.cap_node.empty()) X.cap_node[tidx] = capture_last_node(s);  // the block-task launch
+          if (chain) {
+            // two launches (chain, then block tasks released by it): whatever follows on this
+            // stream, and the successors waiting on its event, depend on both
+            if (!X.cap_node2.empty()) X.cap_node2[tidx] = chain;
+            CUDA_TRY(cudaStreamUpdateCaptureDependencies(s, &chain, 1, cudaStreamAddCaptureDependencies),
+                     "POTRF join");
+          }
         } else
           CUDA_TRY(stfk::potrf_lower(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info),
                    "POTRF launch");
@@ -267,6 +296,14 @@ struct Lowerer {
           const int nbk = (int)(nb / 64);
           const int* pflag = src >= 0 && X.task_ws[(size_t)src] ? X.task_ws[(size_t)src] + 2 : nullptr;
           if (pflag && !X.cap_node.empty() && X.cap_node[(size_t)src]) {
+            // one programmatic edge, from the POTRF's last launch (a node with several
+            // programmatic edges is not launched early: profiles/r02/pdl_and_tail.txt); the
+            // chain launch of a two-launch POTRF is its ancestor through that edge, and the
+            // TRSM reads L_kk through the progress flags, so its edge is dropped here
+            if (X.cap_node2[(size_t)src]) {
+              int r = capture_drop_dependency(s, X.cap_node2[(size_t)src]);
+              if (r) return r;
+            }
             int r = capture_make_programmatic(s, X.cap_node[(size_t)src]);
             if (r) return r;
           }
@@ -277,7 +314,9 @@ struct Lowerer {
                                   nullptr, pflag, nbk, kflag, trig),
                    "TRSM launch");
           if (!X.cap_node.empty()) X.cap_node[tidx] = capture_last_node(s);
-        } else if (X.opt.trsm == 3 && (t.i == t.k + 1 || X.n - t.k * nb <= X.opt.trsm_res_tail) &&
+        } else if (X.opt.trsm == 3 &&
+                   (t.i == t.k + 1 ||
+                    X.n - t.k * nb <= (X.opt.trsm_res_tail >= 0 ? X.opt.trsm_res_tail : (nb >= 1024 ? 4096 : 8192))) &&
                    stfk::trsm_res_supported((int)nb, X.buf[(size_t)t.in[0]], nb)) {
           // the next panel's TRSM(k+1,k) is on the critical path, and near the end of the
           // factorisation every TRSM is latency-bound: the resident-panel kernel (16 rows per
@@ -781,6 +820,7 @@ int prepare(Context& C, Exec& X, const stf_matrix_desc* desc) {
   // pdl: TRSM(k+1,k) that follows its POTRF(k) on the same slot and stream
   X.pdl_src.assign(P.tasks.size(), -1);
   X.cap_node.assign(X.opt.graph && X.opt.pdl ? P.tasks.size() : 0, nullptr);
+  X.cap_node2.assign(X.cap_node.size(), nullptr);
   if (X.opt.pdl && X.opt.dataflow && X.opt.trsm == 3) {
     std::vector<int64_t> potrf_of((size_t)T, -1);
     for (size_t t = 0; t < P.tasks.size(); ++t)

@@ -156,12 +156,19 @@ static int bench_chain(int64_t M, int reps, double* avg_ms) {
     step(cudaMemcpyAsync(B, B0, bytes, cudaMemcpyDeviceToDevice, s));
     step(cudaMemcpyAsync(Cm, C0, bytes, cudaMemcpyDeviceToDevice, s));
     step(stfk::info_reset(s, info));
+    cudaGraphNode_t extra = capture_last_node(s);  // debug: an extra full dependency of the TRSM
     step(cudaEventRecordWithFlags(e0, s, cudaEventRecordExternal));
     const int nbk = (int)(M / 64);
     const int trig = pdl ? (int)std::max<int64_t>(0, nbk - o.pdl_lead) : -1;
-    step(stfk::potrf_tile(s, 0, (int)M, A, M, 0, info, ws, nullptr, nullptr, 0, trig));
+    cudaGraphNode_t chain = nullptr;
+    step(stfk::potrf_tile(s, 0, (int)M, A, M, 0, info, ws, nullptr, nullptr, 0, trig, &chain));
+    cudaGraphNode_t pn = capture_last_node(s);
+    if (chain) step(cudaStreamUpdateCaptureDependencies(s, &chain, 1, cudaStreamAddCaptureDependencies));
     if (pdl) {
-      cudaGraphNode_t pn = capture_last_node(s);
+      // one programmatic edge into the TRSM (see exec.cpp); debug: a second, full edge
+      static const int dbg = getenv("STF_DEBUG_CHAIN_MODE") ? atoi(getenv("STF_DEBUG_CHAIN_MODE")) : 0;
+      if (chain && !r) r = capture_drop_dependency(s, chain);
+      if ((dbg & 2) && extra) step(cudaStreamUpdateCaptureDependencies(s, &extra, 1, cudaStreamAddCaptureDependencies));
       if (pn && !r) r = capture_make_programmatic(s, pn);
       int* kflag = ws + 2 + nbk * nbk;
       step(stfk::trsm_res(s, 0, (int)M, (int)M, A, M, B, M, nullptr, nullptr, ws + 2, nbk, kflag, trig));
@@ -177,6 +184,27 @@ static int bench_chain(int64_t M, int reps, double* avg_ms) {
     step(cudaEventRecordWithFlags(e1, s, cudaEventRecordExternal));
     cudaError_t ec = cudaStreamEndCapture(s, &g);
     step(ec);
+  }
+  if (e == cudaSuccess && !r && getenv("STF_DEBUG_CHAIN")) {  // edges of the captured chain graph
+    size_t nn = 0;
+    cudaGraphGetNodes(g, nullptr, &nn);
+    std::vector<cudaGraphNode_t> nodes(nn);
+    cudaGraphGetNodes(g, nodes.data(), &nn);
+    for (size_t i = 0; i < nn; ++i) {
+      cudaGraphNodeType ty;
+      cudaGraphNodeGetType(nodes[i], &ty);
+      size_t nd = 0;
+      cudaGraphNodeGetDependencies_v2(nodes[i], nullptr, nullptr, &nd);
+      std::vector<cudaGraphNode_t> d(nd);
+      std::vector<cudaGraphEdgeData> ed(nd);
+      cudaGraphNodeGetDependencies_v2(nodes[i], d.data(), ed.data(), &nd);
+      fprintf(stderr, "node %zu type %d deps:", i, (int)ty);
+      for (size_t k = 0; k < nd; ++k) {
+        size_t j = std::find(nodes.begin(), nodes.end(), d[k]) - nodes.begin();
+        fprintf(stderr, " %zu(type %d port %d)", j, (int)ed[k].type, (int)ed[k].from_port);
+      }
+      fprintf(stderr, "\n");
+    }
   }
   if (e == cudaSuccess && !r) step(cudaGraphInstantiate(&ge, g, 0));
   double total = 0;

@@ -49,6 +49,9 @@ constexpr int LDB = 65;     // smem stride of substitution / Cholesky blocks [ro
 constexpr int NT = 256;
 // critical CTA: D [W][LDB] + XS [W][LDO] + Rc [W] + 4 swizzled 16-row panels + 4 x Y [W] + a counter
 constexpr int SMEM_BYTES = (W * LDB + W * LDO + W + 4 * 16 * W + 4 * W) * 8 + 16;  // 104,720 B
+// bulk_kernel: the largest block task (U operands; S panels + L block; ragged S)
+constexpr int cmax(int a, int b) { return a > b ? a : b; }
+constexpr int BULK_SMEM_BYTES = cmax(2 * W * LDO, cmax(4 * 16 * W + W * LDB + W, 2 * W * LDB + W)) * 8 + 16;  // 69,648 B
 enum : uint32_t { T_P = 0, T_S = 1, T_U = 2 };
 
 __host__ __device__ inline uint32_t enc(uint32_t t, uint32_t i, uint32_t j, uint32_t k) {
@@ -835,27 +838,23 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
   }
 }
 
-__global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
-  extern __shared__ __align__(16) double sm[];
-  __shared__ int s_task;
+// The ticket loop of the block tasks (see the header comment).  kBulk: the POTRF
+// block tasks other than the critical chain's (S and U only; the launch that runs
+// them next to the chain launch), compiled for 2 CTAs per SM.
+template <bool kBulk>
+__device__ __forceinline__ void ticket_loop(const DfParams& p, double* sm, int* s_task) {
   const int W = df::W;
   int* prog = p.ws + 2;
-  if (p.crit) {
-    // the first CTA to start takes the critical chain (it is resident by construction)
-    if (threadIdx.x == 0) s_task = (atomicCAS(&p.ws[1], 0, 1) == 0);
-    __syncthreads();
-    if (s_task) {
-      critical_chain(p, sm);
-      return;
-    }
-    __syncthreads();
-  }
-  if (p.trig >= 0) griddep_launch_dependents();
+  bool triggered = false;
   for (;;) {
-    if (threadIdx.x == 0) s_task = atomicAdd(&p.ws[0], 1);
+    if (threadIdx.x == 0) *s_task = atomicAdd(&p.ws[0], 1);
     __syncthreads();
-    const int ticket = s_task;
+    const int ticket = *s_task;
     if (ticket >= p.ntasks) return;
+    if (kBulk && !triggered && p.trig >= 0 && ticket >= p.trig) {  // the dependent TRSM(k+1,k) may start
+      griddep_launch_dependents();
+      triggered = true;
+    }
     DF_STAMP(6 * p.Nb + 3 * ticket + 0);
     const uint32_t code = p.tasks[ticket];
     const uint32_t type = code >> 30;
@@ -863,7 +862,7 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
     const int rows = min(W, p.m - ib * W);
     if (threadIdx.x == 0) {
       if (p.potrf) {
-        if (type == df::T_P) {
+        if (!kBulk && type == df::T_P) {
           wait_geq(&prog[kb * p.Nb + kb], kb);
         } else if (type == df::T_S) {
           wait_geq(&prog[kb * p.Nb + kb], kb + 1);
@@ -884,10 +883,10 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
     }
     __syncthreads();
     DF_STAMP(6 * p.Nb + 3 * ticket + 1);
-    if (p.potrf) {
+    if (kBulk || p.potrf) {
       double* Xkk = p.X + (int64_t)kb * W * p.ldx + kb * W;
       const int nk = min(W, p.n - kb * W);
-      if (type == df::T_P) {
+      if (!kBulk && type == df::T_P) {
         task_chol(sm, Xkk, p.ldx, nk, p.col0 + (int64_t)kb * W, p.info, &p.mir, Xkk - p.X);
       } else if (type == df::T_S) {
         double* Xik = p.X + (int64_t)kb * W * p.ldx + ib * W;
@@ -916,6 +915,35 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
     }
     DF_STAMP(6 * p.Nb + 3 * ticket + 2);
   }
+}
+
+__global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
+  extern __shared__ __align__(16) double sm[];
+  __shared__ int s_task;
+  if (p.crit) {
+    // the first CTA to start takes the critical chain (it is resident by construction)
+    if (threadIdx.x == 0) s_task = (atomicCAS(&p.ws[1], 0, 1) == 0);
+    __syncthreads();
+    if (s_task) {
+      critical_chain(p, sm);
+      return;
+    }
+    __syncthreads();
+  }
+  if (p.trig >= 0) griddep_launch_dependents();
+  ticket_loop<false>(p, sm, &s_task);
+}
+
+// POTRF as two launches: the critical chain alone (dataflow_kernel with one CTA:
+// the register-heavy panel code) and the block tasks (bulk_kernel, 2 CTAs per SM
+// with 70 KB of shared memory: they fit next to a GEMM CTA).  The chain releases
+// the bulk launch at its first step (programmatic dependent launch: both are
+// resident together, each only waits on the other's progress counters); the bulk
+// CTAs release the next dependent (TRSM(k+1,k)) once the tickets reach p.trig.
+__global__ void __launch_bounds__(df::NT, 2) bulk_kernel(const DfParams p) {
+  extern __shared__ __align__(16) double sm[];
+  __shared__ int s_task;
+  ticket_loop<true>(p, sm, &s_task);
 }
 
 // ------------------------------------------------------------------ host side
@@ -976,6 +1004,9 @@ std::vector<uint32_t> build_tasks(bool potrf, int Mb, int Nb, bool crit) {
 
 std::mutex g_mu;
 std::map<std::tuple<int, int, int, int>, std::pair<uint32_t*, int>> g_tables;  // (dev, mode, Mb, Nb)
+// mode 2 (POTRF without the chain): ticket at which the tasks of panel step s start
+// (the position P(s) has in the full order), s = 0..Nb
+std::map<std::pair<int, int>, std::vector<int>> g_step_ticket;  // (Mb, Nb)
 int g_num_sms[64];
 
 // mode: 0 TRSM, 1 POTRF (all tasks), 2 POTRF without the critical chain
@@ -993,6 +1024,15 @@ cudaError_t get_table(int mode, int Mb, int Nb, const uint32_t** out, int* count
   // Must not be called while a stream is being captured (cudaMemcpy); the runtime
   // calls dataflow_prepare() before capture.
   std::vector<uint32_t> t = build_tasks(mode >= 1, Mb, Nb, mode == 2);
+  if (mode == 2) {
+    std::vector<int> st((size_t)Nb + 1, (int)t.size());
+    int cnt = 0;
+    for (uint32_t c : build_tasks(true, Mb, Nb, false)) {
+      if ((c >> 30) == df::T_P) st[(size_t)(c & 1023)] = cnt;
+      if (!on_chain(c)) ++cnt;
+    }
+    g_step_ticket[{Mb, Nb}] = st;
+  }
   uint32_t* d = nullptr;
   cudaError_t e = cudaMalloc(&d, t.size() * sizeof(uint32_t));
   if (e != cudaSuccess) return e;
@@ -1075,12 +1115,25 @@ static int df_crit() {
 }
 
 cudaError_t dataflow_init_attrs() {
-  return cudaFuncSetAttribute(dataflow_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, df::SMEM_BYTES);
+  cudaError_t e = cudaFuncSetAttribute(dataflow_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, df::SMEM_BYTES);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(bulk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, df::BULK_SMEM_BYTES);
+  return e;
+}
+
+// STF_DF_SPLIT=0: the chain and the block tasks in one launch (round-2 form, A/B)
+static int df_split() {
+  static int v = [] {
+    const char* e = getenv("STF_DF_SPLIT");
+    return e ? atoi(e) : 1;
+  }();
+  return v;
 }
 
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                        unsigned long long* info, int* ws, const Mirrors* mirrors, unsigned long long* trace,
-                       int ctas_override, int pdl_trig) {
+                       int ctas_override, int pdl_trig, cudaGraphNode_t* chain_node) {
+  if (chain_node) *chain_node = nullptr;
   if (n <= 0) return cudaSuccess;
   DfParams p{};
   p.X = A;
@@ -1105,7 +1158,49 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   if (p.crit) ctas = std::min(p.ntasks, std::max(ctas, 2) - 1) + 1;
   p.trace = trace;
   p.trig = pdl_trig;
-  return launch_df(stream, prio, p, ctas);
+  if (!p.crit || !df_split() || p.ntasks == 0) return launch_df(stream, prio, p, ctas);
+  // two launches: the chain (dataflow_kernel, 1 CTA), then bulk_kernel (ctas - 1) released by it
+  e = cudaMemsetAsync(p.ws, 0, dataflow_ws_bytes(p.m, p.n), stream);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributePriority;
+  attr[0].val.priority = prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cfg.blockDim = dim3(df::NT);
+  cfg.stream = stream;
+  cfg.gridDim = dim3(1);
+  cfg.dynamicSmemBytes = df::SMEM_BYTES;
+  DfParams pc = p;
+  pc.trig = 0;  // the chain releases its dependent (the bulk launch) at its start
+  ++launch_count();
+  e = cudaLaunchKernelEx(&cfg, dataflow_kernel, pc);
+  if (e != cudaSuccess) return e;
+  if (chain_node) {
+    cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+    const cudaGraphNode_t* deps = nullptr;
+    size_t nd = 0;
+    if (cudaStreamGetCaptureInfo_v3(stream, &st, nullptr, nullptr, &deps, nullptr, &nd) == cudaSuccess &&
+        st == cudaStreamCaptureStatusActive && nd == 1)
+      *chain_node = deps[0];
+    cudaGetLastError();
+  }
+  // bulk CTAs release TRSM(k+1,k) at the first ticket of panel step pdl_trig
+  DfParams pb = p;
+  pb.trig = -1;
+  if (pdl_trig >= 0) {
+    std::lock_guard<std::mutex> g(g_mu);
+    const std::vector<int>& stt = g_step_ticket[{p.Mb, p.Nb}];
+    pb.trig = stt.empty() ? 0 : stt[(size_t)std::min(pdl_trig, p.Nb)];
+  }
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.numAttrs = 2;
+  cfg.gridDim = dim3(ctas - 1);
+  cfg.dynamicSmemBytes = df::BULK_SMEM_BYTES;
+  ++launch_count();
+  return cudaLaunchKernelEx(&cfg, bulk_kernel, pb);
 }
 
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,

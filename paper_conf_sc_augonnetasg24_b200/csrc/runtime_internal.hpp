@@ -67,7 +67,7 @@ struct Options {
   int64_t mem_cap_tiles = 0;   // HOST_COLMAJOR on one GPU: device tile frames (0 = no cap)
   int64_t ooc_order = -1;      // out-of-core program order: 0 tall, 1 2D-blocked, -1 auto
   int64_t host_stream = 1;     // HOST_COLMAJOR on one GPU, nb >= 512, T >= 16: frame-per-tile OOC builder
-  int64_t trsm_res_tail = 4096;  // trsm 3: resident panel for every TRSM once n - k nb <= this
+  int64_t trsm_res_tail = -1;   // -1 auto: 4096 at nb >= 1024 (n = 8192 +7%), else 8192 (nb = 512 +6%)  // trsm 3: resident panel for every TRSM once n - k nb <= this
   int64_t trsm_rows = 128;     // row panel: rows per CTA (32, 64, 128)
   int64_t trsm_res_split = 2;  // resident-panel TRSMs in 2 (or 4) column parts with GEMMs between; 1 = one launch
   int64_t gemm_merge = 2;      // D > 0: merged tile updates for tiles >= D columns right of the panel
@@ -135,6 +135,7 @@ constexpr size_t kCacheMax = 4;
 // the capture edge from kernel node `from` into a programmatic one.
 cudaGraphNode_t capture_last_node(cudaStream_t s);
 int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from);
+int capture_drop_dependency(cudaStream_t s, cudaGraphNode_t from);
 
 struct Exec {
   // key
@@ -154,6 +155,7 @@ struct Exec {
   std::vector<int*> task_ws;                  // per task: dataflow-kernel workspace (POTRF/TRSM), else null
   std::vector<int64_t> pdl_src;               // per task: TRSM(k+1,k) -> index of POTRF(k) it may overlap, else -1
   std::vector<cudaGraphNode_t> cap_node;      // per task: its last captured node (POTRFs with a pdl consumer)
+  std::vector<cudaGraphNode_t> cap_node2;     // per task: a POTRF's chain node (its first launch)
   std::vector<cudaEvent_t> events;            // per task, null if not needed
   std::vector<int> events_dev;
   cudaGraph_t graph = nullptr;

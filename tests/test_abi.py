@@ -88,7 +88,7 @@ def test_init_without_gpu_fails_cleanly():
 
 OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (3, 1), "streams": (32, 3), "serial": (0, 1),
            "priority": (1, 0), "grid_p": (0, 2), "lookahead": (1, 0), "threads": (8, 2), "trsm_split": (4, 2), "push": (0, 2),
-           "trsm_res_tail": (4096, 0), "trsm_rows": (128, 64), "trsm_res_split": (2, 1), "stream_pool": (0, 1),
+           "trsm_res_tail": (-1, 0), "trsm_rows": (128, 64), "trsm_res_split": (2, 1), "stream_pool": (0, 1),
            "order_mode": (-1, 2), "order_tail": (-1, 0), "order_asap": (0, 1), "sched_width": (0, 3), "prio_mode": (0, 2),
            "ooc_reorder": (1, 0), "dev_order": (0, 1), "ooc_budget_pct": (-1, 40), "host_stream_budget_pct": (90, 75),
            "host_eager": (0, 1), "mem_cap_tiles": (0, 10), "ooc_order": (-1, 0), "host_stream": (1, 0), "pdl": (1, 0), "pdl_lead": (8, 16),
