@@ -11,7 +11,7 @@ prof gemm_tile gemm_nt 1 1 0 1024 1024 1024
 prof gemm_full gemm_nt 1 1 0 8192 8192 1024
 prof syrk_tile gemm_nt 1 1 1 1024 1024 1024
 prof trsm_tile "trsm_res|gemm_nt" 3 3 2 1024 1024 0
-prof potrf_tile dataflow 1 1 3 1024 1024 0
+prof potrf_tile "dataflow|bulk" 2 2 3 1024 1024 0
 for cfg in "65536 1024" "32768 1024"; do
   set -- $cfg
   timeout 1500 ncu --graph-profiling graph --nvtx --nvtx-include "stf_potrf/" --clock-control none \
