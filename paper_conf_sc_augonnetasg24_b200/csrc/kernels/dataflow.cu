@@ -369,13 +369,12 @@ __device__ __forceinline__ void st_release_s(int* p, int v) {
 // Correctly rounded sqrt and division (div_by with y = RN(1/s)); every element
 // receives its updates in increasing column order, each a single fma or a DMMA
 // k-step pair: the same operations as without look-ahead, deterministic.
-// (An rsqrt issued next to the sqrt plus one Newton step against the rounded s
-// gives the same y = RN(1/s) -- tools/check_rcp.cu, 0 mismatches in 3 x 2^32
-// pivots -- but P(kb) measured 7% slower with it: warp 0 is issue-bound as much as
-// latency-bound, tools/p_lab.cu, profiles/r02/potrf_chain.txt.)
-// Non-positive pivot (or NaN): info = min(info, col0 + col + 1), s = NaN.
-template <bool kRsq = false>
-__device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info, int* dpanel) {
+// The pivot's sqrt and reciprocal are the library's (IEEE); a branch-free
+// rsqrt-based form with the same bits (tools/check_rcp.cu: 0 mismatches in 5 x 2^32
+// operands) shortens the chain in isolation (tools/p_lab.cu: P 11.2 -> 10.1 us) but
+// made the POTRF tile slower in the factorisation kernel (354 -> 370 us, same box,
+// profiles/r02/potrf_chain.txt), so it is not used.
+__device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info, int* dpanel, double* Ypub = nullptr) {
   constexpr int LD = df::LDB, BAR_DONE = 1, BAR_NEXT = 2, GRP = 128;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
   const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
@@ -387,7 +386,7 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
     auto panel = [&](int p, auto V1, auto V2) {
       constexpr bool kV1 = decltype(V1)::value, kV2 = decltype(V2)::value;
       const int c0 = 8 * p;
-      double dg[8][8];
+      double dg[8][8], yp[8];
 #pragma unroll
       for (int i = 0; i < 8; ++i)
 #pragma unroll
@@ -405,16 +404,9 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
         const double d = dg[i][i];
         const bool ok = d > 0.0;
         if (!ok && bad == 0) bad = c0 + i + 1;
-        double sq, y;
-        if (kRsq) {
-          const double rs = rsqrt(d);
-          sq = ok ? sqrt(d) : kNaN;
-          y = fma(rs, fma(-sq, rs, 1.0), rs);
-        } else {
-          sq = ok ? sqrt(d) : kNaN;
-          y = 1.0 / sq;
-        }
+        const double sq = ok ? sqrt(d) : kNaN, y = 1.0 / sq;
         dg[i][i] = sq;
+        yp[i] = y;
 #pragma unroll
         for (int r = i + 1; r < 8; ++r) dg[r][i] = div_by(dg[r][i], sq, y);
 #pragma unroll
@@ -435,6 +427,9 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
         for (int i = 0; i < 8; ++i)
 #pragma unroll
           for (int j = 0; j <= i; ++j) D[(c0 + i) * LD + c0 + j] = dg[i][j];
+        if (Ypub)  // the pivots' reciprocals RN(1/L_cc) for the S warps' divisions
+#pragma unroll
+          for (int i = 0; i < 8; ++i) Ypub[c0 + i] = yp[i];
       }
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
@@ -617,7 +612,7 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
   double* Lc = XS;                         // 3 W: chol_core scratch (XS is dead during P)
   double* Dp = XS + 3 * W;                 // W + 2
   double* Xp = Rc + W;                     // 4 x [16 x 64] swizzled panels of S(kb+1, kb)
-  double* Yc = Xp + 4 * 16 * W;            // 4 x W: per S-warp 1 / L_cc
+  double* Yc = Xp + 4 * 16 * W;            // W: 1 / L_cc of L_kk, published by the P warp with each panel (4 W reserved)
   int* dpanel = reinterpret_cast<int*>(Yc + 4 * W);  // panels of P(kb) final so far
   int* prog = p.ws + 2;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
@@ -645,7 +640,7 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
       if (threadIdx.x == 0) *dpanel = 0;
       __syncthreads();
       if (warp < 4) {  // ---- group D: P(kb), then L_kk to global and published
-        chol_block_grp(D, p.col0 + (int64_t)kb * W, p.info, dpanel);
+        chol_block_grp(D, p.col0 + (int64_t)kb * W, p.info, dpanel, Yc);
         for (int idx = threadIdx.x; idx < W * W; idx += 128) {
           const int rr = idx & (W - 1), cc = idx >> 6;
           if (rr >= cc) Xkk[(int64_t)cc * p.ldx + rr] = D[rr * df::LDB + cc];
@@ -698,15 +693,14 @@ __device__ void critical_chain(const DfParams& p, double* sm) {
           }
         }
         bar_sync_id(3, 128);
-        double* Yw = Yc + sw * W;  // this warp's copy of 1 / L_cc (IEEE)
-        auto gate = [&](int P) {   // sub-block P needs panel P of L_kk final
+        // 1 / L_cc: published by the P warp with each panel (RN(1/L_cc), the value the
+        // division by L_cc needs); sub-block P needs panel P of L_kk final
+        auto gate = [&](int P) {
           while (ld_volatile_s(dpanel) <= P) __nanosleep(40);  // keep the issue slots for the P warps
           __threadfence_block();
-          if (lane < 8) Yw[8 * P + lane] = 1.0 / D[(8 * P + lane) * df::LDB + 8 * P + lane];
-          __syncwarp();
         };
         const int rr = 16 * sw + (lane & 15);
-        solve_block<0>(Xp + sw * 16 * W, 0, sb::RowMajor<df::LDB>{D}, Yw, lane, Xik, p.ldx, rr, lane < 16 && rr < rows,
+        solve_block<0>(Xp + sw * 16 * W, 0, sb::RowMajor<df::LDB>{D}, Yc, lane, Xik, p.ldx, rr, lane < 16 && rr < rows,
                        gate);
         __syncwarp();
         for (int m = 0; m < p.mir.n; ++m) {  // fused push of the finished block
@@ -934,12 +928,14 @@ __global__ void __launch_bounds__(df::NT) dataflow_kernel(const DfParams p) {
   ticket_loop<false>(p, sm, &s_task);
 }
 
-// POTRF as two launches: the critical chain alone (dataflow_kernel with one CTA:
-// the register-heavy panel code) and the block tasks (bulk_kernel, 2 CTAs per SM
-// with 70 KB of shared memory: they fit next to a GEMM CTA).  The chain releases
-// the bulk launch at its first step (programmatic dependent launch: both are
-// resident together, each only waits on the other's progress counters); the bulk
-// CTAs release the next dependent (TRSM(k+1,k)) once the tickets reach p.trig.
+// POTRF as two launches: the critical chain plus a few block-task CTAs
+// (dataflow_kernel: the register-heavy panel code, one CTA per SM) and most block
+// tasks (bulk_kernel, 2 CTAs per SM with 70 KB of shared memory: they fit next to
+// a GEMM CTA).  The first launch releases the second at its start (programmatic
+// dependent launch) and both take tickets from one counter; the first can finish
+// every task alone, so the tile completes even when the launches are serialised
+// (profilers, sanitizers).  The bulk CTAs release the next dependent (TRSM(k+1,k))
+// once the tickets reach p.trig.
 __global__ void __launch_bounds__(df::NT, 2) bulk_kernel(const DfParams p) {
   extern __shared__ __align__(16) double sm[];
   __shared__ int s_task;
@@ -1158,8 +1154,9 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   if (p.crit) ctas = std::min(p.ntasks, std::max(ctas, 2) - 1) + 1;
   p.trace = trace;
   p.trig = pdl_trig;
-  if (!p.crit || !df_split() || p.ntasks == 0) return launch_df(stream, prio, p, ctas);
-  // two launches: the chain (dataflow_kernel, 1 CTA), then bulk_kernel (ctas - 1) released by it
+  if (!p.crit || !df_split() || p.ntasks == 0 || ctas < 3) return launch_df(stream, prio, p, ctas);
+  // two launches: the chain + `heavy` block-task CTAs (dataflow_kernel), then bulk_kernel with
+  // the rest of the CTAs, released by the first at its start
   e = cudaMemsetAsync(p.ws, 0, dataflow_ws_bytes(p.m, p.n), stream);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -1170,10 +1167,11 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   cfg.numAttrs = 1;
   cfg.blockDim = dim3(df::NT);
   cfg.stream = stream;
-  cfg.gridDim = dim3(1);
+  const int heavy = std::max(1, std::min(4, (ctas - 1) / 8));
+  cfg.gridDim = dim3(1 + heavy);
   cfg.dynamicSmemBytes = df::SMEM_BYTES;
   DfParams pc = p;
-  pc.trig = 0;  // the chain releases its dependent (the bulk launch) at its start
+  pc.trig = 0;  // releases its dependent (the bulk launch) at its start
   ++launch_count();
   e = cudaLaunchKernelEx(&cfg, dataflow_kernel, pc);
   if (e != cudaSuccess) return e;
@@ -1197,7 +1195,7 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.numAttrs = 2;
-  cfg.gridDim = dim3(ctas - 1);
+  cfg.gridDim = dim3(ctas - 1 - heavy);
   cfg.dynamicSmemBytes = df::BULK_SMEM_BYTES;
   ++launch_count();
   return cudaLaunchKernelEx(&cfg, bulk_kernel, pb);

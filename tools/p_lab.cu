@@ -18,8 +18,7 @@ std::atomic<int64_t>& launch_count() {
 
 using namespace stfk;
 
-// mode bit 0: S warps solve concurrently; bit 1: S warps spin on DMMA (pipe hog) instead;
-// bit 2: IEEE reciprocal of the pivot after the sqrt (round-1/2 form) instead of rsqrt + Newton
+// mode bit 0: S warps solve concurrently; bit 1: S warps spin on DMMA (pipe hog) instead
 __global__ void __launch_bounds__(256, 1) k_p(const double* A, const double* X0, double* L, double* Xo, int mode,
                                               long long* clk) {
   extern __shared__ __align__(16) double sm[];
@@ -39,10 +38,7 @@ __global__ void __launch_bounds__(256, 1) k_p(const double* A, const double* X0,
     __syncthreads();
     long long t0 = clock64();
     if (warp < 4) {
-      if (mode & 4)
-        chol_block_grp<false>(D, 0, nullptr, dpanel);
-      else
-        chol_block_grp<true>(D, 0, nullptr, dpanel);
+      chol_block_grp(D, 0, nullptr, dpanel);
       if (threadIdx.x == 0) clk[rep] = clock64() - t0;
     } else if (mode & 1) {
       const int sw = warp - 4;
@@ -93,10 +89,9 @@ int main() {
   cudaMemcpy(X0, hX, sizeof hX, cudaMemcpyHostToDevice);
   const int smem = (W * df::LDB + 4 * 16 * W + 4 * W) * 8 + 16;
   cudaFuncSetAttribute(k_p, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  const char* names[] = {"P alone", "P + S warps (production)", "P + DMMA hog on warps 4-7", "P alone, IEEE 1/s",
-                         "P + S, IEEE 1/s"};
-  const int modes[] = {0, 1, 2, 4, 5};
-  for (int v = 0; v < 5; ++v) {
+  const char* names[] = {"P alone", "P + S warps (production)", "P + DMMA hog on warps 4-7"};
+  const int modes[] = {0, 1, 2};
+  for (int v = 0; v < 3; ++v) {
     for (int i = 0; i < 16; ++i) clk[i] = 0;
     k_p<<<1, 256, smem>>>(A, X0, L + v * W * W, Xo + v * W * W, modes[v], clk);
     cudaError_t e = cudaDeviceSynchronize();
@@ -107,10 +102,10 @@ int main() {
     printf("%-28s P %6lld clk (%.2f us at 1.965 GHz)  S warps %lld %lld %lld %lld\n", names[v], clk[2],
            clk[2] / 1965.0, clk[4], clk[5], clk[6], clk[7]);
   }
-  static double hL[5][W * W];
+  static double hL[3][W * W];
   cudaMemcpy(hL, L, sizeof hL, cudaMemcpyDeviceToHost);
-  int diff = 0, diff2 = 0;
-  for (int i = 0; i < W * W; ++i) diff += hL[0][i] != hL[1][i], diff2 += hL[0][i] != hL[3][i];
-  printf("bits P alone vs with S: %d mismatches; rsqrt+Newton vs IEEE 1/s: %d mismatches\n", diff, diff2);
+  int diff = 0;
+  for (int i = 0; i < W * W; ++i) diff += hL[0][i] != hL[1][i];
+  printf("bits P alone vs with S: %d mismatches\n", diff);
   return 0;
 }
