@@ -461,6 +461,8 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
                          (n // nb * (n // nb + 1) / 2 * nb * nb * 8 / 1e9),
                    "graph": bool(stats["graph"]), "graph_fallback": bool(stats["graph_fallback"]),
                    "streams": stf.get_option("streams"),
+                   "panel_chain": ("programmatic launch, lead %d blocks (pdl)" % stf.get_option("pdl_lead")
+                                   if stf.get_option("pdl") else "full-completion edges"),
                    "virtual_slots": bool(args.virtual),
                    "processes": ("one per GPU (stf_mp_*, CUDA-IPC replicas, device-side flags)" if mode == "mp"
                                  else "one process drives all %d GPU(s) (stf_potrf)" % N)},
@@ -471,7 +473,7 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
         "e2e": e2e,
         "plan": {k: stats[k] for k in ("tasks", "dag_tasks", "edges", "critical_path", "graph_nodes", "kernel_launches",
                                        "transfers", "transfer_bytes", "pushed", "replicas_max", "data_plane",
-                                       "devices", "slots", "peer_transfers", "merged_gemms", "build_ms")},
+                                       "devices", "slots", "peer_transfers", "merged_gemms", "pdl_edges", "build_ms")},
         "check": check,
         "first_call_ms": round(first_ms, 1) if first_ms else None,
         "step_ms": [round(x, 3) for x in steps_ms],

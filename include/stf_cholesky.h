@@ -228,6 +228,8 @@ typedef struct stf_plan_stats {
   int64_t slots;          /* GPU slots of the call (ngpus) */
   int64_t peer_transfers; /* transfers whose source and destination are distinct devices */
   int64_t merged_gemms;   /* GEMM tasks that carry two consecutive tile updates ("gemm_merge") */
+  int64_t pdl_edges;      /* programmatic graph edges of the panel chain (option "pdl"): a TRSM(k+1,k)
+                             or SYRK(k+1,k) that may launch before its producer ends */
 } stf_plan_stats;
 
 int stf_last_stats(stf_plan_stats *out);

@@ -56,6 +56,7 @@ class stf_plan_stats(ctypes.Structure):
         ("slots", ctypes.c_int64),
         ("peer_transfers", ctypes.c_int64),
         ("merged_gemms", ctypes.c_int64),
+        ("pdl_edges", ctypes.c_int64),
     ]
 
     def as_dict(self):

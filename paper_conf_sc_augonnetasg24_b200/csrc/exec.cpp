@@ -154,7 +154,8 @@ cudaGraphNode_t capture_last_node(cudaStream_t s) {
 // Turn the capture edge from kernel node `from` (a current dependency of stream s)
 // into a programmatic one: the next kernel captured on s may launch once every CTA
 // of `from` has executed griddepcontrol.launch_dependents (or exited).  The other
-// dependencies keep full-completion edges.  No-op when `from` is not a dependency.
+// dependencies keep full-completion edges.  No-op (0) when `from` is not a
+// dependency; 1 when the edge was converted; negative on error.
 int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from) {
   cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
   const cudaGraphNode_t* deps = nullptr;
@@ -176,7 +177,7 @@ int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from) {
   if (!found) return 0;
   CUDA_TRY(cudaStreamUpdateCaptureDependencies_v2(s, d.data(), e.data(), nd, cudaStreamSetCaptureDependencies),
            "programmatic capture edge");
-  return 0;
+  return 1;  // converted
 }
 
 // Remove node `from` from the current capture dependencies of stream s (no-op when absent).
@@ -305,7 +306,8 @@ struct Lowerer {
               if (r) return r;
             }
             int r = capture_make_programmatic(s, X.cap_node[(size_t)src]);
-            if (r) return r;
+            if (r < 0) return r;
+            X.pdl_edges += r;
           }
           // column-block counters for a SYRK(k+1,k) that overlaps this TRSM in turn
           int* kflag = pflag ? X.task_ws[(size_t)src] + 2 + nbk * nbk : nullptr;
@@ -370,7 +372,8 @@ struct Lowerer {
           kflag = X.task_ws[(size_t)X.pdl_src[(size_t)src]] + 2 + nbk * nbk;
           if (!X.cap_node.empty() && X.cap_node[(size_t)src]) {
             int r = capture_make_programmatic(s, X.cap_node[(size_t)src]);
-            if (r) return r;
+            if (r < 0) return r;
+            X.pdl_edges += r;
           }
         }
         const double* A = X.buf[(size_t)t.in[0]];
@@ -615,6 +618,7 @@ int mp_reset_flags(Context& C, Exec& X) {
 
 // fork + every task + join (+ flag reset) on the current capture / eager streams
 int issue_all(Context& C, Exec& X) {
+  X.pdl_edges = 0;
   int r = fork_streams(C, X);
   Lowerer L{C, X};
   if (!r) r = L.issue();
@@ -995,6 +999,7 @@ void fill_plan_stats(const stf::Plan& P, int64_t nb, stf_plan_stats* s) {
 
 void fill_stats(const Exec& X, bool hit, stf_plan_stats* s) {
   fill_plan_stats(X.plan, X.nb, s);
+  s->pdl_edges = X.pdl_edges;
   s->graph_nodes = X.graph_nodes;
   s->kernel_launches = X.launches;
   s->build_ms = hit ? 0.0 : X.build_ms;

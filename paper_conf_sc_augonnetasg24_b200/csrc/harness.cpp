@@ -169,11 +169,11 @@ static int bench_chain(int64_t M, int reps, double* avg_ms) {
       static const int dbg = getenv("STF_DEBUG_CHAIN_MODE") ? atoi(getenv("STF_DEBUG_CHAIN_MODE")) : 0;
       if (chain && !r) r = capture_drop_dependency(s, chain);
       if ((dbg & 2) && extra) step(cudaStreamUpdateCaptureDependencies(s, &extra, 1, cudaStreamAddCaptureDependencies));
-      if (pn && !r) r = capture_make_programmatic(s, pn);
+      if (pn && !r) r = std::min(0, capture_make_programmatic(s, pn));
       int* kflag = ws + 2 + nbk * nbk;
       step(stfk::trsm_res(s, 0, (int)M, (int)M, A, M, B, M, nullptr, nullptr, ws + 2, nbk, kflag, trig));
       cudaGraphNode_t tn = capture_last_node(s);
-      if (tn && !r) r = capture_make_programmatic(s, tn);
+      if (tn && !r) r = std::min(0, capture_make_programmatic(s, tn));
       const double* Bp = B;
       step(stfk::gemm_nt_multi(s, 0, (int)M, (int)M, (int)M, 1, &Bp, M, &Bp, M, Cm, M, 1, 0, kflag,
                                (int)(M / stfk::kTrsmResRows)));

@@ -156,6 +156,7 @@ struct Exec {
   std::vector<int64_t> pdl_src;               // per task: TRSM(k+1,k) -> index of POTRF(k) it may overlap, else -1
   std::vector<cudaGraphNode_t> cap_node;      // per task: its last captured node (POTRFs with a pdl consumer)
   std::vector<cudaGraphNode_t> cap_node2;     // per task: a POTRF's chain node (its first launch)
+  int64_t pdl_edges = 0;                      // programmatic capture edges of the last capture
   std::vector<cudaEvent_t> events;            // per task, null if not needed
   std::vector<int> events_dev;
   cudaGraph_t graph = nullptr;

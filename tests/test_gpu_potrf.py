@@ -428,6 +428,20 @@ def test_chain_overlap_p2_exact(stf, lead):
         assert st["graph"] == 1 and st["graph_fallback"] == 0
 
 
+def test_chain_overlap_edges_reported(stf):
+    """The plan statistics count the programmatic edges of the panel chain: two per
+    panel step (TRSM(k+1,k), SYRK(k+1,k)) with the graph backend, none without pdl
+    or with the eager backend."""
+    n, nb = 4096, 1024
+    T = n // nb
+    for opts, want in (({"pdl": 1}, 2 * (T - 1)), ({"pdl": 0}, 0), ({"pdl": 1, "graph": 0}, 0)):
+        _options(stf, **opts)
+        M, info = _factor_spd(stf, n, nb, seed=2)
+        assert info == 0
+        assert stf.last_stats()["pdl_edges"] == want, opts
+    _options(stf, pdl=1, graph=1)
+
+
 def test_chain_step_bench_overlap_is_faster(stf):
     """stf_bench_kernel kind 4 (POTRF -> TRSM -> SYRK on 1024 tiles, one graph): the
     programmatic overlap shortens the chain step (measured 507 -> 374 us)."""
