@@ -184,6 +184,12 @@ const char *stf_last_error(void);
  *                           resident-panel launch (trsm_res_split does not apply to it) in
  *                           every grid, so the bits do not depend on where it runs; they
  *                           equal pdl = 0 with trsm_res_split = 1 (tested)
+ *   "potrf_split" STF_POTRF_SPLIT 1 (default): a POTRF tile is two launches -- the critical-chain
+ *                           CTA with a few block-task CTAs, then 2-per-SM block-task CTAs it
+ *                           releases (programmatic launch; the first completes the tile alone
+ *                           when launches are serialised); 0: one launch.  Same bits
+ *   "potrf_ctas" STF_POTRF_CTAS CTAs of a POTRF tile launch (0 default: 3 per 64-block column,
+ *                           16..96); the critical chain needs at least one block-task CTA
  *   "pdl_lead" STF_PDL_LEAD 64-block steps before its end at which a chain kernel lets its
  *                           dependent launch (default 8; >= nb/64: at its start)
  *   "debug_skip" STF_DEBUG_SKIP bit mask (or names potrf,trsm,syrk,gemm,copy,trsm_as_gemm,

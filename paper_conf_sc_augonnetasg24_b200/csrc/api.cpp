@@ -73,6 +73,8 @@ const std::vector<OptDesc>& option_table() {
       {"stream_pool", "STF_STREAM_POOL", &Options::stream_pool, 0, 2, true},
       {"pdl", "STF_PDL", &Options::pdl, 0, 1, true},
       {"pdl_lead", "STF_PDL_LEAD", &Options::pdl_lead, 0, 1024, true},
+      {"potrf_split", "STF_POTRF_SPLIT", &Options::potrf_split, 0, 1, true},
+      {"potrf_ctas", "STF_POTRF_CTAS", &Options::potrf_ctas, 0, 1024, true},
       {"debug_skip", "STF_DEBUG_SKIP", &Options::debug_skip, 0, INT64_MAX, true},
       {"debug_trace", "STF_DEBUG_TRACE", &Options::debug_trace, 0, 1, true},
       {"nvtx", "STF_NVTX", &Options::nvtx, 0, 1, false},

@@ -263,7 +263,7 @@ struct Lowerer {
           const int trig = X.opt.pdl ? (int)std::max<int64_t>(0, nbk - X.opt.pdl_lead) : -1;
           cudaGraphNode_t chain = nullptr;
           CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir,
-                                    nullptr, 0, trig, &chain),
+                                    nullptr, (int)X.opt.potrf_ctas, trig, &chain, (int)X.opt.potrf_split),
                    "POTRF launch");
           if (!X.cap_node.empty()) X.cap_node[tidx] = capture_last_node(s);  // the block-task launch
           if (chain) {

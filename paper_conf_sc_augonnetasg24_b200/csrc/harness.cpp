@@ -104,7 +104,8 @@ int stf_kernel_potrf(int64_t n, double* A, int64_t lda, int64_t* info) {
   cudaError_t e = cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)n, (int)n));
   if (e == cudaSuccess) e = stfk::info_reset(0, d_info);
   if (e == cudaSuccess)
-    e = ctx().opt.dataflow ? stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws)
+    e = ctx().opt.dataflow ? stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws, nullptr, nullptr,
+                                              (int)ctx().opt.potrf_ctas, -1, nullptr, (int)ctx().opt.potrf_split)
                            : stfk::potrf_lower(0, 0, (int)n, A, lda, 0, d_info);
   unsigned long long v = ULLONG_MAX;
   if (e == cudaSuccess) e = cudaMemcpy(&v, d_info, sizeof v, cudaMemcpyDeviceToHost);
@@ -161,7 +162,8 @@ static int bench_chain(int64_t M, int reps, double* avg_ms) {
     const int nbk = (int)(M / 64);
     const int trig = pdl ? (int)std::max<int64_t>(0, nbk - o.pdl_lead) : -1;
     cudaGraphNode_t chain = nullptr;
-    step(stfk::potrf_tile(s, 0, (int)M, A, M, 0, info, ws, nullptr, nullptr, 0, trig, &chain));
+    step(stfk::potrf_tile(s, 0, (int)M, A, M, 0, info, ws, nullptr, nullptr, (int)o.potrf_ctas, trig, &chain,
+                          (int)o.potrf_split));
     cudaGraphNode_t pn = capture_last_node(s);
     if (chain) step(cudaStreamUpdateCaptureDependencies(s, &chain, 1, cudaStreamAddCaptureDependencies));
     if (pdl) {
@@ -288,7 +290,8 @@ int stf_bench_kernel(int kind, int64_t M, int64_t N, int64_t K, int reps, double
                            : stfk::trsm_rlt(s, 0, (int)M, (int)N, Src, ldm, Cm, ldm));
           break;
         case 3:
-          step(dataflow ? stfk::potrf_tile(s, 0, (int)M, Cm, ldm, 0, info, ws)
+          step(dataflow ? stfk::potrf_tile(s, 0, (int)M, Cm, ldm, 0, info, ws, nullptr, nullptr,
+                                           (int)ctx().opt.potrf_ctas, -1, nullptr, (int)ctx().opt.potrf_split)
                         : stfk::potrf_lower(s, 0, (int)M, Cm, ldm, 0, info));
           break;
       }
@@ -337,7 +340,9 @@ int64_t stf_debug_potrf_trace(int64_t n, double* A, int64_t lda, int ctas, int64
   if (e == cudaSuccess) e = cudaMalloc(&ws, stfk::dataflow_ws_bytes((int)n, (int)n));
   if (e == cudaSuccess) e = stfk::dataflow_prepare((int)n, (int)n, true);
   if (e == cudaSuccess) e = stfk::info_reset(0, d_info);
-  if (e == cudaSuccess) e = stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws, nullptr, d_tr, ctas);
+  if (e == cudaSuccess)
+    e = stfk::potrf_tile(0, 0, (int)n, A, lda, 0, d_info, ws, nullptr, d_tr, ctas > 0 ? ctas : (int)ctx().opt.potrf_ctas,
+                         -1, nullptr, (int)ctx().opt.potrf_split);
   if (e == cudaSuccess) e = cudaStreamSynchronize(0);
   const int64_t cnt = std::min<int64_t>(cap, slots);
   if (e == cudaSuccess && trace) e = cudaMemcpy(trace, d_tr, (size_t)cnt * 8, cudaMemcpyDeviceToHost);

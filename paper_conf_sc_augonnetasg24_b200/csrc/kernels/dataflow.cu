@@ -1040,19 +1040,12 @@ cudaError_t get_table(int mode, int Mb, int Nb, const uint32_t** out, int* count
   return cudaSuccess;
 }
 
-// CTAs of a dataflow POTRF launch: STF_DF_CTAS, else 3 per 64-block column
+// CTAs of a dataflow POTRF launch (option potrf_ctas = 0): 3 per 64-block column
 // (16 .. 96): the critical chain needs the bulk updates of the next columns
 // done in time (profiles: nb = 1024 0.69 -> 0.59 ms, nb = 2048 3.4 -> 1.3 ms at 2
 // per column; with the look-ahead P of round 2 the chain waited for its S input
 // at 2 per column: 396 -> 375 us at 3, tools/potrf_trace.py).
-int df_max_ctas(int T = 16) {
-  static int v = [] {
-    const char* e = getenv("STF_DF_CTAS");
-    return e ? atoi(e) : 0;
-  }();
-  if (v > 0) return v;
-  return std::min(96, std::max(16, 3 * T));
-}
+int df_max_ctas(int T = 16) { return std::min(96, std::max(16, 3 * T)); }
 
 int num_sms() {
   int dev = 0;
@@ -1117,18 +1110,11 @@ cudaError_t dataflow_init_attrs() {
   return e;
 }
 
-// STF_DF_SPLIT=0: the chain and the block tasks in one launch (round-2 form, A/B)
-static int df_split() {
-  static int v = [] {
-    const char* e = getenv("STF_DF_SPLIT");
-    return e ? atoi(e) : 1;
-  }();
-  return v;
-}
+
 
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                        unsigned long long* info, int* ws, const Mirrors* mirrors, unsigned long long* trace,
-                       int ctas_override, int pdl_trig, cudaGraphNode_t* chain_node) {
+                       int ctas_override, int pdl_trig, cudaGraphNode_t* chain_node, int split) {
   if (chain_node) *chain_node = nullptr;
   if (n <= 0) return cudaSuccess;
   DfParams p{};
@@ -1154,7 +1140,7 @@ cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t 
   if (p.crit) ctas = std::min(p.ntasks, std::max(ctas, 2) - 1) + 1;
   p.trace = trace;
   p.trig = pdl_trig;
-  if (!p.crit || !df_split() || p.ntasks == 0 || ctas < 3) return launch_df(stream, prio, p, ctas);
+  if (!p.crit || !split || p.ntasks == 0 || ctas < 3) return launch_df(stream, prio, p, ctas);
   // two launches: the chain + `heavy` block-task CTAs (dataflow_kernel), then bulk_kernel with
   // the rest of the CTAs, released by the first at its start
   e = cudaMemsetAsync(p.ws, 0, dataflow_ws_bytes(p.m, p.n), stream);

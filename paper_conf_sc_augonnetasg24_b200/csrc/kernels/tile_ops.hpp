@@ -69,9 +69,10 @@ struct Mirrors {
 cudaError_t potrf_tile(cudaStream_t stream, int prio, int n, double* A, int64_t lda, int64_t col0,
                        unsigned long long* info, int* ws, const Mirrors* mirrors = nullptr,
                        unsigned long long* trace = nullptr, int ctas = 0, int pdl_trig = -1,
-                       cudaGraphNode_t* chain_node = nullptr);
-// (POTRF is two launches on `stream` -- the critical chain, then the block tasks
-// released by it through programmatic dependent launch; when capturing, *chain_node
+                       cudaGraphNode_t* chain_node = nullptr, int split = 1);
+// (With split, POTRF is two launches on `stream` -- the critical chain with a few
+// block-task CTAs, then the other block-task CTAs released by it through
+// programmatic dependent launch; ctas > 0 overrides the CTA count; when capturing, *chain_node
 // returns the chain's graph node: work that needs the finished tile must depend on
 // it as well as on the stream's last node.)
 cudaError_t trsm_tile(cudaStream_t stream, int prio, int M, int n, const double* L, int64_t ldl, double* B,

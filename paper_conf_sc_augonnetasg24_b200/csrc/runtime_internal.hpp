@@ -84,6 +84,8 @@ struct Options {
   int64_t host_eager = 0;      // 1: HOST_COLMAJOR calls on pinned memory lowered eagerly
   int64_t stream_pool = 0;     // 0 default pool; 1 one compute + one copy stream per slot; 2 one stream (ablations)
   int64_t pdl = 1;             // programmatic dependent launch: TRSM(k+1,k) overlaps POTRF(k) (graph backend)
+  int64_t potrf_split = 1;     // POTRF tile as two launches (chain + few block tasks, then 2-per-SM block tasks)
+  int64_t potrf_ctas = 0;      // CTAs of a POTRF tile launch (0: 3 per 64-block column, 16..96)
   int64_t pdl_lead = 8;        // pdl: the POTRF lets its TRSM start this many 64-block steps before its end
   int64_t debug_skip = 0;      // bit mask of task kinds not launched (timing what-ifs; results invalid)
   int64_t debug_trace = 0;     // timing events around every task (one slot)
