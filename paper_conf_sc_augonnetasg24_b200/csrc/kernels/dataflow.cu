@@ -1041,10 +1041,12 @@ cudaError_t get_table(int mode, int Mb, int Nb, const uint32_t** out, int* count
 }
 
 // CTAs of a dataflow POTRF launch (option potrf_ctas = 0): 3 per 64-block column
-// (16 .. 96): the critical chain needs the bulk updates of the next columns
-// done in time (profiles: nb = 1024 0.69 -> 0.59 ms, nb = 2048 3.4 -> 1.3 ms at 2
-// per column; with the look-ahead P of round 2 the chain waited for its S input
-// at 2 per column: 396 -> 375 us at 3, tools/potrf_trace.py).
+// (16 .. 96) for one launch: the critical chain needs the bulk updates of the next
+// columns done in time (profiles: nb = 1024 0.69 -> 0.59 ms, nb = 2048 3.4 -> 1.3 ms
+// at 2 per column; with the look-ahead P of round 2 the chain waited for its S input
+// at 2 per column: 396 -> 375 us at 3, tools/potrf_trace.py).  With the two-launch
+// form, 2 per column measured n = 8192 -0.7%, n = 16384 -0.2%, n = 32768 -0.1% time
+// against 3 but the tile alone 348 -> 369 us (profiles/r02/split_potrf.txt): 3 kept.
 int df_max_ctas(int T = 16) { return std::min(96, std::max(16, 3 * T)); }
 
 int num_sms() {
