@@ -380,11 +380,12 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
   const double kNaN = __longlong_as_double(0x7ff8000000000000LL);
   if (warp == 0) {
     int bad = 0;
-    // one panel; the rows below it live in v1 (rows lane) and v2 (rows lane + 32), each
-    // stream only while some of its rows lie below the panel (v1: p <= 2, v2: p <= 6),
-    // so the warp issues no FP64 work for rows that are all above it
-    auto panel = [&](int p, auto V1, auto V2) {
-      constexpr bool kV1 = decltype(V1)::value, kV2 = decltype(V2)::value;
+    // one panel; the rows below it live in v1 (rows lane) and v2 (rows lane + 32).
+    // (Instantiating it per panel range without the row streams that lie wholly above
+    // the panel saves FP64 issue slots but made the tile 2% slower: the larger kernel
+    // code; profiles/r02/potrf_chain.txt.)
+    auto panel = [&](int p) {
+      constexpr bool kV1 = true, kV2 = true;
       const int c0 = 8 * p;
       double dg[8][8], yp[8];
 #pragma unroll
@@ -440,12 +441,7 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
 #pragma unroll 1
     for (int p = 0; p < 8; ++p) {
       if (p > 0) bar_sync_id(BAR_NEXT, GRP);
-      if (p <= 2)
-        panel(p, std::true_type{}, std::true_type{});
-      else if (p <= 6)
-        panel(p, std::false_type{}, std::true_type{});
-      else
-        panel(p, std::false_type{}, std::false_type{});
+      panel(p);
       __syncwarp();
       if (lane == 0) st_release_s(dpanel, p + 1);  // panel p is final: the S warps may use it
       bar_arrive_id(BAR_DONE, GRP);
