@@ -31,6 +31,8 @@ VARIANTS = [
     ("1 GPU: no priorities (priority=0)", {"STF_PRIO": "0"}, ONE),
     ("1 GPU: no look-ahead, fence per panel step (lookahead=0)", {"STF_LOOKAHEAD": "0"}, ONE),
     ("1 GPU: eager streams + events, no graph (graph=0)", {"STF_GRAPH": "0"}, ONE),
+    ("1 GPU: panel chain with full-completion edges (pdl=0)", {"STF_PDL": "0"}, ONE),
+    ("1 GPU: POTRF tile as one launch (potrf_split=0)", {"STF_POTRF_SPLIT": "0"}, ONE),
     ("8 virtual slots: 2D block-cyclic 2x4 (default)", {}, VIRT + ["--grid", "2x4"]),
     ("8 virtual slots: 1D column block-cyclic 1x8", {}, VIRT + ["--grid", "1x8"]),
     ("8 virtual slots: 1D column block-cyclic 1x8 + fence per step (cuSolverMg model)", {"STF_LOOKAHEAD": "0"},
