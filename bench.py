@@ -160,6 +160,24 @@ def p2_check(tiles, n, nb, owned=None):
         by_dev.setdefault(t.device, []).append(ij)
     L0s = {}
     for dev in by_dev:
+        free, _ = torch.cuda.mem_get_info(dev)
+        if n * n * 8 > free // 2:
+            # the full L0 does not fit next to the tiles (n = 131072: 128 GiB): accumulate
+            # A_ij = sum_k L0_ik L0_jk^T panel by panel (exact in any order, P2) and let
+            # p2_compare regenerate the reference blocks
+            T = n // nb
+            mine = set(by_dev[dev])
+            for ij in mine:
+                tiles[ij].zero_()
+            for k in range(T):
+                P = dyadic_unit_lower_block_torch(101, n, k * nb, k * nb, n - k * nb, nb, device=dev)
+                for (i, j) in mine:
+                    if j >= k:
+                        tiles[(i, j)] += (P[(i - k) * nb:(i - k + 1) * nb] @ P[(j - k) * nb:(j - k + 1) * nb].T).T
+                del P
+            L0s[dev] = None
+            torch.cuda.synchronize(dev)
+            continue
         L0 = torch.empty((n, n), dtype=torch.float64, device=dev)
         for r in range(0, n, 4096):
             L0[r:r + 4096] = dyadic_unit_lower_block_torch(101, n, r, 0, min(4096, n - r), n, device=dev)
@@ -171,13 +189,17 @@ def p2_check(tiles, n, nb, owned=None):
     return L0s
 
 
-def p2_compare(tiles, L0s, nb):
+def p2_compare(tiles, L0s, nb, n):
     import torch
+
+    from synth.spd import dyadic_unit_lower_block_torch
 
     bad = 0
     for (i, j), t in tiles.items():
         got = t.T
-        ref = L0s[t.device][i * nb:(i + 1) * nb, j * nb:(j + 1) * nb]
+        L0 = L0s[t.device]
+        ref = (L0[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb] if L0 is not None else
+               dyadic_unit_lower_block_torch(101, n, i * nb, j * nb, nb, nb, device=t.device))
         if i == j:
             got, ref = torch.tril(got), torch.tril(ref)
         bad += not torch.equal(got, ref)
@@ -284,7 +306,7 @@ def run_ours(args, rank, world):
         if not args.no_check:
             L0s = p2_check(M.tiles, n, nb)
             info = M.potrf()
-            ntile, bad = p2_compare(M.tiles, L0s, nb)
+            ntile, bad = p2_compare(M.tiles, L0s, nb, n)
             del L0s
             check = {"input": "P2 dyadic A = L0 L0^T (m=25, seed 101), same plan, after the timed steps",
                      "info": info, "tiles_checked": ntile, "tiles_mismatched": bad, "bit_exact": bad == 0 and info == 0}
@@ -356,7 +378,7 @@ def run_mp(args, rank, world, P, Q):
         dist.barrier()
         info = A.potrf()
         dist.barrier()
-        ntile, bad = p2_compare(A.tiles, L0s, nb)
+        ntile, bad = p2_compare(A.tiles, L0s, nb, n)
         del L0s
         torch.cuda.empty_cache()
         got = [None] * world
