@@ -33,7 +33,6 @@
 #include <map>
 #include <mutex>
 #include <tuple>
-#include <type_traits>
 #include <vector>
 
 #include "ptx.cuh"
@@ -385,7 +384,6 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
     // the panel saves FP64 issue slots but made the tile 2% slower: the larger kernel
     // code; profiles/r02/potrf_chain.txt.)
     auto panel = [&](int p) {
-      constexpr bool kV1 = true, kV2 = true;
       const int c0 = 8 * p;
       double dg[8][8], yp[8];
 #pragma unroll
@@ -393,12 +391,12 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
 #pragma unroll
         for (int j = 0; j <= i; ++j) dg[i][j] = D[(c0 + i) * LD + c0 + j];
       const int r1 = lane, r2 = lane + 32;
-      const bool b1 = kV1 && r1 >= c0 + 8, b2 = kV2 && r2 >= c0 + 8;
+      const bool b1 = r1 >= c0 + 8, b2 = r2 >= c0 + 8;
       double v1[8], v2[8];
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
-        if (kV1) v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
-        if (kV2) v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
+        v1[j] = b1 ? D[r1 * LD + c0 + j] : 0.0;
+        v2[j] = b2 ? D[r2 * LD + c0 + j] : 0.0;
       }
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
@@ -414,12 +412,12 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
         for (int r = i + 1; r < 8; ++r)
 #pragma unroll
           for (int c = i + 1; c <= r; ++c) dg[r][c] = fma(-dg[r][i], dg[c][i], dg[r][c]);
-        if (kV1) v1[i] = div_by(v1[i], sq, y);
-        if (kV2) v2[i] = div_by(v2[i], sq, y);
+        v1[i] = div_by(v1[i], sq, y);
+        v2[i] = div_by(v2[i], sq, y);
 #pragma unroll
         for (int c = i + 1; c < 8; ++c) {
-          if (kV1) v1[c] = fma(-v1[i], dg[c][i], v1[c]);
-          if (kV2) v2[c] = fma(-v2[i], dg[c][i], v2[c]);
+          v1[c] = fma(-v1[i], dg[c][i], v1[c]);
+          v2[c] = fma(-v2[i], dg[c][i], v2[c]);
         }
       }
       __syncwarp();  // every lane has read the diagonal block before lane 0 overwrites it
@@ -434,8 +432,8 @@ __device__ void chol_block_grp(double* D, int64_t col0, unsigned long long* info
       }
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
-        if (kV1 && b1) D[r1 * LD + c0 + j] = v1[j];
-        if (kV2 && b2) D[r2 * LD + c0 + j] = v2[j];
+        if (b1) D[r1 * LD + c0 + j] = v1[j];
+        if (b2) D[r2 * LD + c0 + j] = v2[j];
       }
     };
 #pragma unroll 1
