@@ -151,3 +151,29 @@ def test_generator_bits_match_synth(abi):
         got = t.cpu().numpy().T
         ref = synth.spd_block(7, n, r0, c0, rows, cols)
         assert np.array_equal(got.view(np.uint64), np.ascontiguousarray(ref).view(np.uint64))
+
+
+def test_potrf_tile_completes_with_serialised_launches():
+    """The two-launch POTRF tile (option potrf_split) must complete when its launches
+    run one after the other (CUDA_LAUNCH_BLOCKING=1, as under profilers and
+    sanitizers): the first launch carries block-task CTAs of its own.  Run in a
+    subprocess with a timeout, so a hang fails the test instead of the suite."""
+    import os
+    import subprocess
+    import sys
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = (
+        "import ctypes, sys; sys.path.insert(0, %r); import numpy as np; import oracle, synth\n"
+        "from gpu_util import to_dev, from_dev\n"
+        "from paper_conf_sc_augonnetasg24_b200 import _abi\n"
+        "n = 1024; A = synth.spd_matrix(31, n); dA = to_dev(A, n); info = ctypes.c_int64(-7)\n"
+        "assert _abi.stf_kernel_potrf(n, dA.data_ptr(), n, ctypes.byref(info)) == 0\n"
+        "L = np.tril(from_dev(dA, n)); Lo, _ = oracle.potrf(A)\n"
+        "print(info.value, np.linalg.norm(L - Lo) / np.linalg.norm(Lo))\n" % root)
+    env = dict(os.environ, CUDA_LAUNCH_BLOCKING="1", STF_POTRF_SPLIT="1",
+               PYTHONPATH=os.pathsep.join([root, os.path.join(root, "tests")]))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, timeout=300)
+    assert r.returncode == 0, r.stderr[-800:]
+    info, rel = r.stdout.split()
+    assert int(info) == 0 and float(rel) <= 1e-13
