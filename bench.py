@@ -163,18 +163,9 @@ def p2_check(tiles, n, nb, owned=None):
         free, _ = torch.cuda.mem_get_info(dev)
         if n * n * 8 > free // 2:
             # the full L0 does not fit next to the tiles (n = 131072: 128 GiB): accumulate
-            # A_ij = sum_k L0_ik L0_jk^T panel by panel (exact in any order, P2) and let
-            # p2_compare regenerate the reference blocks
-            T = n // nb
-            mine = set(by_dev[dev])
-            for ij in mine:
-                tiles[ij].zero_()
-            for k in range(T):
-                P = dyadic_unit_lower_block_torch(101, n, k * nb, k * nb, n - k * nb, nb, device=dev)
-                for (i, j) in mine:
-                    if j >= k:
-                        tiles[(i, j)] += (P[(i - k) * nb:(i - k + 1) * nb] @ P[(j - k) * nb:(j - k + 1) * nb].T).T
-                del P
+            # A_ij = sum_k L0_ik L0_jk^T panel by panel and let p2_compare regenerate the
+            # reference blocks
+            p2_fill_by_panels(tiles, by_dev[dev], n, nb, dev)
             L0s[dev] = None
             torch.cuda.synchronize(dev)
             continue
@@ -187,6 +178,22 @@ def p2_check(tiles, n, nb, owned=None):
             tiles[(i, j)].copy_((L0[i * nb:(i + 1) * nb, :K] @ L0[j * nb:(j + 1) * nb, :K].T).T)
         torch.cuda.synchronize(dev)
     return L0s
+
+
+def p2_fill_by_panels(tiles, mine, n, nb, dev):
+    """Tiles (i, j) in `mine` <- (L0 L0^T)_ij accumulated over the column panels k of L0
+    (P2: exact in FP64 in any summation order); only one n x nb panel of L0 is held."""
+    from synth.spd import dyadic_unit_lower_block_torch
+
+    mine = set(mine)
+    for ij in mine:
+        tiles[ij].zero_()
+    for k in range(n // nb):
+        P = dyadic_unit_lower_block_torch(101, n, k * nb, k * nb, n - k * nb, nb, device=dev)
+        for (i, j) in mine:
+            if j >= k:
+                tiles[(i, j)] += (P[(i - k) * nb:(i - k + 1) * nb] @ P[(j - k) * nb:(j - k + 1) * nb].T).T
+        del P
 
 
 def p2_compare(tiles, L0s, nb, n):

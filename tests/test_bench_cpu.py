@@ -71,3 +71,26 @@ def test_max_over_ranks_gloo(tmp_path):
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stderr[-2000:]
     assert "RANK0 MAX 20.0" in r.stdout and "RANK1 MAX 20.0" in r.stdout
+
+
+def test_p2_fill_by_panels_matches_the_full_product():
+    """bench.py's memory-light P2 input (used when the full L0 does not fit, n = 131072)
+    equals the tiles of L0 L0^T formed at once, bit for bit (P2 is exact in any order)."""
+    import importlib.util
+
+    import numpy as np
+    import torch
+
+    import synth
+
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    bench = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(bench)
+    n, nb = 256, 64
+    T = n // nb
+    tiles = {(i, j): torch.empty((nb, nb), dtype=torch.float64) for i in range(T) for j in range(i + 1)}
+    bench.p2_fill_by_panels(tiles, list(tiles), n, nb, "cpu")
+    A, _ = synth.dyadic_spd(101, n)
+    for (i, j), t in tiles.items():
+        ref = A[i * nb:(i + 1) * nb, j * nb:(j + 1) * nb]
+        assert np.array_equal(t.numpy().T, ref), (i, j)
