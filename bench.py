@@ -490,7 +490,9 @@ def report(args, stf, N, P, Q, total_ms, steps_ms, stats, clk, first_ms, mode, g
                          (n // nb * (n // nb + 1) / 2 * nb * nb * 8 / 1e9),
                    "graph": bool(stats["graph"]), "graph_fallback": bool(stats["graph_fallback"]),
                    "streams": stf.get_option("streams"),
-                   "panel_chain": ("programmatic launch, lead %d blocks (pdl)" % stf.get_option("pdl_lead")
+                   "panel_chain": ("programmatic launch, lead %d blocks (pdl)" % (stf.get_option("pdl_lead") if
+                                                                                 stf.get_option("pdl_lead") >= 0 else
+                                                                                 max(2, nb // 128))
                                    if stf.get_option("pdl") else "full-completion edges"),
                    "virtual_slots": bool(args.virtual),
                    "processes": ("one per GPU (stf_mp_*, CUDA-IPC replicas, device-side flags)" if mode == "mp"

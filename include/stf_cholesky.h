@@ -191,7 +191,8 @@ const char *stf_last_error(void);
  *   "potrf_ctas" STF_POTRF_CTAS CTAs of a POTRF tile launch (0 default: 3 per 64-block column,
  *                           16..96); the critical chain needs at least one block-task CTA
  *   "pdl_lead" STF_PDL_LEAD 64-block steps before its end at which a chain kernel lets its
- *                           dependent launch (default 8; >= nb/64: at its start)
+ *                           dependent launch (-1 default: nb/128, at least 2; >= nb/64: at its
+ *                           start)
  *   "debug_skip" STF_DEBUG_SKIP bit mask (or names potrf,trsm,syrk,gemm,copy,trsm_as_gemm,
  *                           trsm_as_half_gemm) of task kinds NOT launched: timing what-ifs only,
  *                           results invalid

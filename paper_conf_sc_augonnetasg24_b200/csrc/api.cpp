@@ -72,7 +72,7 @@ const std::vector<OptDesc>& option_table() {
       {"host_eager", "STF_HOST_EAGER", &Options::host_eager, 0, 1, true},
       {"stream_pool", "STF_STREAM_POOL", &Options::stream_pool, 0, 2, true},
       {"pdl", "STF_PDL", &Options::pdl, 0, 1, true},
-      {"pdl_lead", "STF_PDL_LEAD", &Options::pdl_lead, 0, 1024, true},
+      {"pdl_lead", "STF_PDL_LEAD", &Options::pdl_lead, -1, 1024, true},
       {"potrf_split", "STF_POTRF_SPLIT", &Options::potrf_split, 0, 1, true},
       {"potrf_ctas", "STF_POTRF_CTAS", &Options::potrf_ctas, 0, 1024, true},
       {"debug_skip", "STF_DEBUG_SKIP", &Options::debug_skip, 0, INT64_MAX, true},

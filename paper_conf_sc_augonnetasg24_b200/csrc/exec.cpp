@@ -201,6 +201,11 @@ int capture_drop_dependency(cudaStream_t s, cudaGraphNode_t from) {
   return 0;
 }
 
+// 64-block steps before its end at which a chain kernel releases its dependent (option
+// pdl_lead; -1: nb / 128, at least 2 -- the chain step alone: lead 8 best at nb = 1024,
+// 4 at nb = 512, profiles/r02/pdl_and_tail.txt)
+int64_t pdl_lead_of(int64_t opt, int64_t nb) { return opt >= 0 ? opt : std::max<int64_t>(2, nb / 128); }
+
 // ------------------------------------------------------------------ lowering
 namespace {
 
@@ -260,7 +265,7 @@ struct Lowerer {
           stfk::Mirrors mir = mirrors_of(t);  // fused push of L_kk (NEXT-3): final blocks also into the replicas
           // pdl: the chain CTA releases the dependent TRSM(k+1,k) pdl_lead 64-block steps before its end
           const int nbk = (int)((nb + 63) / 64);
-          const int trig = X.opt.pdl ? (int)std::max<int64_t>(0, nbk - X.opt.pdl_lead) : -1;
+          const int trig = X.opt.pdl ? (int)std::max<int64_t>(0, nbk - pdl_lead_of(X.opt.pdl_lead, nb)) : -1;
           cudaGraphNode_t chain = nullptr;
           CUDA_TRY(stfk::potrf_tile(s, prio, (int)nb, X.buf[(size_t)t.out], nb, (int64_t)t.k * nb, S.d_info, ws, &mir,
                                     nullptr, (int)X.opt.potrf_ctas, trig, &chain, (int)X.opt.potrf_split),
@@ -311,7 +316,7 @@ struct Lowerer {
           }
           // column-block counters for a SYRK(k+1,k) that overlaps this TRSM in turn
           int* kflag = pflag ? X.task_ws[(size_t)src] + 2 + nbk * nbk : nullptr;
-          const int trig = kflag ? std::max(0, nbk - (int)X.opt.pdl_lead) : -1;
+          const int trig = kflag ? std::max(0, nbk - (int)pdl_lead_of(X.opt.pdl_lead, nb)) : -1;
           CUDA_TRY(stfk::trsm_res(s, prio, (int)nb, (int)nb, X.buf[(size_t)t.in[0]], nb, X.buf[(size_t)t.out], nb, &mir,
                                   nullptr, pflag, nbk, kflag, trig),
                    "TRSM launch");

@@ -160,7 +160,7 @@ static int bench_chain(int64_t M, int reps, double* avg_ms) {
     cudaGraphNode_t extra = capture_last_node(s);  // debug: an extra full dependency of the TRSM
     step(cudaEventRecordWithFlags(e0, s, cudaEventRecordExternal));
     const int nbk = (int)(M / 64);
-    const int trig = pdl ? (int)std::max<int64_t>(0, nbk - o.pdl_lead) : -1;
+    const int trig = pdl ? (int)std::max<int64_t>(0, nbk - pdl_lead_of(o.pdl_lead, M)) : -1;
     cudaGraphNode_t chain = nullptr;
     step(stfk::potrf_tile(s, 0, (int)M, A, M, 0, info, ws, nullptr, nullptr, (int)o.potrf_ctas, trig, &chain,
                           (int)o.potrf_split));

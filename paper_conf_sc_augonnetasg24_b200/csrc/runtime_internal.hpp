@@ -86,7 +86,7 @@ struct Options {
   int64_t pdl = 1;             // programmatic dependent launch: TRSM(k+1,k) overlaps POTRF(k) (graph backend)
   int64_t potrf_split = 1;     // POTRF tile as two launches (chain + few block tasks, then 2-per-SM block tasks)
   int64_t potrf_ctas = 0;      // CTAs of a POTRF tile launch (0: 3 per 64-block column, 16..96)
-  int64_t pdl_lead = 8;        // pdl: the POTRF lets its TRSM start this many 64-block steps before its end
+  int64_t pdl_lead = -1;       // pdl: the POTRF lets its TRSM start this many 64-block steps before its end (-1: nb / 128)
   int64_t debug_skip = 0;      // bit mask of task kinds not launched (timing what-ifs; results invalid)
   int64_t debug_trace = 0;     // timing events around every task (one slot)
   int64_t nvtx = 0;            // NVTX range per task submission (eager backend; the graph launch is one range)
@@ -138,6 +138,7 @@ constexpr size_t kCacheMax = 4;
 cudaGraphNode_t capture_last_node(cudaStream_t s);
 int capture_make_programmatic(cudaStream_t s, cudaGraphNode_t from);
 int capture_drop_dependency(cudaStream_t s, cudaGraphNode_t from);
+int64_t pdl_lead_of(int64_t opt, int64_t nb);
 
 struct Exec {
   // key

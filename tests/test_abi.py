@@ -91,7 +91,7 @@ OPTIONS = {"graph": (1, 0), "dataflow": (1, 0), "trsm": (3, 1), "streams": (32, 
            "trsm_res_tail": (-1, 0), "trsm_rows": (128, 64), "trsm_res_split": (2, 1), "stream_pool": (0, 1),
            "order_mode": (-1, 2), "order_tail": (-1, 0), "order_asap": (0, 1), "sched_width": (0, 3), "prio_mode": (0, 2),
            "ooc_reorder": (1, 0), "dev_order": (0, 1), "ooc_budget_pct": (-1, 40), "host_stream_budget_pct": (90, 75),
-           "host_eager": (0, 1), "mem_cap_tiles": (0, 10), "ooc_order": (-1, 0), "host_stream": (1, 0), "pdl": (1, 0), "pdl_lead": (8, 16), "potrf_split": (1, 0), "potrf_ctas": (0, 24),
+           "host_eager": (0, 1), "mem_cap_tiles": (0, 10), "ooc_order": (-1, 0), "host_stream": (1, 0), "pdl": (1, 0), "pdl_lead": (-1, 16), "potrf_split": (1, 0), "potrf_ctas": (0, 24),
            "debug_skip": (0, 8), "debug_trace": (0, 1), "nvtx": (0, 1), "gemm_merge": (2, 0), "gemm_group": (-1, 4)}
 
 

@@ -69,7 +69,7 @@ def _reset_options(request):
         s = request.getfixturevalue("stf")
         _options(s, graph=1, serial=0, priority=1, streams=32, grid_p=0, dataflow=1, trsm=3, threads=8, lookahead=1, trsm_split=4, push=0,
                  trsm_rows=128, stream_pool=0, prio_mode=0, order_mode=-1, dev_order=0, order_asap=0, host_eager=0,
-                 pdl=1, pdl_lead=8, trsm_res_split=2)
+                 pdl=1, pdl_lead=-1, trsm_res_split=2)
 
 
 def _factor_spd(stf, n, nb, p=1, q=1, seed=1):
